@@ -1,0 +1,259 @@
+/*
+ * abacus.h -- C ABI of the B200-native Abacus candidate-search library
+ * (libabacus.so, built from paper_conf_sc_cui0czlzsmylg21_b200/csrc).
+ *
+ * What it computes: the data-parallel hot path of Abacus's headroom-based
+ * query controller (Cui et al., "Enable Simultaneous DNN Services Based on
+ * Deterministic Operator Overlap and Precise Latency Prediction", SC'21).
+ * Citations are P:<line> into the paper text plus the section /
+ * equation / figure; "reading cN" refers to DESIGN.md "Readings of the paper".
+ *
+ *   a1 headroom + order      Eq. 2, Eq. 3, sort
+ *   a2 candidate enumeration operator groups
+ *   a3 feature encoding      Fig. 8
+ *   a4 predictor forward     MLP, 3 hidden layers of 32
+ *   a5 mask + selection      largest group under the tightest headroom
+ *   a6 cross-GPU combine     one NCCL collective (no counterpart in the paper)
+ *   a7 decision assembly     drop mechanism
+ *
+ * Conventions (all entry points)
+ *   - Return value: ABACUS_OK (0) or a negative ABACUS_E_* code.  On error no
+ *     output is written and abacus_last_error(ctx) returns a message.  The
+ *     decision OUTCOME is the separate field abacus_decision_t.status.
+ *   - Ownership: the caller owns every buffer it passes.  Host structs are
+ *     read during the call and never retained.  Device pointers must be
+ *     allocations on the ctx's device.  The ctx owns its weight copies and a
+ *     fixed scratch area allocated in abacus_create / abacus_load_predictor;
+ *     no entry point allocates device memory on the hot path.
+ *   - Streams: encode / predict / select are asynchronous on the given CUDA
+ *     stream (NULL = the ctx's own stream).  abacus_search and
+ *     abacus_search_grid block until the decision is in host memory.
+ *   - Thread safety: none; use one ctx per host thread.
+ *   - There is no CPU fallback: abacus_create fails with ABACUS_E_DEVICE on
+ *     anything but an sm_100 device.
+ *
+ * Notation: N models (ids 1..N, Table 1 order, reading c6), L_m ops of model m
+ * (1-based, inclusive ranges, reading c7), k co-located queries, K_MAX = 4,
+ * D = N + 4*K_MAX feature width.
+ */
+#ifndef ABACUS_H
+#define ABACUS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ABACUS_K_MAX 4
+#define ABACUS_HIDDEN 32
+#define ABACUS_ABI_VERSION 1
+
+/* status codes */
+enum {
+    ABACUS_OK = 0,
+    ABACUS_E_INVALID = -1,    /* bad argument (ranges, sizes, null pointers)        */
+    ABACUS_E_DUP_MODEL = -2,  /* two queries/slots of one model (reading c9)        */
+    ABACUS_E_NOT_LOADED = -3, /* no predictor loaded for the requested precision    */
+    ABACUS_E_CUDA = -4,       /* CUDA runtime error                                 */
+    ABACUS_E_NCCL = -5,       /* NCCL error                                         */
+    ABACUS_E_DEVICE = -6      /* device is not sm_100 (no fallback exists)          */
+};
+
+/* predictor arithmetic (reading c16) */
+enum {
+    ABACUS_FP32 = 0, /* SIMT FFMA, fp32 weights and activations                     */
+    ABACUS_BF16 = 1, /* tcgen05 kind::f16, bf16 operands (weights split hi+lo),     */
+                     /* fp32 accumulation in TMEM                                   */
+    ABACUS_FP16 = 2  /* tcgen05 kind::f16, fp16 operands with exact power-of-two    */
+                     /* layer scaling, fp32 accumulation in TMEM                    */
+};
+
+/* candidate space of abacus_search (reading c13) */
+enum {
+    ABACUS_SPACE_GRID = 0,  /* every end-op combination (exhaustive)                */
+    ABACUS_SPACE_CHAIN = 1, /* the paper's chain: prefix of full queries, then one  */
+                            /* partial query                          */
+    ABACUS_SPACE_AUTO = 2   /* GRID if |GRID| <= grid_budget, else CHAIN            */
+};
+
+/* decision outcome */
+enum {
+    ABACUS_DECIDE_OK = 0,   /* end_op[] holds the group                             */
+    ABACUS_DECIDE_DROP = 1, /* the critical query alone exceeds H: drop it          */
+                            /* (reading c14)                           */
+    ABACUS_DECIDE_NONE = 2  /* sweep only: no candidate fits under H                */
+};
+
+typedef struct abacus_ctx abacus_ctx; /* opaque; one per device per host thread */
+
+/* One service of a candidate grid.  Digit d of the slot: allow_absent ?
+ * (d == 0 -> absent, else ope = end_lo + d - 1) : ope = end_lo + d; radix
+ * rho = allow_absent + end_hi - end_lo + 1.  seqlen is 0 for non-Bert models
+ * (reading c8). */
+typedef struct {
+    int32_t model_id;     /* 1..N                                          */
+    int32_t start_op;     /* ops: first op of the range, 1-based           */
+    int32_t batch;        /* bs >= 1                                       */
+    int32_t seqlen;       /* >= 0                                          */
+    int32_t end_lo, end_hi; /* candidate ope range, start_op <= lo <= hi <= L */
+    int32_t allow_absent; /* 0 or 1                                        */
+} abacus_slot_t;
+
+/* A candidate grid: slots in priority (headroom) order.  Candidate index
+ * t in [0, T), T = prod rho_j < 2^40, mixed radix with the LAST slot fastest. */
+typedef struct {
+    int32_t k;
+    abacus_slot_t slot[ABACUS_K_MAX];
+} abacus_grid_t;
+
+/* An explicit operator group (one row of config-5 instance samples). */
+typedef struct {
+    int32_t k;                       /* present models, 0..K_MAX            */
+    struct {
+        int32_t model_id, ops, ope, batch, seqlen;
+    } slot[ABACUS_K_MAX];            /* any order; encoded by model id       */
+} abacus_group_t;
+
+/* One active query (Fig. 4, Eq. 2). */
+typedef struct {
+    int32_t model_id; /* 1..N                                  */
+    int32_t next_op;  /* s: first op not yet run, 1..L         */
+    int32_t batch;
+    int32_t seqlen;
+    double qos_ms;     /* T_QoS                                 */
+    double t_start_ms; /* T_start                               */
+} abacus_query_t;
+
+typedef struct {
+    int32_t status;     /* ABACUS_DECIDE_*                                         */
+    int32_t critical;   /* index into the caller's query array (sweeps: 0)         */
+    int32_t order[4];   /* headroom order as caller indices (sweeps: identity)     */
+    int32_t end_op[4];  /* per caller query / grid slot: ope, 0 = not in the group */
+    uint64_t key;       /* ((sum_n + 1) << 40) | index, 0 = nothing fits           */
+    uint64_t index;     /* t* (GRID / sweep) or u* (CHAIN)                         */
+    uint64_t evaluated; /* candidates evaluated (sweep: over all ranks)            */
+    int32_t total_ops;  /* sum over the group of (ope - ops + 1)                   */
+    float headroom_ms;  /* H, the fp32 threshold compared against                  */
+    float pred_ms;      /* predicted latency of the chosen group (feeds Eq. 3)     */
+    float pred_critical_only_ms; /* y of the critical query alone (drop test)     */
+} abacus_decision_t;
+
+/* ------------------------------------------------------------------------ */
+/* Context                                                                   */
+/* ------------------------------------------------------------------------ */
+
+/* Create a ctx on CUDA device `device` for a registry of n_models models with
+ * ops_per_model[m-1] = L_m (host array, copied).  k_max must be 4.
+ * Errors: E_INVALID (n_models < 1 or > 64, L_m < 1 or > 32767, k_max != 4),
+ * E_DEVICE (not sm_100), E_CUDA.  *out is written only on success. */
+int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, int32_t k_max,
+                  abacus_ctx** out);
+
+/* Free the ctx and everything it owns (NULL is a no-op). */
+void abacus_destroy(abacus_ctx* ctx);
+
+/* Last error message of this ctx ("" if none); valid until the next call. */
+const char* abacus_last_error(const abacus_ctx* ctx);
+
+/* Load predictor weights (host, fp32, little endian), row-major [out][in]:
+ *   W1[32][D] b1[32] W2[32][32] b2[32] W3[32][32] b3[32] w4[32] b4
+ * n_params must be 32*D + 2*32*32 + 4*32 + 1 (2945 for D = 24).
+ * `precision` selects the arithmetic later calls use (ABACUS_FP32/BF16/FP16);
+ * the fp32 copy is always kept.  The ctx converts once at load time (RNE) and
+ * owns the device copies.  Errors: E_INVALID (size / precision / non-finite). */
+int abacus_load_predictor(abacus_ctx* ctx, const float* params, size_t n_params, int precision);
+
+/* ------------------------------------------------------------------------ */
+/* Building blocks (asynchronous on `stream`)                                */
+/* ------------------------------------------------------------------------ */
+
+/* a2 + a3: encode candidates t in [first, first+count) of `grid` (host struct)
+ * into d_features (device, int16, count x D row-major, 16-byte aligned) per
+ * Fig. 8: x[m-1] = 1 per present model; present models in
+ * ascending id fill x[N+4p .. N+4p+3] = (ops, ope, bs, seqlen); zeros
+ * elsewhere.  Errors: E_INVALID (grid validation as in abacus_search_grid,
+ * first + count > T), E_DUP_MODEL. */
+int abacus_encode_candidates(abacus_ctx* ctx, const abacus_grid_t* grid, uint64_t first, uint64_t count,
+                             int16_t* d_features, void* stream);
+
+/* a3 for explicit groups: d_groups (device, count records) -> d_features
+ * (device, count x D).  A group with an invalid or duplicate model id is
+ * encoded as all zeros and counted in *d_bad (device uint32, accumulated;
+ * may be NULL). */
+int abacus_encode_groups(abacus_ctx* ctx, const abacus_group_t* d_groups, uint64_t count,
+                         int16_t* d_features, uint32_t* d_bad, void* stream);
+
+/* a4: y = MLP(x) for count feature rows (device int16, count x D) into
+ * d_latency_ms (device fp32, count), with the loaded precision.
+ * Errors: E_NOT_LOADED, E_INVALID. */
+int abacus_predict_batch(abacus_ctx* ctx, const int16_t* d_features, uint64_t count, float* d_latency_ms,
+                         void* stream);
+
+/* a5: fold candidates t in [first, first+count) of `grid` with predicted
+ * latencies d_latency_ms[t - first] into the running max key *d_best_key
+ * (device, in/out, initialise to 0): key(t) = ((sum_n + 1) << 40) | t over
+ * y(t) <= headroom_ms (inclusive, readings c11/c12). */
+int abacus_select_group(abacus_ctx* ctx, const abacus_grid_t* grid, uint64_t first, uint64_t count,
+                        const float* d_latency_ms, float headroom_ms, unsigned long long* d_best_key,
+                        void* stream);
+
+/* ------------------------------------------------------------------------ */
+/* Fused search (blocking)                                                   */
+/* ------------------------------------------------------------------------ */
+
+/* a1..a7 for one scheduling round (P:630-753 steps 1-2, §6.2-6.3):
+ * h_i = qos_i - (now_ms - t_start_i) - inflight_pred_ms (Eq. 2 + Eq. 3, c15);
+ * order ascending by (h, model id) (c10); H = (float)h_critical; critical
+ * query fully included; other queries contribute ope in
+ * [next_op, L] or are absent; candidate space per `space` / grid_budget;
+ * result = largest feasible group (max sum_n, ties to lower-headroom queries,
+ * c12); DROP iff y(critical alone) > H (c14).  q: host array of k queries
+ * (1 <= k <= 4).  out: host.  Errors: E_INVALID, E_DUP_MODEL, E_NOT_LOADED,
+ * E_CUDA. */
+int abacus_search(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                  int32_t space, uint64_t grid_budget, abacus_decision_t* out);
+
+/* a2..a6 over a sweep grid: candidates t in [first, first+count) of `grid`
+ * (host) under `headroom_ms`; this rank's shard.  With nccl_comm != NULL
+ * (an ncclComm_t on this device, e.g. from abacus_nccl_comm_init) the
+ * per-rank results are combined with one collective so every rank returns
+ * the same global decision (status OK or NONE, end_op per slot, pred_ms of
+ * t*, evaluated summed over ranks).  Validation: 1 <= k <= 4, model ids in
+ * [1, N] and distinct, 1 <= start_op <= end_lo <= end_hi <= L, batch >= 1,
+ * seqlen >= 0, T < 2^40, max sum_n + 1 < 2^24.  Errors: E_INVALID,
+ * E_DUP_MODEL, E_NOT_LOADED, E_CUDA, E_NCCL. */
+int abacus_search_grid(abacus_ctx* ctx, const abacus_grid_t* grid, float headroom_ms, uint64_t first,
+                       uint64_t count, void* nccl_comm, abacus_decision_t* out);
+
+/* ------------------------------------------------------------------------ */
+/* NCCL bootstrap helpers (multi-GPU sweeps; one process per GPU)            */
+/* ------------------------------------------------------------------------ */
+
+/* 128-byte ncclUniqueId into `id128` (host).  Call on one rank, broadcast the
+ * bytes (e.g. with torch.distributed), then abacus_nccl_comm_init on all. */
+int abacus_nccl_unique_id(uint8_t* id128);
+/* Create an ncclComm_t for (nranks, rank) on the ctx's device; *comm_out
+ * receives it (owned by the caller; free with abacus_nccl_comm_destroy). */
+int abacus_nccl_comm_init(abacus_ctx* ctx, int32_t nranks, int32_t rank, const uint8_t* id128,
+                          void** comm_out);
+void abacus_nccl_comm_destroy(void* comm);
+
+/* ------------------------------------------------------------------------ */
+/* Introspection                                                             */
+/* ------------------------------------------------------------------------ */
+
+/* Number of device kernels the library launched on this ctx since creation
+ * (used by bench.py for "gpu_launches"). */
+uint64_t abacus_kernel_launches(const abacus_ctx* ctx);
+/* Device time (ms, CUDA events on the launching stream) of the last fused
+ * search kernel launch of this ctx; -1 if none. */
+float abacus_last_kernel_ms(const abacus_ctx* ctx);
+/* ABI version (ABACUS_ABI_VERSION). */
+int abacus_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ABACUS_H */
