@@ -1,0 +1,291 @@
+"""bench.py -- headline benchmark of the Abacus candidate-search hot path on B200.
+
+Step = one abacus_search_grid over config 4 of BASELINE.json: the offline
+exhaustive overlap sweep of ResNet-152 (bs 8), Inception-v3 (bs 8), BERT-base
+(bs 8, seq 128) and BERT-large (bs 4, seq 512), 361*221*244*472 =
+9,188,218,208 candidates (enumerate -> Fig.-8 encode -> MLP -> headroom mask ->
+max key), sharded contiguously over the ranks with one NCCL all-gather of the
+per-rank best (a6).  Metric: predictor candidates/s (whole job).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--precision fp16|bf16|fp32]
+  python bench.py --impl reference ...   # the fp64 CPU oracle on a bounded sample
+
+Inputs are synthetic (seeded weights of the paper's MLP shape, synth/); the
+candidate space is generated on the fly inside the kernel, so there is no
+input tensor to keep out of L2 -- the timed kernel reads only its ~20 KB of
+weights and writes 48 bytes (config "l2": "no per-candidate memory traffic").
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+FLOP_PER_CAND = 2 * (synth.D * 32 + 32 * 32 + 32 * 32 + 32)  # 5,696 algorithmic FLOP (D = 24)
+METRIC = "predictor candidates/sec (config 4 exhaustive overlap sweep, abacus_search_grid)"
+PREC = {"fp32": 0, "bf16": 1, "fp16": 2}
+DTYPE = {"fp32": "f32", "bf16": "bf16 (weights hi+lo), f32 accum", "fp16": "f16, f32 accum"}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured (MEASURED_PEAKS.json)"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback (B200_PROFILING.md)"
+
+
+class Clocks:
+    """nvidia-smi sampler during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + q,
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([v.strip() for v in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 2 + i and "Active" in r[2 + i]
+                          and "Not" not in r[2 + i]})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def cpu_oracle_rate(params, slots, H, budget_s=12.0, chunk=100_000):
+    """The fp64 oracle as it stands, 1 thread, on a contiguous sample of the
+    config-4 grid starting at T/2 (all four services mostly present)."""
+    import oracle
+    T = oracle.grid_size(slots)
+    first = T // 2
+    n = 0
+    t0 = time.perf_counter()
+    while time.perf_counter() - t0 < budget_s:
+        oracle.sweep(params, slots, H, first=first + n, count=chunk)
+        n += chunk
+    dt = time.perf_counter() - t0
+    return n / dt, n, dt
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    import oracle
+    params = synth.weights(1)
+    slots = synth.cfg4_grid()
+    H = synth.cfg4_headroom()
+    T = oracle.grid_size(slots)
+    per_step = 60_000
+    for i in range(args.warmup):
+        oracle.sweep(params, slots, H, first=T // 2 + i * per_step, count=per_step)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        oracle.sweep(params, slots, H, first=T // 2 + (args.warmup + i) * per_step, count=per_step)
+    dt = time.perf_counter() - t0
+    rate = per_step * args.steps / dt
+    line = {"impl": "reference", "metric": METRIC, "value": rate, "unit": "candidates/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": "cfg4 sweep (sample of %d candidates/step from T/2)"
+                                                        % per_step, "candidates_total": T},
+            "cpu_baseline": {"value": rate, "unit": "candidates/s", "cores": 1, "kind": "oracle",
+                             "sample": "%d contiguous config-4 candidates per step from index T/2" % per_step},
+            "e2e": {"value": rate, "unit": "candidates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--precision", default="fp16", choices=list(PREC))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-decisions", action="store_true")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_cui0czlzsmylg21_b200 as ab
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    params = synth.weights(1)
+    slots = synth.cfg4_grid()
+    H = synth.cfg4_headroom()
+    grid = ab.make_grid(slots)
+    T = 1
+    for s in slots:
+        T *= s.allow_absent + s.end_hi - s.end_lo + 1
+    first, count = ab.shard_range(T, rank, world)
+
+    ctx = ab.abacus_create(local, list(synth.OPS_PER_MODEL))
+    ab.abacus_load_predictor(ctx, params, PREC[args.precision])
+    stream = torch.cuda.current_stream()
+    ab.abacus_set_stream(ctx, stream)
+    ab.abacus_set_timing(ctx, True)
+    comm = ab.nccl_comm_from_process_group(ctx) if world > 1 else None
+
+    for _ in range(args.warmup):
+        d = ab.abacus_search_grid(ctx, grid, H, first, count, comm)
+    # ---- device-timed region ------------------------------------------------
+    launches0 = ab.abacus_kernel_launches(ctx)
+    kernel_ms = []
+    with Clocks(local) as clk:
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            d = ab.abacus_search_grid(ctx, grid, H, first, count, comm)
+            kernel_ms.append(ab.abacus_last_kernel_ms(ctx))
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    launches = ab.abacus_kernel_launches(ctx) - launches0
+    elapsed = e0.elapsed_time(e1) / 1e3
+    t = torch.tensor([elapsed, float(np.mean(kernel_ms))], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    elapsed, kms = float(t[0]), float(t[1])
+
+    # ---- end to end through the public API (host structs in, host decision out) ----
+    e2e_steps = max(2, args.steps // 2)
+    if world > 1:
+        dist.barrier()
+    w0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        d = ab.abacus_search_grid(ctx, grid, H, first, count, comm)
+    w1 = time.perf_counter()
+    te = torch.tensor([w1 - w0], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_rate = T * e2e_steps / float(te[0])
+
+    # ---- per-decision latency (config 2, 3-way; 1 GPU each) -----------------
+    dec = None
+    if rank == 0 and not args.no_decisions:
+        dec = decision_latency(ab, ctx)
+
+    if rank == 0:
+        pk, src = peaks()
+        peak = pk["bf16_tflops_sustained"]  # fp16 dense = bf16 dense on B200; kernel runs back to back
+        achieved = FLOP_PER_CAND * count / (kms / 1e3) / 1e12
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tp):
+            with open(tp) as f:
+                traffic = json.load(f).get("fused_" + args.precision)
+        cpu = None
+        if not args.no_cpu_baseline:
+            rate, n, dt = cpu_oracle_rate(params, slots, H)
+            cpu = {"value": rate, "unit": "candidates/s", "cores": 1, "kind": "oracle",
+                   "sample": "%d contiguous config-4 candidates from index T/2 (%.1f s, 1 thread)" % (n, dt)}
+        value = T * args.steps / elapsed
+        line = {
+            "metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": elapsed / args.steps * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[args.precision], "data": "synthetic",
+            "config": {"workload": "cfg4: 4-way exhaustive overlap sweep (ResNet-152, Inception-v3, BERT-base "
+                                   "seq128, BERT-large seq512), %d candidates" % T,
+                       "candidates_per_step": T, "headroom_ms": H, "precision": args.precision,
+                       "parallelism": "candidate shards x%d, NCCL all-gather of the best key" % world,
+                       "l2": "no per-candidate memory traffic (candidates generated on chip)"},
+            "per_gpu": value / world,
+            "selected": {"key": d.key, "index": d.index, "total_ops": d.total_ops, "pred_ms": d.pred_ms,
+                         "end_op": list(d.end_op)},
+            "roofline": {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "fused_tc_kernel" if args.precision != "fp32" else "fused_fp32_kernel",
+                         "kernel_ms": kms, "flop_per_candidate": FLOP_PER_CAND, "peak_source": src + ", sustained"},
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_rate, "unit": "candidates/s", "h2d_bytes_per_step": 120,
+                    "d2h_bytes_per_step": 48},
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "decision_latency": dec,
+        }
+        print(json.dumps(line))
+    if comm:
+        ab.abacus_nccl_comm_destroy(comm)
+    ab.abacus_destroy(ctx)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def decision_latency(ab, ctx, n=10_000, warm=100):
+    """Host wall clock around each blocking abacus_search (launch + kernel +
+    decision in host memory), config 2 (3-way), GRID space."""
+    decs = synth.cfg2_decisions(n + warm)
+    lat = []
+    sizes = []
+    for i, (qs, now, infl) in enumerate(decs):
+        t0 = time.perf_counter()
+        d = ab.abacus_search(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID)
+        t1 = time.perf_counter()
+        if i >= warm:
+            lat.append((t1 - t0) * 1e6)
+            sizes.append(d.evaluated)
+    a = np.array(lat)
+    return {"workload": "cfg2 3-way (ResNet-101, Inception-v3, BERT-base), GRID", "decisions": n,
+            "p50_us": float(np.percentile(a, 50)), "p99_us": float(np.percentile(a, 99)),
+            "p999_us": float(np.percentile(a, 99.9)), "grid_p50": float(np.percentile(sizes, 50)),
+            "grid_max": int(max(sizes))}
+
+
+if __name__ == "__main__":
+    main()

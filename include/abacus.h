@@ -250,6 +250,12 @@ uint64_t abacus_kernel_launches(const abacus_ctx* ctx);
 /* Device time (ms, CUDA events on the launching stream) of the last fused
  * search kernel launch of this ctx; -1 if none. */
 float abacus_last_kernel_ms(const abacus_ctx* ctx);
+/* Use `stream` (a cudaStream_t on the ctx's device; NULL = the ctx's own
+ * stream) for the blocking calls and as the default of the async ones. */
+int abacus_set_stream(abacus_ctx* ctx, void* stream);
+/* Enable (on != 0) CUDA-event timing of the fused search kernel on the ctx
+ * stream, read back with abacus_last_kernel_ms. */
+int abacus_set_timing(abacus_ctx* ctx, int on);
 /* ABI version (ABACUS_ABI_VERSION). */
 int abacus_abi_version(void);
 

@@ -1,0 +1,833 @@
+// abacus.cu -- host side of the C ABI declared in include/abacus.h.
+//
+// Responsibilities: argument validation, the per-call launch plan (segments
+// of the candidate space, see common.cuh), the a1 headroom/order step of a
+// decision (Eq. 2 + Eq. 3, P:1170-1182 / P:1366-1376, on the host like the
+// paper's controller), weight preparation at load time, kernel launches,
+// the NCCL combine of sharded sweeps, and reading back the decision.
+// Every step of a2..a7 runs in the kernels (kernels_simt.cu, kernels_tc.cu).
+#include <cuda_fp16.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/abacus.h"
+#include "common.cuh"
+#include "internal.h"
+#include "tc_ptx.cuh"
+
+using namespace abacus;
+
+struct abacus_ctx {
+    int device = 0;
+    int nsm = 0;
+    int32_t n_models = 0, D = 0;
+    std::vector<int32_t> L;
+    cudaStream_t stream = nullptr;      // stream of the blocking calls (default: own_stream)
+    cudaStream_t own_stream = nullptr;
+    Scratch* S = nullptr;         // device
+    Result* host_result = nullptr;  // pinned
+    std::string err;
+    uint64_t launches = 0;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    bool timed = false;
+    // predictor
+    bool loaded = false;
+    int precision = ABACUS_FP32;
+    std::vector<float> params;    // host fp32 copy
+    float* d_w1b1 = nullptr;      // device W1[32][D] + b1[32]
+    W234 w234{};
+    uint8_t* d_blob[2] = {nullptr, nullptr};  // tensor-core weight blobs (fp16, bf16)
+    TcWeights tw[2]{};
+};
+
+namespace {
+
+int fail(abacus_ctx* c, int code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    return code;
+}
+
+
+// ---- NCCL, resolved at run time -------------------------------------------
+// The library does not link libnccl: a process that already loaded NCCL
+// (e.g. through torch.distributed) must keep using that copy, so the symbols
+// are looked up with dlopen(RTLD_NOLOAD) first and only then loaded.
+struct NcclApi {
+    bool ok = false;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
+    ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+const NcclApi& nccl() {
+    static NcclApi api;
+    static bool tried = false;
+    if (tried) return api;
+    tried = true;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return api;
+    api.GetUniqueId = (decltype(api.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    api.CommInitRank = (decltype(api.CommInitRank))dlsym(h, "ncclCommInitRank");
+    api.CommDestroy = (decltype(api.CommDestroy))dlsym(h, "ncclCommDestroy");
+    api.CommCount = (decltype(api.CommCount))dlsym(h, "ncclCommCount");
+    api.AllGather = (decltype(api.AllGather))dlsym(h, "ncclAllGather");
+    api.GetErrorString = (decltype(api.GetErrorString))dlsym(h, "ncclGetErrorString");
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.CommCount && api.AllGather &&
+             api.GetErrorString;
+    return api;
+}
+
+#define CUDA_TRY(ctx, call)                                                                         \
+    do {                                                                                            \
+        cudaError_t e__ = (call);                                                                   \
+        if (e__ != cudaSuccess) return fail(ctx, ABACUS_E_CUDA, "%s: %s", #call, cudaGetErrorString(e__)); \
+    } while (0)
+
+FastDiv make_fastdiv(uint32_t d) {
+    FastDiv f{};
+    f.d = d;
+    uint32_t p = 0;
+    while ((1ull << p) < d) p++;
+    f.shift = p;
+    f.mul = (uint32_t)(((1ull << 32) * ((1ull << p) - d)) / d + 1);
+    return f;
+}
+
+// ---- validation -----------------------------------------------------------
+int validate_grid(abacus_ctx* c, const abacus_grid_t* g, uint64_t* T_out) {
+    if (!g) return fail(c, ABACUS_E_INVALID, "grid is NULL");
+    if (g->k < 1 || g->k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", g->k);
+    uint64_t T = 1;
+    int64_t max_sum_n = 0;
+    for (int j = 0; j < g->k; j++) {
+        const abacus_slot_t& s = g->slot[j];
+        if (s.model_id < 1 || s.model_id > c->n_models)
+            return fail(c, ABACUS_E_INVALID, "slot %d: model_id %d outside [1,%d]", j, s.model_id, c->n_models);
+        for (int i = 0; i < j; i++)
+            if (g->slot[i].model_id == s.model_id)
+                return fail(c, ABACUS_E_DUP_MODEL, "slots %d and %d share model %d", i, j, s.model_id);
+        const int32_t L = c->L[s.model_id - 1];
+        if (s.start_op < 1 || s.start_op > s.end_lo || s.end_lo > s.end_hi || s.end_hi > L)
+            return fail(c, ABACUS_E_INVALID, "slot %d: need 1 <= start_op <= end_lo <= end_hi <= L=%d", j, L);
+        if (s.batch < 1 || s.batch > 32767) return fail(c, ABACUS_E_INVALID, "slot %d: batch %d", j, s.batch);
+        if (s.seqlen < 0 || s.seqlen > 32767) return fail(c, ABACUS_E_INVALID, "slot %d: seqlen %d", j, s.seqlen);
+        if (s.allow_absent != 0 && s.allow_absent != 1)
+            return fail(c, ABACUS_E_INVALID, "slot %d: allow_absent must be 0/1", j);
+        const uint64_t rho = (uint64_t)s.allow_absent + (uint64_t)(s.end_hi - s.end_lo + 1);
+        T *= rho;
+        if (T >= (1ull << 40)) return fail(c, ABACUS_E_INVALID, "grid size >= 2^40");
+        max_sum_n += s.end_hi - s.start_op + 1;
+    }
+    if (max_sum_n + 1 >= (1ll << 24)) return fail(c, ABACUS_E_INVALID, "sum_n + 1 >= 2^24");
+    *T_out = T;
+    return ABACUS_OK;
+}
+
+// ---- plans ------------------------------------------------------------------
+void fill_slots(Plan& P, const abacus_grid_t* g) {
+    for (int j = 0; j < kKMax; j++) {
+        SlotP& s = P.slot[j];
+        if (j < g->k) {
+            const abacus_slot_t& a = g->slot[j];
+            s = SlotP{a.model_id, a.start_op, a.batch, a.seqlen, a.end_lo, a.end_hi, a.allow_absent,
+                      a.allow_absent + a.end_hi - a.end_lo + 1};
+        } else {
+            s = SlotP{0, 0, 0, 0, 0, 0, 0, 1};
+        }
+    }
+}
+
+void finish_box(SegP& s) {
+    uint64_t b = 1;
+    for (int j = kKMax - 1; j >= 0; j--) {
+        s.bstride[j] = b;
+        s.rbstride[j] = 1.0 / (double)b;
+        s.fd[j] = make_fastdiv(s.cnt[j]);
+        b *= s.cnt[j];
+    }
+}
+
+uint64_t box_size(const SegP& s) {
+    uint64_t b = 1;
+    for (int j = 0; j < kKMax; j++) b *= s.cnt[j];
+    return b;
+}
+
+// whole grid as one box: digits = grid digits (encode / select kernels)
+Plan plan_whole_grid(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T) {
+    Plan P{};
+    P.k = g->k;
+    P.n_models = c->n_models;
+    P.D = c->D;
+    P.mode = kModeGrid;
+    P.T = T;
+    fill_slots(P, g);
+    P.n_seg = 1;
+    SegP& s = P.seg[0];
+    for (int j = 0; j < kKMax; j++) {
+        s.cnt[j] = j < g->k ? (uint32_t)P.slot[j].radix : 1u;
+        s.pos[j] = -1;
+    }
+    finish_box(s);
+    return P;
+}
+
+// number of elements of box `s` (digit sets per slot, see below) with index < a
+uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, uint64_t a) {
+    if (a >= P.T) return box_size(s);
+    uint32_t dig[kKMax] = {0, 0, 0, 0};
+    uint64_t rem = a;
+    for (int j = P.k - 1; j >= 0; j--) {
+        dig[j] = (uint32_t)(rem % (uint64_t)P.slot[j].radix);
+        rem /= (uint64_t)P.slot[j].radix;
+    }
+    uint64_t cnt = 0;
+    for (int j = 0; j < P.k; j++) {
+        const bool present = (s.mask >> j) & 1u;
+        uint64_t below;
+        bool inside;
+        if (present) {
+            const int64_t b = (int64_t)dig[j] - (int64_t)dlo[j];
+            below = (uint64_t)std::min<int64_t>(std::max<int64_t>(b, 0), (int64_t)s.cnt[j]);
+            inside = dig[j] >= dlo[j] && dig[j] < dlo[j] + s.cnt[j];
+        } else {
+            below = dig[j] > 0 ? 1 : 0;
+            inside = dig[j] == 0;
+        }
+        cnt += below * s.bstride[j];
+        if (!inside) return cnt;
+    }
+    return cnt;
+}
+
+void set_positions(const Plan& P, SegP& s) {
+    for (int j = 0; j < kKMax; j++) {
+        s.pos[j] = -1;
+        if (j >= P.k || !((s.mask >> j) & 1u)) continue;
+        int p = 0;
+        for (int i = 0; i < P.k; i++)
+            if (((s.mask >> i) & 1u) && P.slot[i].model_id < P.slot[j].model_id) p++;
+        s.pos[j] = p;
+    }
+}
+
+// GRID / sweep: one segment per presence pattern, restricted to [first, last)
+Plan plan_grid_segments(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T, uint64_t first, uint64_t last,
+                        float H) {
+    Plan P{};
+    P.k = g->k;
+    P.n_models = c->n_models;
+    P.D = c->D;
+    P.mode = kModeGrid;
+    P.T = T;
+    P.H = H;
+    P.want_y0 = first == 0 && last > 0;
+    fill_slots(P, g);
+    uint64_t tstride[kKMax];
+    {
+        uint64_t b = 1;
+        for (int j = kKMax - 1; j >= 0; j--) {
+            tstride[j] = j < g->k ? b : 0;
+            if (j < g->k) b *= (uint64_t)P.slot[j].radix;
+        }
+    }
+    uint64_t tiles = 0, n_eval = 0;
+    for (uint32_t mask = 0; mask < (1u << g->k); mask++) {
+        bool ok = true;
+        for (int j = 0; j < g->k; j++)
+            if (!g->slot[j].allow_absent && !((mask >> j) & 1u)) ok = false;
+        if (!ok) continue;
+        SegP s{};
+        s.mask = mask;
+        uint32_t dlo[kKMax] = {0, 0, 0, 0};
+        s.n_base = 0;
+        s.t_base = 0;
+        for (int j = 0; j < kKMax; j++) {
+            const bool present = j < g->k && ((mask >> j) & 1u);
+            if (present) {
+                const abacus_slot_t& a = g->slot[j];
+                s.cnt[j] = (uint32_t)(a.end_hi - a.end_lo + 1);
+                dlo[j] = a.allow_absent ? 1u : 0u;
+                s.ope0[j] = a.end_lo;
+                s.istride[j] = tstride[j];
+                s.t_base += (uint64_t)dlo[j] * tstride[j];
+                s.n_base += a.end_lo - a.start_op + 1;
+            } else {
+                s.cnt[j] = 1;
+                s.ope0[j] = 0;
+                s.istride[j] = 0;
+            }
+        }
+        finish_box(s);
+        set_positions(P, s);
+        s.u_begin = box_count_lt(P, s, dlo, first);
+        s.u_end = box_count_lt(P, s, dlo, last);
+        if (s.u_end <= s.u_begin) continue;
+        s.tile0 = tiles;
+        tiles += (s.u_end - s.u_begin + kTileM - 1) / kTileM;
+        n_eval += s.u_end - s.u_begin;
+        P.seg[P.n_seg++] = s;
+    }
+    P.n_tiles = tiles;
+    P.n_eval = n_eval;
+    return P;
+}
+
+// CHAIN (decision mode): u = 0 critical only; block j: slots < j full, slot j
+// grows op by op, later slots absent
+Plan plan_chain(const abacus_ctx* c, const abacus_grid_t* g, float H, uint64_t* n_out) {
+    Plan P{};
+    P.k = g->k;
+    P.n_models = c->n_models;
+    P.D = c->D;
+    P.mode = kModeChain;
+    P.H = H;
+    P.want_y0 = 1;
+    fill_slots(P, g);
+    uint64_t cum = 0;
+    uint64_t tiles = 0;
+    for (int j = 0; j < g->k; j++) {
+        SegP s{};
+        s.mask = (2u << j) - 1u;
+        s.n_base = 0;
+        for (int i = 0; i < kKMax; i++) {
+            s.cnt[i] = 1;
+            s.istride[i] = 0;
+            s.ope0[i] = 0;
+        }
+        for (int i = 0; i < j; i++) {
+            s.ope0[i] = g->slot[i].end_hi;
+            s.n_base += g->slot[i].end_hi - g->slot[i].start_op + 1;
+        }
+        if (j == 0) {
+            s.ope0[0] = g->slot[0].end_hi;
+            s.n_base = g->slot[0].end_hi - g->slot[0].start_op + 1;
+        } else {
+            s.cnt[j] = (uint32_t)(g->slot[j].end_hi - g->slot[j].start_op + 1);
+            s.ope0[j] = g->slot[j].start_op;
+            s.istride[j] = 1;
+            s.n_base += 1;
+        }
+        P.chain_cum[j] = cum;
+        s.t_base = cum;
+        finish_box(s);
+        set_positions(P, s);
+        s.u_begin = 0;
+        s.u_end = box_size(s);
+        s.tile0 = tiles;
+        tiles += (s.u_end + kTileM - 1) / kTileM;
+        cum += s.u_end;
+        P.seg[P.n_seg++] = s;
+    }
+    P.chain_cum[g->k] = cum;
+    P.T = cum;
+    P.n_tiles = tiles;
+    P.n_eval = cum;
+    *n_out = cum;
+    return P;
+}
+
+// ---- weight preparation for the tensor-core path ----------------------------
+uint16_t f2h_bits(float v) {
+    __half h = __float2half_rn(v);
+    uint16_t b;
+    memcpy(&b, &h, 2);
+    return b;
+}
+float h2f(uint16_t b) {
+    __half h;
+    memcpy(&h, &b, 2);
+    return __half2float(h);
+}
+uint16_t f2b_bits(float v) {
+    __nv_bfloat16 h = __float2bfloat16_rn(v);
+    uint16_t b;
+    memcpy(&b, &h, 2);
+    return b;
+}
+float b2f(uint16_t b) {
+    __nv_bfloat16 h;
+    memcpy(&h, &b, 2);
+    return __bfloat162float(h);
+}
+
+// smallest s >= 0 with bound * 2^-s <= 2^14 (fp16 activations stay < 65504)
+int scale_exp(double bound) {
+    int s = 0;
+    while (bound / std::ldexp(1.0, s) > 16384.0 && s < 60) s++;
+    return s;
+}
+
+// blob: [W2 chunks][W3 chunks][out chunks]; chunk = N rows x 16 K, b_offset layout
+std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale) {
+    const int D = c->D;
+    const float* p = c->params.data();
+    const float* W1 = p;
+    const float* b1 = W1 + kHidden * D;
+    const float* W2 = b1 + kHidden;
+    const float* b2 = W2 + kHidden * kHidden;
+    const float* W3 = b2 + kHidden;
+    const float* b3 = W3 + kHidden * kHidden;
+    const float* w4 = b3 + kHidden;
+    const float b4 = w4[kHidden];
+    // exact power-of-two layer scales (fp16 only): worst-case activation bounds
+    // with |x| <= 32768 (any int16 feature row)
+    double s1 = 1, s2 = 1, s3 = 1;
+    if (fmt == 0) {
+        double B1 = 0, B2 = 0, B3 = 0;
+        for (int i = 0; i < kHidden; i++) {
+            double a = std::fabs((double)b1[i]);
+            for (int j = 0; j < D; j++) a += std::fabs((double)W1[i * D + j]) * 32768.0;
+            B1 = std::max(B1, a);
+        }
+        for (int i = 0; i < kHidden; i++) {
+            double a = std::fabs((double)b2[i]);
+            for (int j = 0; j < kHidden; j++) a += std::fabs((double)W2[i * kHidden + j]) * B1;
+            B2 = std::max(B2, a);
+        }
+        for (int i = 0; i < kHidden; i++) {
+            double a = std::fabs((double)b3[i]);
+            for (int j = 0; j < kHidden; j++) a += std::fabs((double)W3[i * kHidden + j]) * B2;
+            B3 = std::max(B3, a);
+        }
+        s1 = std::ldexp(1.0, -scale_exp(B1));
+        s2 = std::ldexp(1.0, -scale_exp(B2));
+        s3 = std::ldexp(1.0, -scale_exp(B3));
+    }
+    *l1_scale = (float)s1;
+    const int nch = fmt == 0 ? 3 : 5;
+    const size_t hid_bytes = (size_t)nch * tc::kChunkBytesN32;
+    const size_t out_bytes = (size_t)nch * tc::kChunkBytesN16;
+    std::vector<uint8_t> blob(2 * hid_bytes + out_bytes, 0);
+    auto put = [&](size_t base, int n, int k, uint16_t v) {
+        memcpy(blob.data() + base + tc::b_offset(n, k), &v, 2);
+    };
+    auto conv = [&](float v) { return fmt == 0 ? f2h_bits(v) : f2b_bits(v); };
+    auto back = [&](uint16_t b) { return fmt == 0 ? h2f(b) : b2f(b); };
+    // hidden layers: out unit n, input j; scale factor maps scaled-in -> scaled-out
+    auto hidden = [&](size_t base, const float* W, const float* b, double sin, double sout) {
+        const double f = sout / sin;  // W' = W * (s_out / s_in) with s = 2^-e
+        for (int n = 0; n < kHidden; n++) {
+            for (int j = 0; j < kHidden; j++) {
+                const float w = (float)((double)W[n * kHidden + j] * f);
+                const int ch = j >> 4, k = j & 15;
+                const uint16_t hi = conv(w);
+                put(base + (size_t)ch * tc::kChunkBytesN32, n, k, hi);
+                if (fmt == 1) put(base + (size_t)(2 + ch) * tc::kChunkBytesN32, n, k, conv(w - back(hi)));
+            }
+            const float bb = (float)((double)b[n] * sout);
+            const uint16_t bh = conv(bb);
+            const size_t cb = base + (size_t)(nch - 1) * tc::kChunkBytesN32;
+            put(cb, n, 0, bh);
+            put(cb, n, 1, conv(bb - back(bh)));
+        }
+    };
+    hidden(0, W2, b2, s1, s2);
+    hidden(hid_bytes, W3, b3, s2, s3);
+    // output layer: row 0 = w4 / s3, rows 1..15 zero; bias (b4 hi, lo)
+    {
+        const size_t base = 2 * hid_bytes;
+        for (int j = 0; j < kHidden; j++) {
+            const float w = (float)((double)w4[j] / s3);
+            const int ch = j >> 4, k = j & 15;
+            const uint16_t hi = conv(w);
+            put(base + (size_t)ch * tc::kChunkBytesN16, 0, k, hi);
+            if (fmt == 1) put(base + (size_t)(2 + ch) * tc::kChunkBytesN16, 0, k, conv(w - back(hi)));
+        }
+        const uint16_t bh = conv(b4);
+        const size_t cb = base + (size_t)(nch - 1) * tc::kChunkBytesN16;
+        put(cb, 0, 0, bh);
+        put(cb, 0, 1, conv(b4 - back(bh)));
+    }
+    return blob;
+}
+
+cudaStream_t pick_stream(abacus_ctx* c, void* st) { return st ? (cudaStream_t)st : c->stream; }
+
+int launch_fused(abacus_ctx* c, const Plan& P) {
+    int grid = 0;
+    cudaError_t e;
+    if (c->timed) cudaEventRecord(c->ev0, c->stream);
+    if (c->precision == ABACUS_FP32) {
+        e = launch_fused_fp32(P, c->w234, c->d_w1b1, c->S, c->nsm, c->stream, &grid);
+    } else {
+        const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
+        e = launch_fused_tc(P, c->tw[fmt], c->d_w1b1, c->S, c->nsm, c->stream, &grid);
+    }
+    if (c->timed) cudaEventRecord(c->ev1, c->stream);
+    if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "fused search launch: %s", cudaGetErrorString(e));
+    c->launches++;
+    return ABACUS_OK;
+}
+
+}  // namespace
+
+// ============================================================================
+// C ABI
+// ============================================================================
+extern "C" {
+
+int abacus_abi_version(void) { return ABACUS_ABI_VERSION; }
+
+int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, int32_t k_max, abacus_ctx** out) {
+    if (!out || !ops_per_model) return ABACUS_E_INVALID;
+    if (n_models < 1 || n_models > 64 || k_max != ABACUS_K_MAX) return ABACUS_E_INVALID;
+    for (int i = 0; i < n_models; i++)
+        if (ops_per_model[i] < 1 || ops_per_model[i] > 32767) return ABACUS_E_INVALID;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return ABACUS_E_DEVICE;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return ABACUS_E_CUDA;
+    if (prop.major != 10 || prop.minor != 0) return ABACUS_E_DEVICE;  // sm_100 only: no fallback
+    if (cudaSetDevice(device) != cudaSuccess) return ABACUS_E_CUDA;
+    abacus_ctx* c = new abacus_ctx();
+    c->device = device;
+    c->nsm = prop.multiProcessorCount;
+    c->n_models = n_models;
+    c->D = n_models + 4 * ABACUS_K_MAX;
+    c->L.assign(ops_per_model, ops_per_model + n_models);
+    bool ok = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaMalloc(&c->S, sizeof(Scratch)) == cudaSuccess &&
+              cudaMemset(c->S, 0, sizeof(Scratch)) == cudaSuccess &&
+              cudaMallocHost(&c->host_result, sizeof(Result)) == cudaSuccess &&
+              cudaEventCreate(&c->ev0) == cudaSuccess && cudaEventCreate(&c->ev1) == cudaSuccess;
+    if (ok) {
+        const float nan = NAN;
+        ok = cudaMemcpy(&c->S->y0, &nan, sizeof(float), cudaMemcpyHostToDevice) == cudaSuccess;
+    }
+    c->stream = c->own_stream;
+    if (!ok) {
+        abacus_destroy(c);
+        return ABACUS_E_CUDA;
+    }
+    *out = c;
+    return ABACUS_OK;
+}
+
+void abacus_destroy(abacus_ctx* c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    if (c->own_stream) cudaStreamSynchronize(c->own_stream);
+    cudaFree(c->S);
+    cudaFree(c->d_w1b1);
+    cudaFree(c->d_blob[0]);
+    cudaFree(c->d_blob[1]);
+    if (c->host_result) cudaFreeHost(c->host_result);
+    if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->own_stream) cudaStreamDestroy(c->own_stream);
+    delete c;
+}
+
+const char* abacus_last_error(const abacus_ctx* c) { return c ? c->err.c_str() : "null ctx"; }
+
+uint64_t abacus_kernel_launches(const abacus_ctx* c) { return c ? c->launches : 0; }
+
+float abacus_last_kernel_ms(const abacus_ctx* c) {
+    if (!c || !c->timed) return -1.0f;
+    float ms = -1.0f;
+    if (cudaEventSynchronize(c->ev1) != cudaSuccess) return -1.0f;
+    if (cudaEventElapsedTime(&ms, c->ev0, c->ev1) != cudaSuccess) return -1.0f;
+    return ms;
+}
+
+int abacus_load_predictor(abacus_ctx* c, const float* params, size_t n_params, int precision) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    const size_t want = (size_t)kHidden * c->D + 2 * kHidden * kHidden + 4 * kHidden + 1;
+    if (!params || n_params != want)
+        return fail(c, ABACUS_E_INVALID, "n_params=%zu, expected %zu for D=%d", n_params, want, c->D);
+    if (precision != ABACUS_FP32 && precision != ABACUS_BF16 && precision != ABACUS_FP16)
+        return fail(c, ABACUS_E_INVALID, "unknown precision %d", precision);
+    for (size_t i = 0; i < n_params; i++)
+        if (!std::isfinite(params[i])) return fail(c, ABACUS_E_INVALID, "param %zu is not finite", i);
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    c->params.assign(params, params + n_params);
+    const int D = c->D;
+    const float* p = c->params.data();
+    if (!c->d_w1b1) CUDA_TRY(c, cudaMalloc(&c->d_w1b1, sizeof(float) * (kHidden * D + kHidden)));
+    CUDA_TRY(c, cudaMemcpy(c->d_w1b1, p, sizeof(float) * (kHidden * D + kHidden), cudaMemcpyHostToDevice));
+    const float* q = p + kHidden * D + kHidden;
+    memcpy(&c->w234.W2[0][0], q, sizeof(float) * kHidden * kHidden);
+    q += kHidden * kHidden;
+    memcpy(c->w234.b2, q, sizeof(float) * kHidden);
+    q += kHidden;
+    memcpy(&c->w234.W3[0][0], q, sizeof(float) * kHidden * kHidden);
+    q += kHidden * kHidden;
+    memcpy(c->w234.b3, q, sizeof(float) * kHidden);
+    q += kHidden;
+    memcpy(c->w234.w4, q, sizeof(float) * kHidden);
+    q += kHidden;
+    c->w234.b4 = *q;
+    for (int fmt = 0; fmt < 2; fmt++) {
+        float l1s = 1.0f;
+        std::vector<uint8_t> blob = build_blob(c, fmt, &l1s);
+        if (c->d_blob[fmt]) cudaFree(c->d_blob[fmt]);
+        CUDA_TRY(c, cudaMalloc(&c->d_blob[fmt], blob.size()));
+        CUDA_TRY(c, cudaMemcpy(c->d_blob[fmt], blob.data(), blob.size(), cudaMemcpyHostToDevice));
+        c->tw[fmt] = TcWeights{fmt, fmt == 0 ? 3 : 5, fmt == 0 ? 3 : 5, (uint32_t)blob.size(), l1s, c->d_blob[fmt]};
+    }
+    c->precision = precision;
+    c->loaded = true;
+    return ABACUS_OK;
+}
+
+int abacus_encode_candidates(abacus_ctx* c, const abacus_grid_t* grid, uint64_t first, uint64_t count,
+                             int16_t* d_features, void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    uint64_t T = 0;
+    int rc = validate_grid(c, grid, &T);
+    if (rc) return rc;
+    if (first > T || count > T - first) return fail(c, ABACUS_E_INVALID, "range beyond T=%llu", (unsigned long long)T);
+    if (count && !d_features) return fail(c, ABACUS_E_INVALID, "d_features is NULL");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    const Plan P = plan_whole_grid(c, grid, T);
+    CUDA_TRY(c, launch_encode_grid(P, first, count, d_features, c->nsm, pick_stream(c, stream)));
+    if (count) c->launches++;
+    return ABACUS_OK;
+}
+
+int abacus_encode_groups(abacus_ctx* c, const abacus_group_t* d_groups, uint64_t count, int16_t* d_features,
+                         uint32_t* d_bad, void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (count && (!d_groups || !d_features)) return fail(c, ABACUS_E_INVALID, "NULL device buffer");
+    static_assert(sizeof(abacus_group_t) == 4 + 4 * 5 * 4, "group record layout");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    CUDA_TRY(c, launch_encode_groups(d_groups, count, c->n_models, c->D, d_features, d_bad, c->nsm,
+                                     pick_stream(c, stream)));
+    if (count) c->launches++;
+    return ABACUS_OK;
+}
+
+int abacus_predict_batch(abacus_ctx* c, const int16_t* d_features, uint64_t count, float* d_latency_ms,
+                         void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (count && (!d_features || !d_latency_ms)) return fail(c, ABACUS_E_INVALID, "NULL device buffer");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    cudaStream_t st = pick_stream(c, stream);
+    if (c->precision == ABACUS_FP32) {
+        CUDA_TRY(c, launch_predict_fp32(c->w234, c->d_w1b1, c->D, d_features, count, d_latency_ms, c->nsm, st));
+    } else {
+        if (c->D > 40) return fail(c, ABACUS_E_INVALID, "tensor predict supports D <= 40");
+        const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
+        CUDA_TRY(c, launch_predict_tc(c->tw[fmt], c->d_w1b1, c->D, d_features, count, d_latency_ms, c->nsm, st));
+    }
+    if (count) c->launches++;
+    return ABACUS_OK;
+}
+
+int abacus_select_group(abacus_ctx* c, const abacus_grid_t* grid, uint64_t first, uint64_t count,
+                        const float* d_latency_ms, float headroom_ms, unsigned long long* d_best_key,
+                        void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    uint64_t T = 0;
+    int rc = validate_grid(c, grid, &T);
+    if (rc) return rc;
+    if (first > T || count > T - first) return fail(c, ABACUS_E_INVALID, "range beyond T");
+    if (!d_best_key || (count && !d_latency_ms)) return fail(c, ABACUS_E_INVALID, "NULL device buffer");
+    if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    const Plan P = plan_whole_grid(c, grid, T);
+    CUDA_TRY(c, launch_select(P, first, count, d_latency_ms, headroom_ms, d_best_key, c->nsm,
+                              pick_stream(c, stream)));
+    if (count) c->launches++;
+    return ABACUS_OK;
+}
+
+int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                  int32_t space, uint64_t grid_budget, abacus_decision_t* out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (!q || !out) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (k < 1 || k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
+    if (space < ABACUS_SPACE_GRID || space > ABACUS_SPACE_AUTO) return fail(c, ABACUS_E_INVALID, "bad space");
+    if (!std::isfinite(now_ms) || !std::isfinite(inflight_pred_ms))
+        return fail(c, ABACUS_E_INVALID, "non-finite time");
+    // a1: Eq. 2 + Eq. 3 headroom per query; ascending order, ties by model id
+    double h[ABACUS_K_MAX];
+    int32_t order[ABACUS_K_MAX];
+    for (int i = 0; i < k; i++) {
+        const abacus_query_t& a = q[i];
+        if (a.model_id < 1 || a.model_id > c->n_models)
+            return fail(c, ABACUS_E_INVALID, "query %d: model_id %d", i, a.model_id);
+        for (int j = 0; j < i; j++)
+            if (q[j].model_id == a.model_id) return fail(c, ABACUS_E_DUP_MODEL, "queries %d, %d share a model", j, i);
+        const int32_t L = c->L[a.model_id - 1];
+        if (a.next_op < 1 || a.next_op > L) return fail(c, ABACUS_E_INVALID, "query %d: next_op %d", i, a.next_op);
+        if (a.batch < 1 || a.batch > 32767 || a.seqlen < 0 || a.seqlen > 32767)
+            return fail(c, ABACUS_E_INVALID, "query %d: batch/seqlen", i);
+        if (!std::isfinite(a.qos_ms) || !std::isfinite(a.t_start_ms))
+            return fail(c, ABACUS_E_INVALID, "query %d: non-finite time", i);
+        h[i] = (a.qos_ms - (now_ms - a.t_start_ms)) - inflight_pred_ms;
+        order[i] = i;
+    }
+    std::stable_sort(order, order + k, [&](int a, int b) {
+        if (h[a] != h[b]) return h[a] < h[b];
+        return q[a].model_id < q[b].model_id;
+    });
+    const float H = (float)h[order[0]];
+    // a2: slots in headroom order; the critical query is fully included
+    abacus_grid_t g{};
+    g.k = k;
+    for (int j = 0; j < k; j++) {
+        const abacus_query_t& a = q[order[j]];
+        const int32_t L = c->L[a.model_id - 1];
+        g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? L : a.next_op, L, j == 0 ? 0 : 1};
+    }
+    uint64_t T = 0;
+    int rc = validate_grid(c, &g, &T);
+    if (rc) return rc;
+    const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
+    Plan P;
+    uint64_t n_eval = 0;
+    if (chain) {
+        P = plan_chain(c, &g, H, &n_eval);
+    } else {
+        P = plan_grid_segments(c, &g, T, 0, T, H);
+        n_eval = P.n_eval;
+    }
+    P.want_y0 = 1;
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    rc = launch_fused(c, P);
+    if (rc) return rc;
+    CUDA_TRY(c, cudaMemcpyAsync(c->host_result, &c->S->result, sizeof(Result), cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    const Result& R = *c->host_result;
+    // a7: decision assembly
+    abacus_decision_t d{};
+    d.critical = order[0];
+    for (int j = 0; j < 4; j++) d.order[j] = j < k ? order[j] : -1;
+    d.headroom_ms = H;
+    d.pred_critical_only_ms = R.y0;
+    d.evaluated = n_eval;
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    if (!(R.y0 <= H)) {  // drop mechanism
+        d.status = ABACUS_DECIDE_DROP;
+        d.pred_ms = R.y0;
+        d.total_ops = 0;
+    } else {
+        d.status = ABACUS_DECIDE_OK;
+        d.pred_ms = R.y_best;
+        d.total_ops = R.total_ops;
+        for (int j = 0; j < k; j++) d.end_op[order[j]] = R.end_op[j];
+    }
+    *out = d;
+    return ABACUS_OK;
+}
+
+int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_ms, uint64_t first, uint64_t count,
+                       void* nccl_comm, abacus_decision_t* out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (!out) return fail(c, ABACUS_E_INVALID, "out is NULL");
+    uint64_t T = 0;
+    int rc = validate_grid(c, grid, &T);
+    if (rc) return rc;
+    if (first > T || count > T - first) return fail(c, ABACUS_E_INVALID, "range beyond T");
+    if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    Plan P = plan_grid_segments(c, grid, T, first, first + count, headroom_ms);
+    rc = launch_fused(c, P);
+    if (rc) return rc;
+    if (nccl_comm) {
+        int nranks = 0;
+        ncclComm_t comm = (ncclComm_t)nccl_comm;
+        if (!nccl().ok) return fail(c, ABACUS_E_NCCL, "libnccl.so.2 not available");
+        if (nccl().CommCount(comm, &nranks) != ncclSuccess || nranks < 1 || nranks > 64)
+            return fail(c, ABACUS_E_NCCL, "bad communicator");
+        ncclResult_t nr = nccl().AllGather(&c->S->result, c->S->gathered, sizeof(Result), ncclUint8, comm, c->stream);
+        if (nr != ncclSuccess) return fail(c, ABACUS_E_NCCL, "ncclAllGather: %s", nccl().GetErrorString(nr));
+        CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->stream));
+        c->launches++;
+    }
+    CUDA_TRY(c, cudaMemcpyAsync(c->host_result, &c->S->result, sizeof(Result), cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    const Result& R = *c->host_result;
+    abacus_decision_t d{};
+    d.critical = 0;
+    for (int j = 0; j < 4; j++) d.order[j] = j < grid->k ? j : -1;
+    d.headroom_ms = headroom_ms;
+    d.pred_critical_only_ms = R.y0;
+    d.evaluated = R.evaluated;
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    d.status = R.key ? ABACUS_DECIDE_OK : ABACUS_DECIDE_NONE;
+    d.pred_ms = R.key ? R.y_best : NAN;
+    d.total_ops = R.total_ops;
+    for (int j = 0; j < grid->k; j++) d.end_op[j] = R.end_op[j];
+    *out = d;
+    return ABACUS_OK;
+}
+
+int abacus_nccl_unique_id(uint8_t* id128) {
+    if (!id128) return ABACUS_E_INVALID;
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    ncclUniqueId id;
+    if (!nccl().ok || nccl().GetUniqueId(&id) != ncclSuccess) return ABACUS_E_NCCL;
+    memcpy(id128, &id, 128);
+    return ABACUS_OK;
+}
+
+int abacus_nccl_comm_init(abacus_ctx* c, int32_t nranks, int32_t rank, const uint8_t* id128, void** comm_out) {
+    if (!c || !id128 || !comm_out || nranks < 1 || nranks > 64 || rank < 0 || rank >= nranks)
+        return fail(c, ABACUS_E_INVALID, "bad NCCL init arguments");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    ncclUniqueId id;
+    memcpy(&id, id128, 128);
+    ncclComm_t comm;
+    if (!nccl().ok) return fail(c, ABACUS_E_NCCL, "libnccl.so.2 not available");
+    ncclResult_t nr = nccl().CommInitRank(&comm, nranks, id, rank);
+    if (nr != ncclSuccess) return fail(c, ABACUS_E_NCCL, "ncclCommInitRank: %s", nccl().GetErrorString(nr));
+    *comm_out = comm;
+    return ABACUS_OK;
+}
+
+void abacus_nccl_comm_destroy(void* comm) {
+    if (comm && nccl().ok) nccl().CommDestroy((ncclComm_t)comm);
+}
+
+int abacus_set_stream(abacus_ctx* c, void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    if (c->own_stream && c->stream != (cudaStream_t)stream && stream) {
+        cudaStreamSynchronize(c->stream);
+    }
+    c->stream = stream ? (cudaStream_t)stream : c->own_stream;
+    return ABACUS_OK;
+}
+
+int abacus_set_timing(abacus_ctx* c, int on) {
+    if (!c) return ABACUS_E_INVALID;
+    c->timed = on != 0;
+    return ABACUS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,141 @@
+// common.cuh -- shared device/host definitions of the CUDA path (sm_100a).
+//
+// The "plan" describes a candidate space as a list of SEGMENTS.  A segment is
+// one presence pattern P of the slots (which services are in the group) and
+// the box of end-op digits of its present slots:
+//     ope_j = ope0_j + v_j,  v_j in [0, cnt_j)          (present slots)
+//     index = t_base + sum_j v_j * istride_j             (t for GRID, u for CHAIN)
+//     sum_n = n_base + sum_j v_j                          (reading c12)
+// Box-local ordinal u in [u_begin, u_end) enumerates v in mixed radix with the
+// last slot fastest, so index(u) is increasing in u.  Every candidate of the
+// grid (ABI abacus_grid_t) lies in exactly one
+// segment, and within a segment the Fig.-8 slot positions are
+// uniform: this is what lets a 128-row tile share one layer-1 operand.
+#pragma once
+#include <cstdint>
+
+namespace abacus {
+
+constexpr int kHidden = 32;
+constexpr int kKMax = 4;
+constexpr int kMaxSeg = 16;
+constexpr int kTileM = 128;  // candidates per tile = TMEM lanes = tcgen05 M
+
+// floor(x / d) for x < 2^31 via multiply-high (Granlund-Montgomery round-up).
+struct FastDiv {
+    uint32_t mul, shift, d;
+};
+
+struct SegP {
+    uint64_t u_begin, u_end;  // box-local ordinal range of this shard
+    uint64_t tile0;           // first work item (tile) of the segment
+    uint64_t t_base;          // index of the v = 0 element
+    uint64_t istride[kKMax];  // index stride per slot (0 if absent)
+    uint64_t bstride[kKMax];  // box stride per slot (product of later cnt)
+    double rbstride[kKMax];   // 1.0 / bstride_j (uniform fp64 split of the tile base)
+    FastDiv fd[kKMax];        // divide by cnt_j
+    uint32_t cnt[kKMax];      // box radix per slot (1 if absent)
+    int32_t ope0[kKMax];      // ope at v = 0, 0 if absent
+    int32_t pos[kKMax];       // Fig.-8 position (rank by model id among present), -1 absent
+    int32_t n_base;           // sum_n at v = 0
+    uint32_t mask;            // present slots
+};
+
+struct SlotP {
+    int32_t model_id, ops, bs, seqlen;
+    int32_t end_lo, end_hi, absent, radix;  // grid digit definition (decode of t*)
+};
+
+enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
+
+struct Plan {
+    int32_t k, n_seg, n_models, D;
+    int32_t mode;           // kModeGrid (t) or kModeChain (u)
+    int32_t want_y0;        // 1 if index 0 is in range (decision drop test)
+    float H;                // headroom threshold (inclusive)
+    int32_t pad;
+    uint64_t n_tiles;       // total work items
+    uint64_t T;             // size of the whole space
+    uint64_t n_eval;        // candidates in this plan (this shard)
+    uint64_t chain_cum[kKMax + 1];  // CHAIN: first u of block j
+    SlotP slot[kKMax];
+    SegP seg[kMaxSeg];
+};
+
+// result record written by the last CTA (and gathered across ranks)
+struct Result {
+    unsigned long long key;  // best key, 0 = none
+    float y_best;            // y(t*)
+    float y0;                // y(index 0), NaN if not evaluated
+    unsigned long long evaluated;
+    int32_t end_op[kKMax];   // decoded t* per slot (grid order), 0 absent
+    int32_t total_ops;
+    int32_t status;          // 0 OK, 2 NONE (set by host for decisions)
+};
+
+struct Scratch {             // device scratch owned by the ctx
+    unsigned long long cta_key[1024];
+    float cta_y[1024];
+    float y0;
+    unsigned int counter;    // last-CTA ticket, self-resetting
+    unsigned int pad;
+    Result result;
+    Result gathered[64];
+};
+
+#ifdef __CUDACC__
+
+__device__ __forceinline__ uint32_t fastdiv(uint32_t x, const FastDiv& f) {
+    uint32_t q = __umulhi(x, f.mul);
+    return (q + x) >> f.shift;
+}
+
+// digits v[j] of the box ordinal u = ub + r (ub uniform across the tile,
+// r < 2^20 per thread): ub is split with an fp64 reciprocal (exact after one
+// correction step since ub < 2^40), r is then added to the last digit and
+// carried with 32-bit multiply-high divisions.
+template <int K>
+__device__ __forceinline__ void decode_box(const SegP& s, uint64_t ub, uint32_t r, uint32_t (&v)[kKMax]) {
+    uint64_t rem = ub;
+#pragma unroll
+    for (int j = 0; j < K; j++) {
+        uint64_t bs = s.bstride[j];
+        uint64_t q;
+        if (bs == 1) {
+            q = rem;
+        } else {
+            q = (uint64_t)((double)rem * s.rbstride[j]);
+            int64_t rr = (int64_t)(rem - q * bs);
+            if (rr < 0) { q--; }
+            else if ((uint64_t)rr >= bs) { q++; }
+        }
+        v[j] = (uint32_t)q;
+        rem -= q * bs;
+    }
+    // add r to the last digit and carry
+    uint32_t carry = r;
+#pragma unroll
+    for (int j = K - 1; j >= 0; j--) {
+        uint32_t x = v[j] + carry;
+        uint32_t q = fastdiv(x, s.fd[j]);
+        v[j] = x - q * s.cnt[j];
+        carry = q;
+    }
+}
+
+__device__ __forceinline__ unsigned long long umax64(unsigned long long a, unsigned long long b) {
+    return a > b ? a : b;
+}
+
+__device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        unsigned long long w = __shfl_xor_sync(0xffffffffu, v, o);
+        v = umax64(v, w);
+    }
+    return v;
+}
+
+#endif  // __CUDACC__
+
+}  // namespace abacus

@@ -1,0 +1,102 @@
+// device_common.cuh -- device helpers shared by the SIMT and tensor-core
+// kernels (header-only: the library is built without relocatable device code).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace abacus {
+
+// grid digit -> ope (0 = absent); SlotP carries the ABI digit definition
+__device__ __forceinline__ int32_t digit_to_ope(const SlotP& s, uint32_t d) {
+    if (s.absent) return d == 0 ? 0 : s.end_lo + (int32_t)d - 1;
+    return s.end_lo + (int32_t)d;
+}
+
+__device__ __forceinline__ int find_segment(const Plan& P, uint64_t w) {
+    int s = 0;
+    for (int i = 1; i < P.n_seg; i++)
+        if (w >= P.seg[i].tile0) s = i;
+    return s;
+}
+
+// ---------------------------------------------------------------------------
+// Last-CTA epilogue shared by the fused kernels (a5 cross-CTA + a7 decode).
+// Each CTA publishes its best (key, y); the last CTA to arrive reduces them,
+// decodes the winning index into end ops per slot and resets the ticket.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void decode_index_to_ope(const Plan& P, unsigned long long idx, int32_t (&ope)[kKMax]) {
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) ope[j] = 0;
+    if (P.mode == kModeGrid) {
+        unsigned long long t = idx;
+        for (int j = P.k - 1; j >= 0; j--) {
+            const unsigned long long r = (unsigned long long)P.slot[j].radix;
+            const uint32_t d = (uint32_t)(t % r);
+            t /= r;
+            ope[j] = digit_to_ope(P.slot[j], d);
+        }
+    } else {
+        int blk = 0;
+        for (int j = 1; j < P.k; j++)
+            if (idx >= P.chain_cum[j]) blk = j;
+        for (int j = 0; j < P.k; j++) {
+            if (j < blk) ope[j] = P.slot[j].end_hi;
+            else if (j == blk) ope[j] = blk == 0 ? P.slot[0].end_hi
+                                                  : P.slot[j].ops + (int32_t)(idx - P.chain_cum[j]);
+        }
+    }
+}
+
+static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratch* S, unsigned long long key, float y) {
+    __shared__ unsigned long long s_key[32];
+    __shared__ float s_y[32];
+    __shared__ bool s_last;
+    // warp (key, y) max: y follows its key
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, key, o);
+        const float y2 = __shfl_xor_sync(0xffffffffu, y, o);
+        if (k2 > key) { key = k2; y = y2; }
+    }
+    const int warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    if ((threadIdx.x & 31) == 0) { s_key[warp] = key; s_y[warp] = y; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long bk = 0;
+        float by = __int_as_float(0x7fc00000);
+        for (int w = 0; w < nwarps; w++)
+            if (s_key[w] > bk) { bk = s_key[w]; by = s_y[w]; }
+        S->cta_key[blockIdx.x] = bk;
+        S->cta_y[blockIdx.x] = by;
+        __threadfence();
+        const unsigned int ticket = atomicAdd(&S->counter, 1u);
+        s_last = ticket == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    if (threadIdx.x == 0) {
+        unsigned long long bk = 0;
+        float by = __int_as_float(0x7fc00000);
+        for (unsigned int b = 0; b < gridDim.x; b++) {
+            const unsigned long long kk = *((volatile unsigned long long*)&S->cta_key[b]);
+            if (kk > bk) { bk = kk; by = *((volatile float*)&S->cta_y[b]); }
+        }
+        Result& R = S->result;
+        R.key = bk;
+        R.y_best = by;
+        R.y0 = *((volatile float*)&S->y0);
+        R.evaluated = P.n_eval;
+        int32_t ope[kKMax];
+        decode_index_to_ope(P, bk & ((1ull << 40) - 1), ope);
+        for (int j = 0; j < kKMax; j++) R.end_op[j] = bk ? ope[j] : 0;
+        R.total_ops = bk ? (int32_t)(bk >> 40) - 1 : 0;
+        R.status = bk ? 0 : 2;
+        S->y0 = __int_as_float(0x7fc00000);
+        S->counter = 0;
+        __threadfence();
+    }
+}
+
+}  // namespace abacus

@@ -1,0 +1,48 @@
+// internal.h -- declarations shared by the host API and the kernel files.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "common.cuh"
+
+namespace abacus {
+
+// layers 2..4 in fp32, passed by value as a kernel parameter (constant bank)
+struct W234 {
+    float W2[kHidden][kHidden];
+    float b2[kHidden];
+    float W3[kHidden][kHidden];
+    float b3[kHidden];
+    float w4[kHidden];
+    float b4;
+};
+
+// tensor-core weight blob: layer 2 / layer 3 / output chunks in the shared
+// memory B-operand layout (tc_ptx.cuh b_offset), prepared at load time
+struct TcWeights {
+    int fmt;           // 0 fp16, 1 bf16
+    int nch_hidden;    // B chunks per hidden layer (fp16 3, bf16 5)
+    int nch_out;       // B chunks of the output layer (fp16 3, bf16 5)
+    uint32_t bytes;    // blob size
+    float l1_scale;    // 2^-s1 applied to layer-1 weights (fp16), 1 (bf16)
+    const uint8_t* blob;  // device
+};
+
+cudaError_t launch_encode_grid(const Plan& P, uint64_t first, uint64_t count, int16_t* out, int nsm,
+                               cudaStream_t st);
+cudaError_t launch_encode_groups(const void* groups, uint64_t count, int32_t n_models, int32_t D, int16_t* out,
+                                 uint32_t* bad, int nsm, cudaStream_t st);
+cudaError_t launch_predict_fp32(const W234& W, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
+                                float* y, int nsm, cudaStream_t st);
+cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const float* lat, float H,
+                          unsigned long long* best, int nsm, cudaStream_t st);
+cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,
+                              cudaStream_t st, int* grid_out);
+cudaError_t launch_finalize_gather(Scratch* S, int nranks, cudaStream_t st);
+
+cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
+                            cudaStream_t st, int* grid_out);
+cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
+                              float* y, int nsm, cudaStream_t st);
+
+}  // namespace abacus

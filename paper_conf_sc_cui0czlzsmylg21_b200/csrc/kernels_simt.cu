@@ -1,0 +1,393 @@
+// kernels_simt.cu -- SIMT kernels of the Abacus candidate search (sm_100a).
+//
+//   encode_grid_kernel      a2+a3  grid range -> Fig.-8 int16 rows
+//   encode_groups_kernel    a3     explicit groups -> Fig.-8 rows
+//   predict_fp32_kernel     a4     MLP forward, fp32 FFMA
+//   select_kernel           a5     headroom mask + max key
+//   fused_fp32_kernel       a2..a5 persistent fused search, fp32 SIMT path
+//   finalize_gather_kernel  a6/a7  max over the ranks' gathered records
+//
+// The fused tensor-core path lives in kernels_tc.cu.
+#include <cuda_runtime.h>
+#include <math.h>
+
+#include "common.cuh"
+#include "device_common.cuh"
+#include "internal.h"
+
+namespace abacus {
+
+// ---------------------------------------------------------------------------
+// shared device helpers
+// ---------------------------------------------------------------------------
+
+// Fig. 8 row for one candidate whose slot j is present with end op ope[j]
+// (ope[j] == 0: absent).  Positions: present slots in ascending model id.
+__device__ __forceinline__ void write_fig8_row(const Plan& P, const int32_t (&ope)[kKMax], int16_t* row) {
+    for (int i = 0; i < P.D; i++) row[i] = 0;
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) {
+        if (j >= P.k || ope[j] == 0) continue;
+        int p = 0;
+#pragma unroll
+        for (int i = 0; i < kKMax; i++)
+            if (i < P.k && ope[i] != 0 && P.slot[i].model_id < P.slot[j].model_id) p++;
+        const SlotP& s = P.slot[j];
+        row[s.model_id - 1] = 1;
+        int16_t* f = row + P.n_models + 4 * p;
+        f[0] = (int16_t)s.ops;
+        f[1] = (int16_t)ope[j];
+        f[2] = (int16_t)s.bs;
+        f[3] = (int16_t)s.seqlen;
+    }
+}
+
+// copy a block's staged rows (smem) to global with 16-byte stores where aligned
+__device__ __forceinline__ void store_rows(const int16_t* sm, int16_t* gout, uint64_t nbytes) {
+    const uintptr_t ga = reinterpret_cast<uintptr_t>(gout);
+    if ((ga & 15) == 0) {
+        const uint64_t n16 = nbytes / 16;
+        const int4* s4 = reinterpret_cast<const int4*>(sm);
+        int4* g4 = reinterpret_cast<int4*>(gout);
+        for (uint64_t i = threadIdx.x; i < n16; i += blockDim.x) g4[i] = s4[i];
+        const char* sb = reinterpret_cast<const char*>(sm);
+        char* gb = reinterpret_cast<char*>(gout);
+        for (uint64_t i = n16 * 16 + threadIdx.x; i < nbytes; i += blockDim.x) gb[i] = sb[i];
+    } else {
+        const uint64_t n2 = nbytes / 2;
+        for (uint64_t i = threadIdx.x; i < n2; i += blockDim.x) gout[i] = sm[i];
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a2 + a3: grid range encode.  One thread per candidate t; the block's rows
+// are staged in shared memory and written with coalesced 16-byte stores.
+// plan.seg[0] is the whole grid as one box (cnt = radix, digits = grid digits).
+// ---------------------------------------------------------------------------
+constexpr int kEncThreads = 128;
+
+__global__ void __launch_bounds__(kEncThreads) encode_grid_kernel(const __grid_constant__ Plan P, uint64_t first,
+                                                                  uint64_t count, int16_t* __restrict__ out) {
+    extern __shared__ int16_t s_rows[];  // kEncThreads * D
+    const SegP& g = P.seg[0];
+    for (uint64_t base = (uint64_t)blockIdx.x * kEncThreads; base < count;
+         base += (uint64_t)gridDim.x * kEncThreads) {
+        const uint64_t idx = base + threadIdx.x;
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, first + base, threadIdx.x, v);
+        int32_t ope[kKMax];
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) ope[j] = j < P.k ? digit_to_ope(P.slot[j], v[j]) : 0;
+        if (idx < count) write_fig8_row(P, ope, s_rows + threadIdx.x * P.D);
+        __syncthreads();
+        const uint64_t nrows = min((uint64_t)kEncThreads, count - base);
+        store_rows(s_rows, out + base * P.D, nrows * P.D * 2);
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3 for explicit groups (config-5 instance samples)
+// ---------------------------------------------------------------------------
+struct GroupRec {
+    int32_t k;
+    int32_t s[kKMax][5];  // model_id, ops, ope, batch, seqlen
+};
+
+__global__ void __launch_bounds__(kEncThreads) encode_groups_kernel(const GroupRec* __restrict__ groups,
+                                                                    uint64_t count, int32_t n_models, int32_t D,
+                                                                    int16_t* __restrict__ out,
+                                                                    uint32_t* __restrict__ bad) {
+    extern __shared__ int16_t s_rows[];
+    for (uint64_t base = (uint64_t)blockIdx.x * kEncThreads; base < count;
+         base += (uint64_t)gridDim.x * kEncThreads) {
+        const uint64_t idx = base + threadIdx.x;
+        int16_t* row = s_rows + threadIdx.x * D;
+        if (idx < count) {
+            const GroupRec g = groups[idx];
+            for (int i = 0; i < D; i++) row[i] = 0;
+            bool ok = g.k >= 0 && g.k <= kKMax;
+            if (ok) {
+                for (int j = 0; j < g.k; j++) {
+                    int m = g.s[j][0];
+                    ok = ok && m >= 1 && m <= n_models;
+                    for (int i = 0; i < j; i++) ok = ok && g.s[i][0] != m;
+                }
+            }
+            if (ok) {
+                for (int j = 0; j < g.k; j++) {
+                    int p = 0;
+                    for (int i = 0; i < g.k; i++) p += g.s[i][0] < g.s[j][0];
+                    row[g.s[j][0] - 1] = 1;
+                    int16_t* f = row + n_models + 4 * p;
+                    f[0] = (int16_t)g.s[j][1];
+                    f[1] = (int16_t)g.s[j][2];
+                    f[2] = (int16_t)g.s[j][3];
+                    f[3] = (int16_t)g.s[j][4];
+                }
+            } else if (bad) {
+                atomicAdd(bad, 1u);
+            }
+        }
+        __syncthreads();
+        const uint64_t nrows = min((uint64_t)kEncThreads, count - base);
+        store_rows(s_rows, out + base * D, nrows * D * 2);
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a4, fp32 SIMT: one thread per candidate row.  Layer 1 weights (runtime D)
+// are staged in shared memory (broadcast reads); layers 2-4 are kernel
+// parameters (constant bank: FFMA with a constant operand, no load).
+// ---------------------------------------------------------------------------
+constexpr int kPredThreads = 128;
+
+__device__ __forceinline__ void mlp_tail_fp32(const W234& W, float (&h1)[kHidden], float& y) {
+    float h2[kHidden];
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) {
+        float s = W.b2[i];
+#pragma unroll
+        for (int j = 0; j < kHidden; j++) s = fmaf(W.W2[i][j], h1[j], s);
+        h2[i] = fmaxf(s, 0.0f);
+    }
+    float acc = W.b4;
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) {
+        float s = W.b3[i];
+#pragma unroll
+        for (int j = 0; j < kHidden; j++) s = fmaf(W.W3[i][j], h2[j], s);
+        acc = fmaf(W.w4[i], fmaxf(s, 0.0f), acc);
+    }
+    y = acc;
+}
+
+__global__ void __launch_bounds__(kPredThreads) predict_fp32_kernel(const __grid_constant__ W234 W,
+                                                                    const float* __restrict__ w1b1, int32_t D,
+                                                                    const int16_t* __restrict__ x, uint64_t count,
+                                                                    float* __restrict__ y) {
+    extern __shared__ float s_w1[];  // W1[32][D] then b1[32]
+    for (int i = threadIdx.x; i < kHidden * D + kHidden; i += blockDim.x) s_w1[i] = w1b1[i];
+    __syncthreads();
+    const float* b1 = s_w1 + kHidden * D;
+    for (uint64_t idx = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < count;
+         idx += (uint64_t)gridDim.x * blockDim.x) {
+        const int16_t* row = x + idx * D;
+        float h1[kHidden];
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) h1[i] = 0.0f;
+        for (int j = 0; j < D; j++) {
+            const float xv = (float)row[j];
+#pragma unroll
+            for (int i = 0; i < kHidden; i++) h1[i] = fmaf(s_w1[i * D + j], xv, h1[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) h1[i] = fmaxf(h1[i] + b1[i], 0.0f);
+        float out;
+        mlp_tail_fp32(W, h1, out);
+        y[idx] = out;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a5: headroom mask + largest-group key over a grid range.  One thread per t;
+// warp shuffle max -> shared -> one atomicMax(u64) per block.
+// ---------------------------------------------------------------------------
+constexpr int kSelThreads = 256;
+
+__global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_constant__ Plan P, uint64_t first,
+                                                             uint64_t count, const float* __restrict__ lat,
+                                                             float H, unsigned long long* best) {
+    __shared__ unsigned long long s_max[kSelThreads / 32];
+    const SegP& g = P.seg[0];
+    unsigned long long mx = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kSelThreads; base < count;
+         base += (uint64_t)gridDim.x * kSelThreads) {
+        const uint64_t idx = base + threadIdx.x;
+        if (idx >= count) break;
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, first + base, threadIdx.x, v);
+        int32_t sum_n = 0;
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) {
+            if (j >= P.k) continue;
+            const int32_t e = digit_to_ope(P.slot[j], v[j]);
+            if (e != 0) sum_n += e - P.slot[j].ops + 1;
+        }
+        const float yv = lat[idx];
+        if (yv <= H) mx = umax64(mx, ((unsigned long long)(sum_n + 1) << 40) | (first + idx));
+    }
+    mx = warp_max_u64(mx);
+    if ((threadIdx.x & 31) == 0) s_max[threadIdx.x >> 5] = mx;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        mx = threadIdx.x < kSelThreads / 32 ? s_max[threadIdx.x] : 0ull;
+        mx = warp_max_u64(mx);
+        if (threadIdx.x == 0 && mx) atomicMax(best, mx);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a2..a5 fused, fp32 SIMT path.  Persistent blocks of 256 threads = two
+// 128-candidate tiles per iteration.  Layer 1 is evaluated per segment as
+//     z1 = c_P + sum_j v_j * w_P,j
+// where c_P = b1 + W1 x0_P (x0_P: the Fig.-8 vector of the segment's v = 0
+// group) and w_P,j = W1[:, N + 4 pos_P(j) + 1] (the ope column of slot j at its
+// Fig.-8 position): x(v) = x0_P + sum_j v_j e_{N+4pos_P(j)+1} is affine in the
+// digits, so this is W1 x + b1 exactly (up to fp32 rounding order).  The
+// per-segment tables are built in the prologue, on device, from fp32 W1/b1.
+// ---------------------------------------------------------------------------
+constexpr int kFusedThreads = 256;
+
+__device__ void build_l1_tables(const Plan& P, const float* __restrict__ w1b1, float* s_c, float* s_w) {
+    // s_c[s][32], s_w[s][4][32]
+    const int D = P.D;
+    const float* b1 = w1b1 + kHidden * D;
+    for (int e = threadIdx.x; e < P.n_seg * kHidden; e += blockDim.x) {
+        const int s = e / kHidden, i = e % kHidden;
+        const SegP& g = P.seg[s];
+        const float* w = w1b1 + i * D;
+        float c = b1[i];
+        for (int j = 0; j < P.k; j++) {
+            if (!((g.mask >> j) & 1u)) {
+                s_w[(s * kKMax + j) * kHidden + i] = 0.0f;
+                continue;
+            }
+            const SlotP& sl = P.slot[j];
+            const int f = P.n_models + 4 * g.pos[j];
+            c = fmaf(w[sl.model_id - 1], 1.0f, c);
+            c = fmaf(w[f + 0], (float)sl.ops, c);
+            c = fmaf(w[f + 1], (float)g.ope0[j], c);
+            c = fmaf(w[f + 2], (float)sl.bs, c);
+            c = fmaf(w[f + 3], (float)sl.seqlen, c);
+            s_w[(s * kKMax + j) * kHidden + i] = w[f + 1];
+        }
+        for (int j = P.k; j < kKMax; j++) s_w[(s * kKMax + j) * kHidden + i] = 0.0f;
+        s_c[s * kHidden + i] = c;
+    }
+}
+
+__global__ void __launch_bounds__(kFusedThreads, 2) fused_fp32_kernel(const __grid_constant__ Plan P,
+                                                                      const __grid_constant__ W234 W,
+                                                                      const float* __restrict__ w1b1, Scratch* S) {
+    __shared__ float s_c[kMaxSeg * kHidden];
+    __shared__ float s_w[kMaxSeg * kKMax * kHidden];
+    build_l1_tables(P, w1b1, s_c, s_w);
+    __syncthreads();
+
+    const uint32_t r = threadIdx.x & (kTileM - 1);
+    const uint64_t half = threadIdx.x >> 7;
+    unsigned long long best = 0;
+    float best_y = __int_as_float(0x7fc00000);
+    for (uint64_t w = (uint64_t)blockIdx.x * 2 + half; w < P.n_tiles; w += (uint64_t)gridDim.x * 2) {
+        const int s = find_segment(P, w);
+        const SegP& g = P.seg[s];
+        const uint64_t ub = g.u_begin + (w - g.tile0) * kTileM;
+        const bool valid = ub + r < g.u_end;
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, ub, r, v);
+        const float* c = s_c + s * kHidden;
+        const float* wc = s_w + s * kKMax * kHidden;
+        float h1[kHidden];
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) {
+            float z = c[i];
+#pragma unroll
+            for (int j = 0; j < kKMax; j++) z = fmaf(wc[j * kHidden + i], (float)v[j], z);
+            h1[i] = fmaxf(z, 0.0f);
+        }
+        float y;
+        mlp_tail_fp32(W, h1, y);
+        uint64_t idx = g.t_base;
+        int32_t sum_n = g.n_base;
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) {
+            idx += (uint64_t)v[j] * g.istride[j];
+            sum_n += (int32_t)v[j];
+        }
+        if (valid && idx == 0) S->y0 = y;
+        if (valid && y <= P.H) {
+            const unsigned long long key = ((unsigned long long)(sum_n + 1) << 40) | idx;
+            if (key > best) { best = key; best_y = y; }
+        }
+    }
+    cta_publish_and_finish(P, S, best, best_y);
+}
+
+// ---------------------------------------------------------------------------
+// a6 tail: after the NCCL all-gather of the per-rank Result records, every
+// rank reduces the same records to the same global decision.
+// ---------------------------------------------------------------------------
+__global__ void finalize_gather_kernel(Scratch* S, int nranks) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    int best = 0;
+    unsigned long long ev = 0;
+    for (int r = 0; r < nranks; r++) {
+        ev += S->gathered[r].evaluated;
+        if (S->gathered[r].key > S->gathered[best].key) best = r;
+    }
+    S->result = S->gathered[best];
+    S->result.evaluated = ev;
+}
+
+// ---------------------------------------------------------------------------
+// launchers
+// ---------------------------------------------------------------------------
+cudaError_t launch_encode_grid(const Plan& P, uint64_t first, uint64_t count, int16_t* out, int nsm,
+                               cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    const uint64_t blocks = (count + kEncThreads - 1) / kEncThreads;
+    const int grid = (int)(blocks < (uint64_t)nsm * 16 ? blocks : (uint64_t)nsm * 16);
+    const size_t smem = (size_t)kEncThreads * P.D * sizeof(int16_t);
+    encode_grid_kernel<<<grid, kEncThreads, smem, st>>>(P, first, count, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_encode_groups(const void* groups, uint64_t count, int32_t n_models, int32_t D, int16_t* out,
+                                 uint32_t* bad, int nsm, cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    const uint64_t blocks = (count + kEncThreads - 1) / kEncThreads;
+    const int grid = (int)(blocks < (uint64_t)nsm * 16 ? blocks : (uint64_t)nsm * 16);
+    const size_t smem = (size_t)kEncThreads * D * sizeof(int16_t);
+    encode_groups_kernel<<<grid, kEncThreads, smem, st>>>(reinterpret_cast<const GroupRec*>(groups), count,
+                                                           n_models, D, out, bad);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_predict_fp32(const W234& W, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
+                                float* y, int nsm, cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    const uint64_t blocks = (count + kPredThreads - 1) / kPredThreads;
+    const int grid = (int)(blocks < (uint64_t)nsm * 8 ? blocks : (uint64_t)nsm * 8);
+    const size_t smem = (size_t)(kHidden * D + kHidden) * sizeof(float);
+    predict_fp32_kernel<<<grid, kPredThreads, smem, st>>>(W, w1b1, D, x, count, y);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const float* lat, float H,
+                          unsigned long long* best, int nsm, cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    const uint64_t blocks = (count + kSelThreads - 1) / kSelThreads;
+    const int grid = (int)(blocks < (uint64_t)nsm * 8 ? blocks : (uint64_t)nsm * 8);
+    select_kernel<<<grid, kSelThreads, 0, st>>>(P, first, count, lat, H, best);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,
+                              cudaStream_t st, int* grid_out) {
+    const uint64_t pairs = (P.n_tiles + 1) / 2;
+    uint64_t g = (uint64_t)nsm * 2;
+    if (pairs < g) g = pairs;
+    if (g < 1) g = 1;
+    *grid_out = (int)g;
+    fused_fp32_kernel<<<(int)g, kFusedThreads, 0, st>>>(P, W, w1b1, S);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_finalize_gather(Scratch* S, int nranks, cudaStream_t st) {
+    finalize_gather_kernel<<<1, 32, 0, st>>>(S, nranks);
+    return cudaGetLastError();
+}
+
+}  // namespace abacus

@@ -1,0 +1,567 @@
+// kernels_tc.cu -- tensor-core (tcgen05 / TMEM) kernels of the Abacus search.
+//
+//   fused_tc_kernel    a2..a5 fused: enumerate -> layer-1 operand in TMEM ->
+//                      3 hidden MMAs + output MMA (bias via a constant-1 K
+//                      column, ReLU + fp16/bf16 pack in the epilogue) ->
+//                      headroom mask -> running max key
+//   predict_tc_kernel  a4 alone: int16 Fig.-8 rows from HBM -> same MLP
+//
+// CTA = NG groups of 4 warps.  A group owns 128 candidate rows = the 128 TMEM
+// lanes (warp q of a group reaches lanes 32q..32q+31) and a private slice of
+// TMEM columns; its first thread issues the group's MMAs (M = 128, N = 32,
+// K = 16 per instruction, A from TMEM, B = weights resident in shared memory)
+// and commits them to the group's mbarrier.  Groups run independently, so
+// while one group waits on its MMA the others run their epilogues.
+//
+// Numerics:
+//   fp16 (FMT 0): weights and activations fp16 RNE, fp32 accumulation; layers
+//     are rescaled by exact powers of two so activations stay in fp16 range
+//     (ReLU is positively homogeneous, so the output is unchanged).
+//   bf16 (FMT 1): activations bf16 RNE; weights split W = W_hi + W_lo (both
+//     bf16) and both halves multiplied (two MMAs per K chunk), fp32 accumulation.
+//   Biases enter as a (hi, lo) pair against a constant-1 K column (both fmts).
+//   Integer digits / features enter split as 256*hi + lo (exact in both fmts).
+#include <cuda_runtime.h>
+#include <math.h>
+
+#include "common.cuh"
+#include "device_common.cuh"
+#include "internal.h"
+#include "tc_ptx.cuh"
+
+namespace abacus {
+
+using namespace tc;
+
+
+struct TcParams {
+    const uint8_t* blob;  // device weight blob (layer 2, layer 3, output chunks)
+    uint32_t bytes;
+    float l1_scale;
+};
+
+template <int FMT>
+struct TcCfg {
+    static constexpr int kNchL1 = FMT == 0 ? 1 : 2;      // layer-1 B chunks per segment (fused)
+    static constexpr int kNchHid = FMT == 0 ? 3 : 5;     // hidden-layer B chunks
+    static constexpr int kNchOut = FMT == 0 ? 3 : 5;     // output-layer B chunks
+    static constexpr uint32_t kOne2 = FMT == 0 ? 0x3C003C00u : 0x3F803F80u;  // (1, 1)
+};
+
+// hi/lo split of an fp32 value into two 16-bit values (hi + lo ~ v)
+template <int FMT>
+__device__ __forceinline__ void split16(float v, uint16_t& hi, uint16_t& lo) {
+    hi = to16<FMT>(v);
+    lo = to16<FMT>(v - from16<FMT>(hi));
+}
+
+// Layer-1 B operand per segment: rows n = hidden unit, K columns
+//   k0 = c_hi, k1 = c_lo, k(2+2j) = 256 w_j, k(3+2j) = w_j   (chunk 0)
+//   bf16: chunk 1 holds the lo halves of the w_j columns.
+// c = b1 + W1 x0 (Fig.-8 vector of the segment's v = 0 group), w_j = the
+// W1 column of slot j's ope at its Fig.-8 position.
+template <int FMT>
+__device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, float scale, uint8_t* s_b1) {
+    constexpr int NCH = TcCfg<FMT>::kNchL1;
+    const int D = P.D;
+    const float* b1 = w1b1 + kHidden * D;
+    for (int e = threadIdx.x; e < P.n_seg * kHidden; e += blockDim.x) {
+        const int s = e / kHidden, n = e % kHidden;
+        const SegP& g = P.seg[s];
+        const float* w = w1b1 + n * D;
+        float c = b1[n];
+        float wj[kKMax];
+        for (int j = 0; j < kKMax; j++) {
+            wj[j] = 0.0f;
+            if (j >= P.k || !((g.mask >> j) & 1u)) continue;
+            const SlotP& sl = P.slot[j];
+            const int f = P.n_models + 4 * g.pos[j];
+            c = fmaf(w[sl.model_id - 1], 1.0f, c);
+            c = fmaf(w[f + 0], (float)sl.ops, c);
+            c = fmaf(w[f + 1], (float)g.ope0[j], c);
+            c = fmaf(w[f + 2], (float)sl.bs, c);
+            c = fmaf(w[f + 3], (float)sl.seqlen, c);
+            wj[j] = w[f + 1] * scale;
+        }
+        c *= scale;
+        uint16_t ch, cl;
+        split16<FMT>(c, ch, cl);
+        uint8_t* base = s_b1 + (size_t)s * NCH * kChunkBytesN32;
+        for (int k = 0; k < 16; k++) {
+            uint16_t v0 = 0, v1 = 0;
+            if (k == 0) v0 = ch;
+            else if (k == 1) v0 = cl;
+            else if (k < 2 + 2 * kKMax) {
+                const int j = (k - 2) >> 1;
+                const float m = ((k - 2) & 1) ? 1.0f : 256.0f;
+                uint16_t h, l;
+                split16<FMT>(wj[j], h, l);
+                if (FMT == 0) {
+                    v0 = to16<FMT>(wj[j] * m);
+                } else {
+                    v0 = to16<FMT>(from16<FMT>(h) * m);
+                    v1 = to16<FMT>(from16<FMT>(l) * m);
+                }
+            }
+            *reinterpret_cast<uint16_t*>(base + b_offset(n, k)) = v0;
+            if (NCH > 1) *reinterpret_cast<uint16_t*>(base + kChunkBytesN32 + b_offset(n, k)) = v1;
+        }
+    }
+}
+
+// issue the MMAs of one hidden layer (N = 32) or the output layer (N = 16)
+template <int FMT>
+__device__ __forceinline__ void issue_layer(uint32_t tD, uint32_t tA, uint32_t tC, uint32_t wbase,
+                                            uint32_t chunk_bytes, uint32_t idesc) {
+    if (FMT == 0) {
+        mma_ts(tD, tA, smem_desc(wbase + 0 * chunk_bytes), idesc, 0u);
+        mma_ts(tD, tA + 8, smem_desc(wbase + 1 * chunk_bytes), idesc, 1u);
+        mma_ts(tD, tC, smem_desc(wbase + 2 * chunk_bytes), idesc, 1u);
+    } else {
+        mma_ts(tD, tA, smem_desc(wbase + 0 * chunk_bytes), idesc, 0u);
+        mma_ts(tD, tA + 8, smem_desc(wbase + 1 * chunk_bytes), idesc, 1u);
+        mma_ts(tD, tA, smem_desc(wbase + 2 * chunk_bytes), idesc, 1u);
+        mma_ts(tD, tA + 8, smem_desc(wbase + 3 * chunk_bytes), idesc, 1u);
+        mma_ts(tD, tC, smem_desc(wbase + 4 * chunk_bytes), idesc, 1u);
+    }
+}
+
+// epilogue of a hidden layer: D (fp32, 32 columns) -> ReLU -> 16-bit pairs -> A
+template <int FMT>
+__device__ __forceinline__ void hidden_epilogue(uint32_t tD_lane, uint32_t tA_lane) {
+    uint32_t r[32];
+    tmem_ld32(tD_lane, r);
+    uint32_t h[16];
+#pragma unroll
+    for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(r[2 * c], r[2 * c + 1]);
+    tmem_st16(tA_lane, h);
+    tmem_wait_st();
+}
+
+// shared-memory carve-up common to both kernels
+struct TcSmem {
+    uint32_t w2, w3, w4;  // byte offsets of the weight chunks
+    uint32_t b1;          // layer-1 B tables
+    uint32_t bars;        // mbarriers
+    uint32_t tmem_slot;
+    uint32_t stage;       // predict: per-group feature staging
+    uint32_t total;
+};
+
+template <int FMT>
+__host__ __device__ inline TcSmem tc_smem_layout(int n_l1_tables, uint32_t l1_table_bytes, int ng,
+                                                  uint32_t stage_bytes_per_group) {
+    TcSmem L{};
+    uint32_t o = 0;
+    L.w2 = o;
+    o += TcCfg<FMT>::kNchHid * kChunkBytesN32;
+    L.w3 = o;
+    o += TcCfg<FMT>::kNchHid * kChunkBytesN32;
+    L.w4 = o;
+    o += TcCfg<FMT>::kNchOut * kChunkBytesN16;
+    o = (o + 1023u) & ~1023u;
+    L.b1 = o;
+    o += (uint32_t)n_l1_tables * l1_table_bytes;
+    o = (o + 15u) & ~15u;
+    L.stage = o;
+    o += (uint32_t)ng * stage_bytes_per_group;
+    o = (o + 7u) & ~7u;
+    L.bars = o;
+    o += 8u * (uint32_t)ng;
+    L.tmem_slot = o;
+    o += 16;
+    L.total = o;
+    return L;
+}
+
+// ---------------------------------------------------------------------------
+// fused search
+// ---------------------------------------------------------------------------
+template <int FMT, int NG>
+__global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
+                                                               const __grid_constant__ TcParams TP,
+                                                               const float* __restrict__ w1b1, Scratch* S) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    using C = TcCfg<FMT>;
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, NG, 0);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
+
+    const int tid = threadIdx.x, warp = tid >> 5, g = warp >> 2, wq = warp & 3;
+
+    // weights -> shared (generic proxy), then make them visible to the tensor core (async proxy)
+    {
+        const int4* src = reinterpret_cast<const int4*>(TP.blob);
+        int4* dst = reinterpret_cast<int4*>(smem);
+        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+    }
+    build_b1_fused<FMT>(P, w1b1, TP.l1_scale, smem + L.b1);
+    if (tid == 0) {
+        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        mbar_fence_init();
+    }
+    if (warp == 0) {
+        tmem_alloc(tmem_slot, 512);
+        tmem_relinquish();
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tbase = *tmem_slot;
+
+    const uint32_t col = (uint32_t)g * 64u;
+    const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
+    const uint32_t tD = tbase + col, tA1 = tbase + col + 32, tA = tbase + col + 40, tC = tbase + col + 56;
+    {
+        uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
+        tmem_st8(tC + lane_off, c8);
+        tmem_wait_st();
+    }
+    const bool leader = (tid & 127) == 0;
+    const uint32_t r = (uint32_t)(tid & 127);
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t w2a = sbase + L.w2, w3a = sbase + L.w3, w4a = sbase + L.w4, b1a = sbase + L.b1;
+    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
+    uint64_t* bar = &bars[g];
+    uint32_t phase = 0;
+
+    unsigned long long best = 0;
+    float best_y = __int_as_float(0x7fc00000);
+    for (uint64_t w = (uint64_t)blockIdx.x * NG + g; w < P.n_tiles; w += (uint64_t)gridDim.x * NG) {
+        const int s = find_segment(P, w);
+        const SegP& sg = P.seg[s];
+        const uint64_t ub = sg.u_begin + (w - sg.tile0) * kTileM;
+        const bool valid = ub + r < sg.u_end;
+        uint32_t v[kKMax];
+        decode_box<kKMax>(sg, ub, r, v);
+
+        // a3 (fused): layer-1 operand row [1, 1, v0_hi, v0_lo, ..., v3_hi, v3_lo, 0...]
+        {
+            uint32_t a[8];
+            a[0] = C::kOne2;
+#pragma unroll
+            for (int j = 0; j < kKMax; j++) a[1 + j] = pack2<FMT>((float)(v[j] >> 8), (float)(v[j] & 255u));
+            a[5] = a[6] = a[7] = 0;
+            tmem_st8(tA1 + lane_off, a);
+            tmem_wait_st();
+        }
+        // layer 1
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            const uint32_t bs = b1a + (uint32_t)s * C::kNchL1 * kChunkBytesN32;
+            mma_ts(tD, tA1, smem_desc(bs), id32, 0u);
+            if (C::kNchL1 > 1) mma_ts(tD, tA1, smem_desc(bs + kChunkBytesN32), id32, 1u);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        // layer 2
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w2a, kChunkBytesN32, id32);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        // layer 3
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w3a, kChunkBytesN32, id32);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        // output layer (N = 16, column 0 = y)
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w4a, kChunkBytesN16, id16);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        uint32_t ybits;
+        tmem_ld1(tD + lane_off, ybits);
+        const float y = __uint_as_float(ybits);
+
+        // a5: headroom mask + key
+        uint64_t idx = sg.t_base;
+        int32_t sum_n = sg.n_base;
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) {
+            idx += (uint64_t)v[j] * sg.istride[j];
+            sum_n += (int32_t)v[j];
+        }
+        if (valid && idx == 0) S->y0 = y;
+        if (valid && y <= P.H) {
+            const unsigned long long key = ((unsigned long long)(sum_n + 1) << 40) | idx;
+            if (key > best) {
+                best = key;
+                best_y = y;
+            }
+        }
+        fence_before();  // order this tile's TMEM reads before the next tile's writes/MMAs
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    if (warp == 0) tmem_dealloc(tbase, 512);
+    cta_publish_and_finish(P, S, best, best_y);
+}
+
+// ---------------------------------------------------------------------------
+// standalone predictor: rows from HBM
+//   A1 row = [x_hi (D values), x_lo (D values), 1, 1, 0...], x = 256 x_hi + x_lo
+//   B1     = [256 W1 | W1 | b1_hi | b1_lo]  (bf16: second set of chunks = lo halves)
+// ---------------------------------------------------------------------------
+template <int FMT>
+__device__ void build_b1_predict(const float* __restrict__ w1b1, int D, float scale, uint8_t* s_b1, int nch) {
+    const float* b1 = w1b1 + kHidden * D;
+    const int K = nch * 16;
+    for (int e = threadIdx.x; e < kHidden * K; e += blockDim.x) {
+        const int n = e / K, k = e % K;
+        uint16_t v0 = 0, v1 = 0;
+        if (k < 2 * D) {
+            const float w = w1b1[n * D + (k % D)] * scale;
+            const float m = k < D ? 256.0f : 1.0f;
+            uint16_t h, l;
+            split16<FMT>(w, h, l);
+            if (FMT == 0) {
+                v0 = to16<FMT>(w * m);
+            } else {
+                v0 = to16<FMT>(from16<FMT>(h) * m);
+                v1 = to16<FMT>(from16<FMT>(l) * m);
+            }
+        } else if (k < 2 * D + 2) {
+            uint16_t h, l;
+            split16<FMT>(b1[n] * scale, h, l);
+            v0 = k == 2 * D ? h : l;
+        }
+        const int ch = k >> 4, kk = k & 15;
+        *reinterpret_cast<uint16_t*>(s_b1 + (size_t)ch * kChunkBytesN32 + b_offset(n, kk)) = v0;
+        if (FMT == 1)
+            *reinterpret_cast<uint16_t*>(s_b1 + (size_t)(nch + ch) * kChunkBytesN32 + b_offset(n, kk)) = v1;
+    }
+}
+
+template <int FMT, int NG>
+__global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_constant__ TcParams TP,
+                                                                 const float* __restrict__ w1b1, int32_t D,
+                                                                 const int16_t* __restrict__ x, uint64_t count,
+                                                                 float* __restrict__ y) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    using C = TcCfg<FMT>;
+    const int nch = (2 * D + 2 + 15) / 16;                 // layer-1 K chunks (A1 columns = 8 nch)
+    const uint32_t stage_bytes = (uint32_t)(kTileM * D * 2 + 15) & ~15u;
+    const TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, NG, stage_bytes);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
+    const int tid = threadIdx.x, warp = tid >> 5, g = warp >> 2, wq = warp & 3;
+
+    {
+        const int4* src = reinterpret_cast<const int4*>(TP.blob);
+        int4* dst = reinterpret_cast<int4*>(smem);
+        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+    }
+    build_b1_predict<FMT>(w1b1, D, TP.l1_scale, smem + L.b1, nch);
+    if (tid == 0) {
+        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        mbar_fence_init();
+    }
+    if (warp == 0) {
+        tmem_alloc(tmem_slot, 512);
+        tmem_relinquish();
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tbase = *tmem_slot;
+
+    // per group: D 32 cols, A1 8*nch cols (<= 48), A 16 cols, C 8 cols -> 128-column slice
+    const uint32_t col = (uint32_t)g * 128u;
+    const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
+    const uint32_t tD = tbase + col, tA1 = tbase + col + 32, tA = tbase + col + 32 + 8 * (uint32_t)nch;
+    const uint32_t tC = tA + 16;
+    {
+        uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
+        tmem_st8(tC + lane_off, c8);
+        tmem_wait_st();
+    }
+    const bool leader = (tid & 127) == 0;
+    const uint32_t r = (uint32_t)(tid & 127);
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t w2a = sbase + L.w2, w3a = sbase + L.w3, w4a = sbase + L.w4, b1a = sbase + L.b1;
+    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
+    uint64_t* bar = &bars[g];
+    int16_t* stage = reinterpret_cast<int16_t*>(smem + L.stage + (uint32_t)g * stage_bytes);
+    uint32_t phase = 0;
+    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+
+    for (uint64_t w = (uint64_t)blockIdx.x * NG + g; w < n_tiles; w += (uint64_t)gridDim.x * NG) {
+        const uint64_t row0 = w * kTileM;
+        const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
+        // stage the tile's rows (contiguous bytes) with 16-byte loads
+        {
+            const uint32_t nbytes = nrows * (uint32_t)D * 2u;
+            const char* src = reinterpret_cast<const char*>(x + row0 * (uint64_t)D);
+            if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+                for (uint32_t i = r; i < nbytes / 16; i += 128)
+                    reinterpret_cast<int4*>(stage)[i] = __ldg(reinterpret_cast<const int4*>(src) + i);
+                for (uint32_t i = (nbytes / 16) * 16 + r; i < nbytes; i += 128)
+                    reinterpret_cast<char*>(stage)[i] = src[i];
+            } else {
+                for (uint32_t i = r; i < nbytes / 2; i += 128) stage[i] = x[row0 * (uint64_t)D + i];
+            }
+        }
+        named_bar_sync(1 + g, 128);
+        // A1 row from the staged features
+        const int16_t* row = stage + (size_t)min(r, nrows - 1) * D;
+        for (int cb = 0; cb < nch; cb++) {
+            uint32_t a[8];
+#pragma unroll
+            for (int i = 0; i < 8; i++) {
+                float v2[2];
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const int k = cb * 16 + 2 * i + h;
+                    float val = 0.0f;
+                    if (k < D) val = (float)(row[k] >> 8);
+                    else if (k < 2 * D) val = (float)(row[k - D] & 255);
+                    else if (k < 2 * D + 2) val = 1.0f;
+                    v2[h] = val;
+                }
+                a[i] = pack2<FMT>(v2[0], v2[1]);
+            }
+            tmem_st8(tA1 + lane_off + 8 * cb, a);
+        }
+        tmem_wait_st();
+        fence_before();
+        named_bar_sync(1 + g, 128);  // also: every thread done reading `stage`
+        if (leader) {
+            fence_after();
+            for (int cb = 0; cb < nch; cb++)
+                mma_ts(tD, tA1 + 8 * cb, smem_desc(b1a + cb * kChunkBytesN32), id32, cb > 0 ? 1u : 0u);
+            if (FMT == 1)
+                for (int cb = 0; cb < nch; cb++)
+                    mma_ts(tD, tA1 + 8 * cb, smem_desc(b1a + (nch + cb) * kChunkBytesN32), id32, 1u);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w2a, kChunkBytesN32, id32);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w3a, kChunkBytesN32, id32);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        if (leader) {
+            fence_after();
+            issue_layer<FMT>(tD, tA, tC, w4a, kChunkBytesN16, id16);
+            mma_commit(bar);
+        }
+        mbar_wait(bar, phase);
+        phase ^= 1u;
+        fence_after();
+        uint32_t ybits;
+        tmem_ld1(tD + lane_off, ybits);
+        if (r < nrows) y[row0 + r] = __uint_as_float(ybits);
+        fence_before();
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    if (warp == 0) tmem_dealloc(tbase, 512);
+}
+
+// ---------------------------------------------------------------------------
+// launchers
+// ---------------------------------------------------------------------------
+constexpr int kFusedNG = 4;
+constexpr int kPredictNG = 4;
+
+template <int FMT>
+static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const float* w1b1, Scratch* S, int nsm,
+                                    cudaStream_t st, int* grid_out) {
+    using C = TcCfg<FMT>;
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, kFusedNG, 0);
+    auto kern = fused_tc_kernel<FMT, kFusedNG>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    if (e != cudaSuccess) return e;
+    uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
+    if (g > (uint64_t)nsm) g = (uint64_t)nsm;
+    if (g < 1) g = 1;
+    *grid_out = (int)g;
+    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, w1b1, S);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
+                            cudaStream_t st, int* grid_out) {
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    if (TW.fmt == 0) return launch_fused_fmt<0>(P, tp, w1b1, S, nsm, st, grid_out);
+    return launch_fused_fmt<1>(P, tp, w1b1, S, nsm, st, grid_out);
+}
+
+template <int FMT>
+static cudaError_t launch_predict_fmt(const TcParams& tp, const float* w1b1, int32_t D, const int16_t* x,
+                                      uint64_t count, float* y, int nsm, cudaStream_t st) {
+    const int nch = (2 * D + 2 + 15) / 16;
+    const uint32_t stage_bytes = (uint32_t)(kTileM * D * 2 + 15) & ~15u;
+    const TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, kPredictNG, stage_bytes);
+    auto kern = predict_tc_kernel<FMT, kPredictNG>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    if (e != cudaSuccess) return e;
+    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    uint64_t g = (n_tiles + kPredictNG - 1) / kPredictNG;
+    if (g > (uint64_t)nsm) g = (uint64_t)nsm;
+    if (g < 1) g = 1;
+    kern<<<(int)g, kPredictNG * 128, L.total, st>>>(tp, w1b1, D, x, count, y);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
+                              float* y, int nsm, cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    if (D > 40) return cudaErrorInvalidValue;  // A1 slice (8 nch <= 48 columns) of a 128-column group
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    if (TW.fmt == 0) return launch_predict_fmt<0>(tp, w1b1, D, x, count, y, nsm, st);
+    return launch_predict_fmt<1>(tp, w1b1, D, x, count, y, nsm, st);
+}
+
+}  // namespace abacus

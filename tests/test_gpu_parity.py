@@ -1,0 +1,316 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Bars (BASELINE.json north_star): enumeration / encoding / indices bit-exact;
+predicted latencies within 1e-4 relative (fp32 path) and 1e-2 relative
+(tensor-core paths); selections identical except where the oracle's margin to
+the headroom is below that tolerance (reading c18: accept the GPU key iff
+maxkey_strict <= key <= maxkey_loose and y64(t_gpu) <= H + eps|H|).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from oracle import brute
+import paper_conf_sc_cui0czlzsmylg21_b200 as ab
+from gpu_util import EPS, NAMES, Ctx, accept_key, rel_err
+from oracle_helpers import LinearPredictor, load_fig12, offsets, unit0_params, zero_params
+
+pytestmark = pytest.mark.gpu
+PRECS = [ab.ABACUS_FP32, ab.ABACUS_FP16, ab.ABACUS_BF16]
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_FP32)
+    yield c
+    c.close()
+
+
+# ------------------------------------------------------------------ encode --
+def test_encode_cfg1_bit_exact(ctx):
+    for b, slots in synth.cfg1_grids():
+        T = oracle.grid_size(slots)
+        _, _, x64, _ = oracle.sweep(ctx.params, slots, 0.0, want_x=True)
+        x = ctx.encode(slots, 0, T)
+        assert np.array_equal(x, x64), b
+
+
+def test_encode_ragged_ranges_bit_exact(ctx):
+    rng = np.random.default_rng(3)
+    for slots in synth.tiny_grids(40, seed=31, max_len=9):
+        T = oracle.grid_size(slots)
+        first = int(rng.integers(0, T))
+        count = int(rng.integers(0, T - first + 1))
+        _, _, x64, _ = oracle.sweep(ctx.params, slots, 0.0, first=first, count=count, want_x=True)
+        x = ctx.encode(slots, first, count)
+        assert np.array_equal(x, x64)
+
+
+def test_encode_cfg4_sampled_ranges(ctx):
+    """Full-size grid (9,188,218,208 candidates): sampled windows incl. the tail."""
+    slots = synth.cfg4_grid()
+    T = oracle.grid_size(slots)
+    assert T == 9_188_218_208
+    rng = np.random.default_rng(4)
+    for first in [0, T - 3000] + [int(v) for v in rng.integers(0, T - 3000, size=6)]:
+        _, _, x64, _ = oracle.sweep(ctx.params, slots, 0.0, first=first, count=3000, want_x=True)
+        assert np.array_equal(ctx.encode(slots, first, 3000), x64)
+
+
+def test_encode_groups_bit_exact(ctx):
+    groups = synth.instance_samples(20000, seed=15)
+    G = [g.slots for g in groups]
+    x64 = oracle.encode_groups(8, 4, G)
+    x, bad = ctx.encode_groups(G)
+    assert bad == 0 and np.array_equal(x, x64)
+    x, bad = ctx.encode_groups([[(3, 1, 2, 4, 0), (3, 2, 5, 4, 0)], [(2, 1, 9, 8, 0)]])
+    assert bad == 1 and not x[0].any() and np.array_equal(x[1], oracle.encode(8, 4, [(2, 1, 9, 8, 0)]))
+
+
+# ----------------------------------------------------------------- predict --
+def _dyadic24():
+    d = 24
+    p = zero_params(d)
+    o = offsets(d)
+    for (i, j), v in {(0, 0): 1.0, (0, 1): 2.0, (1, 0): -1.0, (1, 1): 0.5}.items():
+        p[o["W1"] + i * d + j] = v
+    p[o["b1"] + 0], p[o["b1"] + 1] = 0.5, 1.0
+    for (i, j), v in {(0, 0): 2.0, (0, 1): 4.0, (1, 0): -1.0, (2, 0): 0.25}.items():
+        p[o["W2"] + i * 32 + j] = v
+    p[o["b2"] + 0], p[o["b2"] + 1] = -1.0, 0.25
+    for (i, j), v in {(0, 0): 0.5, (0, 2): 2.0, (1, 0): -1.0, (5, 2): -2.0}.items():
+        p[o["W3"] + i * 32 + j] = v
+    p[o["b3"] + 0], p[o["b3"] + 1], p[o["b3"] + 5] = 0.25, 3.0, 3.0
+    p[o["w4"] + 0], p[o["w4"] + 1], p[o["w4"] + 5] = 1.5, 7.0, 4.0
+    p[o["b4"]] = -2.0
+    return p
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_predict_dyadic_exact(prec):
+    """Hand-computed y = 11 (tests/test_oracle_pins.py::test_dyadic_mlp_hand_computed)."""
+    c = Ctx(params=_dyadic24(), precision=prec)
+    try:
+        X = np.zeros((300, 24), dtype=np.int16)
+        X[:, 0], X[:, 1] = 3, 1
+        assert np.all(c.predict(X) == 11.0)
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", PRECS)
+@pytest.mark.parametrize("variant", ["shaped", "raw"])
+def test_predict_cfg5_tolerance(prec, variant):
+    params = synth.weights(1, variant)
+    c = Ctx(params=params, precision=prec)
+    try:
+        groups = synth.instance_samples(100_003, seed=15)
+        X = oracle.encode_groups(8, 4, [g.slots for g in groups])
+        y64 = oracle.mlp64_batch(params, X)
+        y = c.predict(X)
+        # raw init: outputs cancel towards 0 (w4 of both signs), so the error is
+        # measured against the magnitude of the summed terms |b4| + sum|w4 h3|
+        # (reading c19); shaped weights: plain relative error (y >= 2 ms)
+        floor = output_term_magnitude(params, X) if variant == "raw" else None
+        err = rel_err(y, y64, floor)
+        print(NAMES[prec], variant, "max rel err %.3e p99 %.3e" % (err.max(), np.quantile(err, 0.99)))
+        assert err.max() <= EPS[prec]
+    finally:
+        c.close()
+
+
+def output_term_magnitude(params, X):
+    """|b4| + sum_j |w4_j h3_j(x)| in fp64 (normalisation only, not a reference)."""
+    W1, b1, W2, b2, W3, b3, w4, b4 = [a.astype(np.float64) for a in synth.split_params(params)]
+    h = np.maximum(X.astype(np.float64) @ W1.T + b1, 0)
+    h = np.maximum(h @ W2.T + b2, 0)
+    h = np.maximum(h @ W3.T + b3, 0)
+    return np.abs(b4[0]) + h @ np.abs(w4)
+
+
+# ------------------------------------------------------------------ select --
+def test_select_matches_fp32_decisions(ctx):
+    """y and H in fp32 on both sides (the comparison decides an integer)."""
+    for b, slots in synth.cfg1_grids():
+        _, y64, _, ope = oracle.sweep(ctx.params, slots, 0.0, want_y=True, want_ope=True)
+        y32 = y64.astype(np.float32)
+        for q in (0.1, 0.5, 0.9):
+            H = np.float32(np.quantile(y32, q))
+            sn = np.array([brute.sum_n(slots, o) for o in ope])
+            feas = np.nonzero(y32 <= H)[0]
+            want = int(max(((int(sn[t]) + 1) << 40) | int(t) for t in feas)) if len(feas) else 0
+            assert ctx.select(slots, 0, y32, float(H)) == want
+            # running max semantics over two shards
+            T = len(y32)
+            k1 = ctx.select(slots, 0, y32[: T // 3], float(H))
+            assert ctx.select(slots, T // 3, y32[T // 3:], float(H), init=k1) == want
+
+
+# ------------------------------------------------------------ fused search --
+def _check_sweep(c, slots, H, first=0, count=None, eps=None):
+    T = oracle.grid_size(slots)
+    count = T - first if count is None else count
+    eps = EPS[c.precision] if eps is None else eps
+    d = ab.abacus_search_grid(c.h, ab.make_grid(slots), H, first, count)
+    r, _, _, _ = oracle.sweep(c.params, slots, H, first=first, count=count, eps=eps)
+    assert d.evaluated == count
+    assert accept_key(d.key, r.maxkey_strict, r.maxkey_loose), (d.key, r.maxkey_strict, r.maxkey_loose)
+    if d.key:
+        assert d.status == ab.ABACUS_DECIDE_OK
+        _, yt, _, ope = oracle.sweep(c.params, slots, H, first=d.index, count=1, want_y=True, want_ope=True)
+        assert yt[0] <= H + eps * abs(H)
+        assert abs(d.pred_ms - yt[0]) <= eps * abs(yt[0]) + 1e-6
+        assert list(d.end_op)[:len(slots)] == list(ope[0])
+        assert d.total_ops == brute.sum_n(slots, ope[0])
+    else:
+        assert d.status == ab.ABACUS_DECIDE_NONE
+    return d
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_search_grid_cfg1(prec):
+    c = Ctx(params=synth.weights(1), precision=prec)
+    try:
+        for b, slots in synth.cfg1_grids():
+            _, y64, _, _ = oracle.sweep(c.params, slots, 0.0, want_y=True)
+            Hs = [float(np.float32(np.quantile(y64, q))) for q in (0.1, 0.5, 0.9)]
+            Hs.append(float(np.float32(y64[len(y64) // 2])))   # an exact prediction: tests '<='
+            Hs.append(float(np.float32(y64.min() - 1.0)))       # nothing fits
+            for H in Hs:
+                _check_sweep(c, slots, H)
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_search_grid_ragged_shards(prec):
+    c = Ctx(params=synth.weights(1), precision=prec)
+    rng = np.random.default_rng(9)
+    try:
+        for slots in synth.tiny_grids(25, seed=41, max_len=40):
+            T = oracle.grid_size(slots)
+            _, y64, _, _ = oracle.sweep(c.params, slots, 0.0, want_y=True)
+            H = float(np.float32(np.quantile(y64, rng.uniform(0.05, 0.95))))
+            full = _check_sweep(c, slots, H)
+            G = int(rng.integers(2, 6))
+            keys = []
+            for r in range(G):
+                first, count = ab.shard_range(T, r, G)
+                keys.append(_check_sweep(c, slots, H, first, count).key)
+            assert max(keys) == full.key
+    finally:
+        c.close()
+
+
+def test_search_grid_deterministic(ctx):
+    slots = synth.cfg1_grids()[2][1]
+    T = oracle.grid_size(slots)
+    for prec in PRECS:
+        ctx.load(ctx.params, prec)
+        ds = [ab.abacus_search_grid(ctx.h, ab.make_grid(slots), 15.0, 0, T) for _ in range(4)]
+        assert len({(d.key, d.pred_ms) for d in ds}) == 1
+    ctx.load(ctx.params, ab.ABACUS_FP32)
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_search_grid_cfg4_fullsize_linear_closed_form(prec):
+    """9.19e9 candidates at the launch configuration the bench times; a linear
+    ReLU-transparent predictor makes the answer a closed form (knapsack)."""
+    lp = LinearPredictor(8, 4, c0=2.0, beta=[0.5, 1.25, 0.75, 1.0, 0.25, 0.5, 1.5, 2.0],
+                         a=[0.125, 0.25, 0.375, 0.5])
+    slots = synth.cfg4_grid()
+    T = oracle.grid_size(slots)
+    c = Ctx(params=lp.params(), precision=prec)
+    try:
+        for H in (150.5, 333.25):
+            d = ab.abacus_search_grid(c.h, ab.make_grid(slots), H, 0, T)
+            assert d.evaluated == T
+            if prec == ab.ABACUS_FP32:
+                nstar, tstar = lp.best(slots, H)
+                assert d.index == tstar and d.total_ops == nstar
+                assert d.key == ((nstar + 1) << 40) | tstar
+            else:
+                eps = EPS[prec]
+                ns, ts = lp.best(slots, H * (1 - eps))
+                nl, tl = lp.best(slots, H * (1 + eps))
+                assert ((ns + 1) << 40) | ts <= d.key <= ((nl + 1) << 40) | tl
+            _, _, _, ope = oracle.sweep(c.params, slots, H, first=d.index, count=1, want_ope=True)
+            assert lp.predict(slots, ope[0]) <= H * (1 + EPS[prec])
+    finally:
+        c.close()
+
+
+# --------------------------------------------------------------- decisions --
+@pytest.mark.parametrize("prec", PRECS)
+@pytest.mark.parametrize("space", [ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN, ab.ABACUS_SPACE_AUTO])
+def test_decisions_cfg2(prec, space):
+    c = Ctx(params=synth.weights(1), precision=prec)
+    eps = EPS[prec]
+    try:
+        for qs, now, infl in synth.cfg2_decisions(60):
+            d = ab.abacus_search(c.h, qs, now, infl, space, 20_000)
+            od = oracle.search(c.params, qs, now, infl, space=space, budget=20_000, eps=eps)
+            assert d.critical == od.critical and list(d.order)[:3] == list(od.order)[:3]
+            assert d.headroom_ms == np.float32(od.headroom_ms)
+            assert d.evaluated == od.evaluated
+            assert abs(d.pred_critical_only_ms - od.pred_critical_only_ms) <= eps * abs(od.pred_critical_only_ms)
+            near = abs(od.pred_critical_only_ms - od.headroom_ms) <= eps * abs(od.headroom_ms)
+            if not near:
+                assert d.status == od.status
+            if d.status == ab.ABACUS_DECIDE_OK and od.status == ab.ABACUS_DECIDE_OK:
+                assert accept_key(d.key, od.maxkey_strict, od.maxkey_loose)
+                assert d.total_ops == (d.key >> 40) - 1
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", PRECS)
+@pytest.mark.parametrize("space", [ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN])
+def test_fig12_replay_on_gpu(prec, space):
+    """q3 fully, q2 fully, first two ops of q1; y = H = 25 ms."""
+    f = load_fig12()
+    d_feat = f["n_models"] + 16
+    p = unit0_params(d_feat, f["unit0"]["bias"], {int(k): v for k, v in f["unit0"]["coef"].items()})
+    c = Ctx(ops=f["ops_per_model"], params=p, precision=prec)
+    try:
+        qs = [synth.Query(q["model_id"], q["next_op"], 1, 0, q["headroom_ms"], 0.0) for q in f["queries"]]
+        d = ab.abacus_search(c.h, qs, 0.0, 0.0, space)
+        names = [q["name"] for q in f["queries"]]
+        assert d.status == ab.ABACUS_DECIDE_OK
+        assert names[d.critical] == f["expected"]["critical"]
+        assert {names[i]: d.end_op[i] for i in range(3)} == f["expected"]["end_op"]
+        assert d.pred_ms == f["expected"]["pred_ms"]
+        assert d.index == (f["expected"]["grid_t"] if space == 0 else f["expected"]["chain_u"])
+    finally:
+        c.close()
+
+
+def test_validation_errors():
+    c = Ctx()
+    try:
+        g = [synth.GridSlot(1, 1, 8, 0, 1, 10, 1), synth.GridSlot(1, 1, 8, 0, 1, 10, 1)]
+        with pytest.raises(ab.AbacusError) as e:
+            ab.abacus_search_grid(c.h, ab.make_grid(g[:1]), 1.0, 0, 1)
+        assert e.value.code == ab.ABACUS_E_NOT_LOADED
+        c.load(synth.weights(1), ab.ABACUS_FP32)
+        with pytest.raises(ab.AbacusError) as e:
+            ab.abacus_search_grid(c.h, ab.make_grid(g), 1.0, 0, 1)
+        assert e.value.code == ab.ABACUS_E_DUP_MODEL
+        for bad in [synth.GridSlot(9, 1, 8, 0, 1, 2, 1), synth.GridSlot(1, 3, 8, 0, 2, 5, 1),
+                    synth.GridSlot(1, 1, 8, 0, 1, 123, 1), synth.GridSlot(1, 1, 0, 0, 1, 2, 1)]:
+            with pytest.raises(ab.AbacusError) as e:
+                ab.abacus_search_grid(c.h, ab.make_grid([bad]), 1.0, 0, 1)
+            assert e.value.code == ab.ABACUS_E_INVALID
+        with pytest.raises(ab.AbacusError):
+            ab.abacus_search_grid(c.h, ab.make_grid(g[:1]), 1.0, 5, 100)   # beyond T
+        with pytest.raises(ab.AbacusError) as e:
+            ab.abacus_load_predictor(c.h, np.zeros(10, dtype=np.float32), ab.ABACUS_FP32)
+        assert e.value.code == ab.ABACUS_E_INVALID
+        qs = [synth.Query(2, 5, 8, 0, 30.0, 0.0), synth.Query(2, 7, 8, 0, 30.0, 0.0)]
+        with pytest.raises(ab.AbacusError) as e:
+            ab.abacus_search(c.h, qs, 0.0, 0.0)
+        assert e.value.code == ab.ABACUS_E_DUP_MODEL
+    finally:
+        c.close()
