@@ -21,6 +21,95 @@ __device__ __forceinline__ int find_segment(const Plan& P, uint64_t w) {
 }
 
 // ---------------------------------------------------------------------------
+// Tile walker: a worker (thread row r of a persistent group) walks a
+// contiguous range of tiles [wb, we) of the plan.  The segment state lives in
+// registers and the box digits v[] of its candidate advance by kTileM per tile
+// with a carry chain, so the per-tile enumeration cost is a few integer ops;
+// the slow decode (fp64 split of the tile base) runs only on entry and at
+// segment boundaries.
+// ---------------------------------------------------------------------------
+struct Walker {
+    uint64_t ub;          // box ordinal of the tile's row 0
+    uint64_t u_end;       // segment end (box ordinal)
+    uint64_t next_tile0;  // first work item of the next segment
+    uint64_t t_base;
+    uint64_t istride[kKMax];
+    uint32_t cnt[kKMax];
+    FastDiv fd[kKMax];
+    int32_t n_base;
+    int32_t s;            // segment index
+    uint32_t v[kKMax];    // digits of this row's candidate
+};
+
+__device__ __forceinline__ void walker_enter(const Plan& P, Walker& W, int s, uint64_t w, uint32_t r) {
+    const SegP& g = P.seg[s];
+    W.s = s;
+    W.u_end = g.u_end;
+    W.next_tile0 = s + 1 < P.n_seg ? P.seg[s + 1].tile0 : ~0ull;
+    W.t_base = g.t_base;
+    W.n_base = g.n_base;
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) {
+        W.istride[j] = g.istride[j];
+        W.cnt[j] = g.cnt[j];
+        W.fd[j] = g.fd[j];
+    }
+    W.ub = g.u_begin + (w - g.tile0) * kTileM;
+    decode_box<kKMax>(g, W.ub, r, W.v);
+}
+
+__device__ __forceinline__ void walker_begin(const Plan& P, Walker& W, uint64_t w, uint32_t r) {
+    walker_enter(P, W, find_segment(P, w), w, r);
+}
+
+// move to work item w + 1
+__device__ __forceinline__ void walker_next(const Plan& P, Walker& W, uint64_t w_next, uint32_t r) {
+    if (w_next == W.next_tile0) {
+        walker_enter(P, W, W.s + 1, w_next, r);
+        return;
+    }
+    W.ub += kTileM;
+    uint32_t carry = kTileM;
+#pragma unroll
+    for (int j = kKMax - 1; j >= 0; j--) {
+        const uint32_t x = W.v[j] + carry;
+        const uint32_t q = fastdiv(x, W.fd[j]);
+        W.v[j] = x - q * W.cnt[j];
+        carry = q;
+    }
+}
+
+// contiguous work range of worker group `gid` out of `ngroups`
+__device__ __forceinline__ void work_range(uint64_t n_tiles, uint64_t gid, uint64_t ngroups, uint64_t& wb,
+                                           uint64_t& we) {
+    const uint64_t per = n_tiles / ngroups, extra = n_tiles % ngroups;
+    wb = gid * per + (gid < extra ? gid : extra);
+    we = wb + per + (gid < extra ? 1 : 0);
+}
+
+// fold one evaluated candidate into the running best (key built lazily)
+__device__ __forceinline__ void fold_candidate(const Walker& W, bool valid, float y, float H,
+                                               unsigned long long& best, float& best_y) {
+    if (valid && y <= H) {
+        const uint32_t hi = (uint32_t)(W.n_base + (int32_t)(W.v[0] + W.v[1] + W.v[2] + W.v[3]) + 1);
+        if (hi >= (uint32_t)(best >> 40)) {
+            uint64_t idx = W.t_base;
+#pragma unroll
+            for (int j = 0; j < kKMax; j++) idx += (uint64_t)W.v[j] * W.istride[j];
+            const unsigned long long key = ((unsigned long long)hi << 40) | idx;
+            if (key > best) {
+                best = key;
+                best_y = y;
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ bool walker_is_index0(const Walker& W, uint32_t r) {
+    return W.t_base == 0 && W.ub == 0 && r == 0;
+}
+
+// ---------------------------------------------------------------------------
 // Last-CTA epilogue shared by the fused kernels (a5 cross-CTA + a7 decode).
 // Each CTA publishes its best (key, y); the last CTA to arrive reduces them,
 // decodes the winning index into end ops per slot and resets the ticket.

@@ -229,8 +229,8 @@ __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_consta
 }
 
 // ---------------------------------------------------------------------------
-// a2..a5 fused, fp32 SIMT path.  Persistent blocks of 256 threads = two
-// 128-candidate tiles per iteration.  Layer 1 is evaluated per segment as
+// a2..a5 fused, fp32 SIMT path.  Persistent blocks of 128 threads, one
+// 128-candidate tile per iteration.  Layer 1 is evaluated per segment as
 //     z1 = c_P + sum_j v_j * w_P,j
 // where c_P = b1 + W1 x0_P (x0_P: the Fig.-8 vector of the segment's v = 0
 // group) and w_P,j = W1[:, N + 4 pos_P(j) + 1] (the ope column of slot j at its
@@ -238,7 +238,8 @@ __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_consta
 // digits, so this is W1 x + b1 exactly (up to fp32 rounding order).  The
 // per-segment tables are built in the prologue, on device, from fp32 W1/b1.
 // ---------------------------------------------------------------------------
-constexpr int kFusedThreads = 256;
+constexpr int kFusedThreads = 128;
+constexpr int kFusedBlocksPerSM = 3;
 
 __device__ void build_l1_tables(const Plan& P, const float* __restrict__ w1b1, float* s_c, float* s_w) {
     // s_c[s][32], s_w[s][4][32]
@@ -268,49 +269,38 @@ __device__ void build_l1_tables(const Plan& P, const float* __restrict__ w1b1, f
     }
 }
 
-__global__ void __launch_bounds__(kFusedThreads, 2) fused_fp32_kernel(const __grid_constant__ Plan P,
-                                                                      const __grid_constant__ W234 W,
+__global__ void __launch_bounds__(kFusedThreads, kFusedBlocksPerSM) fused_fp32_kernel(const __grid_constant__ Plan P,
+                                                                      const __grid_constant__ W234 Wt,
                                                                       const float* __restrict__ w1b1, Scratch* S) {
     __shared__ float s_c[kMaxSeg * kHidden];
     __shared__ float s_w[kMaxSeg * kKMax * kHidden];
     build_l1_tables(P, w1b1, s_c, s_w);
     __syncthreads();
 
-    const uint32_t r = threadIdx.x & (kTileM - 1);
-    const uint64_t half = threadIdx.x >> 7;
+    const uint32_t r = threadIdx.x;
     unsigned long long best = 0;
     float best_y = __int_as_float(0x7fc00000);
-    for (uint64_t w = (uint64_t)blockIdx.x * 2 + half; w < P.n_tiles; w += (uint64_t)gridDim.x * 2) {
-        const int s = find_segment(P, w);
-        const SegP& g = P.seg[s];
-        const uint64_t ub = g.u_begin + (w - g.tile0) * kTileM;
-        const bool valid = ub + r < g.u_end;
-        uint32_t v[kKMax];
-        decode_box<kKMax>(g, ub, r, v);
-        const float* c = s_c + s * kHidden;
-        const float* wc = s_w + s * kKMax * kHidden;
+    uint64_t wb, we;
+    work_range(P.n_tiles, (uint64_t)blockIdx.x, (uint64_t)gridDim.x, wb, we);
+    Walker W;
+    if (wb < we) walker_begin(P, W, wb, r);
+    for (uint64_t w = wb; w < we; w++) {
+        if (w != wb) walker_next(P, W, w, r);
+        const bool valid = W.u_end - W.ub > (uint64_t)r;
+        const float* c = s_c + W.s * kHidden;
+        const float* wc = s_w + W.s * kKMax * kHidden;
         float h1[kHidden];
 #pragma unroll
         for (int i = 0; i < kHidden; i++) {
             float z = c[i];
 #pragma unroll
-            for (int j = 0; j < kKMax; j++) z = fmaf(wc[j * kHidden + i], (float)v[j], z);
+            for (int j = 0; j < kKMax; j++) z = fmaf(wc[j * kHidden + i], (float)W.v[j], z);
             h1[i] = fmaxf(z, 0.0f);
         }
         float y;
-        mlp_tail_fp32(W, h1, y);
-        uint64_t idx = g.t_base;
-        int32_t sum_n = g.n_base;
-#pragma unroll
-        for (int j = 0; j < kKMax; j++) {
-            idx += (uint64_t)v[j] * g.istride[j];
-            sum_n += (int32_t)v[j];
-        }
-        if (valid && idx == 0) S->y0 = y;
-        if (valid && y <= P.H) {
-            const unsigned long long key = ((unsigned long long)(sum_n + 1) << 40) | idx;
-            if (key > best) { best = key; best_y = y; }
-        }
+        mlp_tail_fp32(Wt, h1, y);
+        if (valid && walker_is_index0(W, r)) S->y0 = y;
+        fold_candidate(W, valid, y, P.H, best, best_y);
     }
     cta_publish_and_finish(P, S, best, best_y);
 }
@@ -376,9 +366,8 @@ cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const f
 
 cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,
                               cudaStream_t st, int* grid_out) {
-    const uint64_t pairs = (P.n_tiles + 1) / 2;
-    uint64_t g = (uint64_t)nsm * 2;
-    if (pairs < g) g = pairs;
+    uint64_t g = (uint64_t)nsm * kFusedBlocksPerSM;
+    if (P.n_tiles < g) g = P.n_tiles;
     if (g < 1) g = 1;
     *grid_out = (int)g;
     fused_fp32_kernel<<<(int)g, kFusedThreads, 0, st>>>(P, W, w1b1, S);

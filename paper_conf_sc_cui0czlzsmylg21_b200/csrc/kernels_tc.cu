@@ -56,11 +56,13 @@ __device__ __forceinline__ void split16(float v, uint16_t& hi, uint16_t& lo) {
 }
 
 // Layer-1 B operand per segment: rows n = hidden unit, K columns
-//   k0 = c_hi, k1 = c_lo, k(2+2j) = 256 w_j, k(3+2j) = w_j   (chunk 0)
-//   bf16: chunk 1 holds the lo halves of the w_j columns.
+//   k0 = c_hi, k1 = c_lo, then per slot j:
+//     SPLIT:   k(2+2j) = 256 w_j, k(3+2j) = w_j   (digit = 256 hi + lo)
+//     !SPLIT:  k(2+j)  = w_j                      (digit exact in the format)
+//   bf16: chunk 1 holds the lo halves of the w_j columns (weights split hi+lo).
 // c = b1 + W1 x0 (Fig.-8 vector of the segment's v = 0 group), w_j = the
 // W1 column of slot j's ope at its Fig.-8 position.
-template <int FMT>
+template <int FMT, bool SPLIT>
 __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, float scale, uint8_t* s_b1) {
     constexpr int NCH = TcCfg<FMT>::kNchL1;
     const int D = P.D;
@@ -89,11 +91,13 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
         uint8_t* base = s_b1 + (size_t)s * NCH * kChunkBytesN32;
         for (int k = 0; k < 16; k++) {
             uint16_t v0 = 0, v1 = 0;
+            int j = -1;
+            float m = 1.0f;
             if (k == 0) v0 = ch;
             else if (k == 1) v0 = cl;
-            else if (k < 2 + 2 * kKMax) {
-                const int j = (k - 2) >> 1;
-                const float m = ((k - 2) & 1) ? 1.0f : 256.0f;
+            else if (SPLIT && k < 2 + 2 * kKMax) { j = (k - 2) >> 1; m = ((k - 2) & 1) ? 1.0f : 256.0f; }
+            else if (!SPLIT && k < 2 + kKMax) { j = k - 2; }
+            if (j >= 0) {
                 uint16_t h, l;
                 split16<FMT>(wj[j], h, l);
                 if (FMT == 0) {
@@ -123,6 +127,38 @@ __device__ __forceinline__ void issue_layer(uint32_t tD, uint32_t tA, uint32_t t
         mma_ts(tD, tA, smem_desc(wbase + 2 * chunk_bytes), idesc, 1u);
         mma_ts(tD, tA + 8, smem_desc(wbase + 3 * chunk_bytes), idesc, 1u);
         mma_ts(tD, tC, smem_desc(wbase + 4 * chunk_bytes), idesc, 1u);
+    }
+}
+
+template <int FMT>
+__device__ __forceinline__ void issue_layer_e(uint32_t tD, uint32_t tA, uint32_t tC, const uint64_t* d,
+                                              uint32_t idesc) {
+    if (FMT == 0) {
+        mma_ts_elect(tD, tA, d[0], idesc, 0u);
+        mma_ts_elect(tD, tA + 8, d[1], idesc, 1u);
+        mma_ts_elect(tD, tC, d[2], idesc, 1u);
+    } else {
+        mma_ts_elect(tD, tA, d[0], idesc, 0u);
+        mma_ts_elect(tD, tA + 8, d[1], idesc, 1u);
+        mma_ts_elect(tD, tA, d[2], idesc, 1u);
+        mma_ts_elect(tD, tA + 8, d[3], idesc, 1u);
+        mma_ts_elect(tD, tC, d[4], idesc, 1u);
+    }
+}
+
+template <int FMT>
+__device__ __forceinline__ void issue_layer_p(uint32_t pred, uint32_t tD, uint32_t tA, uint32_t tC,
+                                              const uint64_t* d, uint32_t idesc) {
+    if (FMT == 0) {
+        mma_ts_p(pred, tD, tA, d[0], idesc, 0u);
+        mma_ts_p(pred, tD, tA + 8, d[1], idesc, 1u);
+        mma_ts_p(pred, tD, tC, d[2], idesc, 1u);
+    } else {
+        mma_ts_p(pred, tD, tA, d[0], idesc, 0u);
+        mma_ts_p(pred, tD, tA + 8, d[1], idesc, 1u);
+        mma_ts_p(pred, tD, tA, d[2], idesc, 1u);
+        mma_ts_p(pred, tD, tA + 8, d[3], idesc, 1u);
+        mma_ts_p(pred, tD, tC, d[4], idesc, 1u);
     }
 }
 
@@ -176,28 +212,56 @@ __host__ __device__ inline TcSmem tc_smem_layout(int n_l1_tables, uint32_t l1_ta
 
 // ---------------------------------------------------------------------------
 // fused search
+//
+// Each group keeps TWO tiles in flight (TMEM slots X and Y) and interleaves
+// them stage by stage: while the tensor core runs layer l of one tile, the
+// group's warps run the epilogue of the other.  Per group TMEM (128 columns):
+//   X: D [0,32)  A1 [32,40)  A [40,56)     Y: D [64,96)  A1 [96,104)  A [104,120)
+//   constant chunk [56,64) = (1, 1, 0, ...) for the bias columns
 // ---------------------------------------------------------------------------
-template <int FMT, int NG>
+struct TileIO {
+    uint32_t d, a1, a;  // TMEM addresses (column part; lane 0)
+};
+
+template <int FMT, bool SPLIT>
+__device__ __forceinline__ void store_a1(uint32_t taddr, const uint32_t (&v)[kKMax]) {
+    uint32_t a[8];
+    a[0] = TcCfg<FMT>::kOne2;
+    if (SPLIT) {
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) a[1 + j] = pack2<FMT>((float)(v[j] >> 8), (float)(v[j] & 255u));
+        a[5] = a[6] = a[7] = 0;
+    } else {
+        a[1] = pack2<FMT>((float)v[0], (float)v[1]);
+        a[2] = pack2<FMT>((float)v[2], (float)v[3]);
+        a[3] = a[4] = a[5] = a[6] = a[7] = 0;
+    }
+    tmem_st8(taddr, a);
+}
+
+template <int FMT, bool SPLIT, int NG>
 __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
                                                                const __grid_constant__ TcParams TP,
                                                                const float* __restrict__ w1b1, Scratch* S) {
     extern __shared__ __align__(1024) uint8_t smem[];
     using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, NG, 0);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * NG, 0);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);  // 2 per group
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
 
-    const int tid = threadIdx.x, warp = tid >> 5, g = warp >> 2, wq = warp & 3;
+    const int tid = threadIdx.x;
+    // warp-uniform indices (shfl from lane 0: the compiler keeps them uniform)
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+    const int g = warp >> 2, wq = warp & 3;
 
-    // weights -> shared (generic proxy), then make them visible to the tensor core (async proxy)
     {
         const int4* src = reinterpret_cast<const int4*>(TP.blob);
         int4* dst = reinterpret_cast<int4*>(smem);
         for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
     }
-    build_b1_fused<FMT>(P, w1b1, TP.l1_scale, smem + L.b1);
+    build_b1_fused<FMT, SPLIT>(P, w1b1, TP.l1_scale, smem + L.b1);
     if (tid == 0) {
-        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        for (int i = 0; i < 2 * NG; i++) mbar_init(&bars[i], 1);
         mbar_fence_init();
     }
     if (warp == 0) {
@@ -208,114 +272,136 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_before();
     __syncthreads();
     fence_after();
-    const uint32_t tbase = *tmem_slot;
+    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
 
-    const uint32_t col = (uint32_t)g * 64u;
+    const uint32_t col = tbase + (uint32_t)g * 128u;
     const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-    const uint32_t tD = tbase + col, tA1 = tbase + col + 32, tA = tbase + col + 40, tC = tbase + col + 56;
+    const TileIO X{col + 0, col + 32, col + 40}, Y{col + 64, col + 96, col + 104};
+    const uint32_t tC = col + 56;
     {
         uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
         tmem_st8(tC + lane_off, c8);
         tmem_wait_st();
     }
-    const bool leader = (tid & 127) == 0;
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    const uint32_t w2a = sbase + L.w2, w3a = sbase + L.w3, w4a = sbase + L.w4, b1a = sbase + L.b1;
     constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
-    uint64_t* bar = &bars[g];
-    uint32_t phase = 0;
+    uint64_t* barX = &bars[2 * g];
+    uint64_t* barY = &bars[2 * g + 1];
+    uint32_t phX = 0, phY = 0;
+    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
+#pragma unroll
+    for (int i = 0; i < C::kNchHid; i++) {
+        d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
+        d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
+    }
+#pragma unroll
+    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
+    const uint64_t d1base = smem_desc(sbase + L.b1);
+    constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);  // descriptor units per segment table
+
+    auto sync_group = [&]() {
+        fence_before();
+        named_bar_sync(1 + g, 128);
+        fence_after();
+    };
+    const bool issuer = wq == 0;  // warp-uniform: warp 0 of the group issues (one elected lane)
+    auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
+        if (issuer) {
+            const int su = __shfl_sync(0xffffffffu, s, 0);
+            const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
+            mma_ts_elect(T.d, T.a1, db, id32, 0u);
+            if (C::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
+            mma_commit_elect(bar);
+        }
+    };
+    auto issue = [&](const TileIO& T, const uint64_t* dl, uint32_t idesc, uint64_t* bar) {
+        if (issuer) {
+            issue_layer_e<FMT>(T.d, T.a, tC, dl, idesc);
+            mma_commit_elect(bar);
+        }
+    };
 
     unsigned long long best = 0;
     float best_y = __int_as_float(0x7fc00000);
-    for (uint64_t w = (uint64_t)blockIdx.x * NG + g; w < P.n_tiles; w += (uint64_t)gridDim.x * NG) {
-        const int s = find_segment(P, w);
-        const SegP& sg = P.seg[s];
-        const uint64_t ub = sg.u_begin + (w - sg.tile0) * kTileM;
-        const bool valid = ub + r < sg.u_end;
-        uint32_t v[kKMax];
-        decode_box<kKMax>(sg, ub, r, v);
+    uint64_t wb, we;
+    work_range(P.n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
+    Walker W;
+    if (wb < we) walker_begin(P, W, wb, r);
+    for (uint64_t w = wb; w < we; w += 2) {
+        // ---- tile a (slot X) = w, tile b (slot Y) = w + 1 ---------------------
+        if (w != wb) walker_next(P, W, w, r);
+        const uint32_t va[kKMax] = {W.v[0], W.v[1], W.v[2], W.v[3]};
+        const int sa = W.s;
+        const bool valid_a = W.u_end - W.ub > (uint64_t)r;
+        const bool zero_a = walker_is_index0(W, r);
+        const bool has_b = w + 1 < we;
+        if (has_b) walker_next(P, W, w + 1, r);
+        const bool valid_b = has_b && (W.u_end - W.ub > (uint64_t)r);
 
-        // a3 (fused): layer-1 operand row [1, 1, v0_hi, v0_lo, ..., v3_hi, v3_lo, 0...]
+        store_a1<FMT, SPLIT>(X.a1 + lane_off, va);
+        store_a1<FMT, SPLIT>(Y.a1 + lane_off, W.v);
+        tmem_wait_st();
+        sync_group();
+        issue_l1(X, sa, barX);
+        issue_l1(Y, W.s, barY);
+        // layers 2, 3: wait X -> epilogue X -> issue X; then the same for Y
+#pragma unroll 1
+        for (int layer = 0; layer < 2; layer++) {
+            const uint64_t* dl = layer == 0 ? d2 : d3;
+            mbar_wait(barX, phX);
+            phX ^= 1u;
+            fence_after();
+            hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
+            sync_group();
+            issue(X, dl, id32, barX);
+            mbar_wait(barY, phY);
+            phY ^= 1u;
+            fence_after();
+            hidden_epilogue<FMT>(Y.d + lane_off, Y.a + lane_off);
+            sync_group();
+            issue(Y, dl, id32, barY);
+        }
+        // layer 3 epilogue -> output MMA (N = 16)
+        mbar_wait(barX, phX);
+        phX ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
+        sync_group();
+        issue(X, d4, id16, barX);
+        mbar_wait(barY, phY);
+        phY ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(Y.d + lane_off, Y.a + lane_off);
+        sync_group();
+        issue(Y, d4, id16, barY);
+        // outputs + a5 fold
+        mbar_wait(barX, phX);
+        phX ^= 1u;
+        fence_after();
+        uint32_t ya, yb;
+        tmem_ld1(X.d + lane_off, ya);
+        mbar_wait(barY, phY);
+        phY ^= 1u;
+        fence_after();
+        tmem_ld1(Y.d + lane_off, yb);
+        if (valid_a && zero_a) S->y0 = __uint_as_float(ya);
+        if (valid_b && walker_is_index0(W, r)) S->y0 = __uint_as_float(yb);
         {
-            uint32_t a[8];
-            a[0] = C::kOne2;
+            // tile a's segment state (cheap reload: only n_base/t_base/istride)
+            Walker Wa;
+            const SegP& ga = P.seg[sa];
+            Wa.n_base = ga.n_base;
+            Wa.t_base = ga.t_base;
 #pragma unroll
-            for (int j = 0; j < kKMax; j++) a[1 + j] = pack2<FMT>((float)(v[j] >> 8), (float)(v[j] & 255u));
-            a[5] = a[6] = a[7] = 0;
-            tmem_st8(tA1 + lane_off, a);
-            tmem_wait_st();
-        }
-        // layer 1
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            const uint32_t bs = b1a + (uint32_t)s * C::kNchL1 * kChunkBytesN32;
-            mma_ts(tD, tA1, smem_desc(bs), id32, 0u);
-            if (C::kNchL1 > 1) mma_ts(tD, tA1, smem_desc(bs + kChunkBytesN32), id32, 1u);
-            mma_commit(bar);
-        }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        // layer 2
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            issue_layer<FMT>(tD, tA, tC, w2a, kChunkBytesN32, id32);
-            mma_commit(bar);
-        }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        // layer 3
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            issue_layer<FMT>(tD, tA, tC, w3a, kChunkBytesN32, id32);
-            mma_commit(bar);
-        }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        // output layer (N = 16, column 0 = y)
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            issue_layer<FMT>(tD, tA, tC, w4a, kChunkBytesN16, id16);
-            mma_commit(bar);
-        }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        uint32_t ybits;
-        tmem_ld1(tD + lane_off, ybits);
-        const float y = __uint_as_float(ybits);
-
-        // a5: headroom mask + key
-        uint64_t idx = sg.t_base;
-        int32_t sum_n = sg.n_base;
-#pragma unroll
-        for (int j = 0; j < kKMax; j++) {
-            idx += (uint64_t)v[j] * sg.istride[j];
-            sum_n += (int32_t)v[j];
-        }
-        if (valid && idx == 0) S->y0 = y;
-        if (valid && y <= P.H) {
-            const unsigned long long key = ((unsigned long long)(sum_n + 1) << 40) | idx;
-            if (key > best) {
-                best = key;
-                best_y = y;
+            for (int j = 0; j < kKMax; j++) {
+                Wa.istride[j] = ga.istride[j];
+                Wa.v[j] = va[j];
             }
+            fold_candidate(Wa, valid_a, __uint_as_float(ya), P.H, best, best_y);
         }
-        fence_before();  // order this tile's TMEM reads before the next tile's writes/MMAs
+        fold_candidate(W, valid_b, __uint_as_float(yb), P.H, best, best_y);
+        fence_before();
     }
     fence_before();
     __syncthreads();
@@ -515,15 +601,16 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
 constexpr int kFusedNG = 4;
 constexpr int kPredictNG = 4;
 
-template <int FMT>
+template <int FMT, bool SPLIT>
 static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const float* w1b1, Scratch* S, int nsm,
                                     cudaStream_t st, int* grid_out) {
     using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, kFusedNG, 0);
-    auto kern = fused_tc_kernel<FMT, kFusedNG>;
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG, 0);
+    auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
-    uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
+    // two tiles in flight per group: spread the tiles over as many SMs as possible
+    uint64_t g = (P.n_tiles + 2 * kFusedNG - 1) / (2 * kFusedNG);
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     *grid_out = (int)g;
@@ -534,8 +621,16 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
-    if (TW.fmt == 0) return launch_fused_fmt<0>(P, tp, w1b1, S, nsm, st, grid_out);
-    return launch_fused_fmt<1>(P, tp, w1b1, S, nsm, st, grid_out);
+    uint32_t maxcnt = 0;
+    for (int s = 0; s < P.n_seg; s++)
+        for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
+    // digits are < cnt: exact unsplit up to 2048 in fp16, 256 in bf16
+    if (TW.fmt == 0) {
+        if (maxcnt <= 2049) return launch_fused_fmt<0, false>(P, tp, w1b1, S, nsm, st, grid_out);
+        return launch_fused_fmt<0, true>(P, tp, w1b1, S, nsm, st, grid_out);
+    }
+    if (maxcnt <= 257) return launch_fused_fmt<1, false>(P, tp, w1b1, S, nsm, st, grid_out);
+    return launch_fused_fmt<1, true>(P, tp, w1b1, S, nsm, st, grid_out);
 }
 
 template <int FMT>
