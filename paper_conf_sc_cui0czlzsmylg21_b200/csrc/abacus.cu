@@ -379,7 +379,7 @@ int scale_exp(double bound) {
 }
 
 // blob: [W2 chunks][W3 chunks][out chunks]; chunk = N rows x 16 K, b_offset layout
-std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale) {
+std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, float* w4s, float* b4_out) {
     const int D = c->D;
     const float* p = c->params.data();
     const float* W1 = p;
@@ -415,6 +415,8 @@ std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale) {
         s3 = std::ldexp(1.0, -scale_exp(B3));
     }
     *l1_scale = (float)s1;
+    for (int j = 0; j < kHidden; j++) w4s[j] = (float)((double)w4[j] / s3);  // exact: s3 is a power of two
+    *b4_out = b4;
     const int nch = fmt == 0 ? 3 : 5;
     const size_t hid_bytes = (size_t)nch * tc::kChunkBytesN32;
     const size_t out_bytes = (size_t)nch * tc::kChunkBytesN16;
@@ -582,11 +584,18 @@ int abacus_load_predictor(abacus_ctx* c, const float* params, size_t n_params, i
     c->w234.b4 = *q;
     for (int fmt = 0; fmt < 2; fmt++) {
         float l1s = 1.0f;
-        std::vector<uint8_t> blob = build_blob(c, fmt, &l1s);
+        TcWeights tw{};
+        std::vector<uint8_t> blob = build_blob(c, fmt, &l1s, tw.w4s, &tw.b4);
         if (c->d_blob[fmt]) cudaFree(c->d_blob[fmt]);
         CUDA_TRY(c, cudaMalloc(&c->d_blob[fmt], blob.size()));
         CUDA_TRY(c, cudaMemcpy(c->d_blob[fmt], blob.data(), blob.size(), cudaMemcpyHostToDevice));
-        c->tw[fmt] = TcWeights{fmt, fmt == 0 ? 3 : 5, fmt == 0 ? 3 : 5, (uint32_t)blob.size(), l1s, c->d_blob[fmt]};
+        tw.fmt = fmt;
+        tw.nch_hidden = fmt == 0 ? 3 : 5;
+        tw.nch_out = fmt == 0 ? 3 : 5;
+        tw.bytes = (uint32_t)blob.size();
+        tw.l1_scale = l1s;
+        tw.blob = c->d_blob[fmt];
+        c->tw[fmt] = tw;
     }
     c->precision = precision;
     c->loaded = true;

@@ -105,6 +105,23 @@ __device__ __forceinline__ void fold_candidate(const Walker& W, bool valid, floa
     }
 }
 
+// fold a finished candidate given its segment and digits (valid, y known)
+__device__ __forceinline__ void fold_tile(const Plan& P, int s, const uint32_t (&v)[kKMax], float y,
+                                          unsigned long long& best, float& best_y) {
+    if (!(y <= P.H)) return;
+    const SegP& g = P.seg[s];
+    const uint32_t hi = (uint32_t)(g.n_base + (int32_t)(v[0] + v[1] + v[2] + v[3]) + 1);
+    if (hi < (uint32_t)(best >> 40)) return;
+    uint64_t idx = g.t_base;
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) idx += (uint64_t)v[j] * g.istride[j];
+    const unsigned long long key = ((unsigned long long)hi << 40) | idx;
+    if (key > best) {
+        best = key;
+        best_y = y;
+    }
+}
+
 __device__ __forceinline__ bool walker_is_index0(const Walker& W, uint32_t r) {
     return W.t_base == 0 && W.ub == 0 && r == 0;
 }

@@ -239,9 +239,30 @@ __device__ __forceinline__ void store_a1(uint32_t taddr, const uint32_t (&v)[kKM
     tmem_st8(taddr, a);
 }
 
+// output layer in fp32 on the SIMT pipes: y = b4 + sum_j w4s_j relu(z3_j)
+// (w4s = w4 * 2^s3 undoes the fp16 layer scaling; kernel parameter -> FFMA
+// with a constant-bank operand)
+struct OutW {
+    float w4s[kHidden];
+    float b4;
+};
+
+__device__ __forceinline__ float output_dot(uint32_t tD_lane, const OutW& O) {
+    uint32_t z[32];
+    tmem_ld32(tD_lane, z);
+    float acc0 = O.b4, acc1 = 0.0f;
+#pragma unroll
+    for (int j = 0; j < kHidden; j += 2) {
+        acc0 = fmaf(O.w4s[j], fmaxf(__uint_as_float(z[j]), 0.0f), acc0);
+        acc1 = fmaf(O.w4s[j + 1], fmaxf(__uint_as_float(z[j + 1]), 0.0f), acc1);
+    }
+    return acc0 + acc1;
+}
+
 template <int FMT, bool SPLIT, int NG>
 __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
                                                                const __grid_constant__ TcParams TP,
+                                                               const __grid_constant__ OutW O,
                                                                const float* __restrict__ w1b1, Scratch* S) {
     extern __shared__ __align__(1024) uint8_t smem[];
     using C = TcCfg<FMT>;
@@ -250,8 +271,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
 
     const int tid = threadIdx.x;
-    // warp-uniform indices (shfl from lane 0: the compiler keeps them uniform)
-    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform for the compiler
     const int g = warp >> 2, wq = warp & 3;
 
     {
@@ -274,38 +294,42 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_after();
     const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
 
-    const uint32_t col = tbase + (uint32_t)g * 128u;
+    // TMEM: group g owns 96 columns at 96 g: D_X [0,32) D_Y [32,64) A_X [64,80)
+    // A_Y [80,96); the layer-1 operand A1 aliases the first 8 columns of A.
+    // One constant chunk (1, 1, 0, ...) for the bias columns at 480.
+    const uint32_t col = tbase + (uint32_t)g * 96u;
     const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-    const TileIO X{col + 0, col + 32, col + 40}, Y{col + 64, col + 96, col + 104};
-    const uint32_t tC = col + 56;
-    {
+    const TileIO X{col + 0, col + 64, col + 64}, Y{col + 32, col + 80, col + 80};
+    const uint32_t tC = tbase + 480;
+    if (g == 0) {
         uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
         tmem_st8(tC + lane_off, c8);
         tmem_wait_st();
     }
+    fence_before();
+    __syncthreads();
+    fence_after();
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
+    constexpr uint32_t id32 = idesc_f16(FMT, 32);
     uint64_t* barX = &bars[2 * g];
     uint64_t* barY = &bars[2 * g + 1];
     uint32_t phX = 0, phY = 0;
-    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
+    uint64_t d2[C::kNchHid], d3[C::kNchHid];
 #pragma unroll
     for (int i = 0; i < C::kNchHid; i++) {
         d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
         d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
     }
-#pragma unroll
-    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
     const uint64_t d1base = smem_desc(sbase + L.b1);
-    constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);  // descriptor units per segment table
+    constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
+    const bool issuer = wq == 0;  // warp 0 of the group issues (one elected lane)
 
     auto sync_group = [&]() {
         fence_before();
         named_bar_sync(1 + g, 128);
         fence_after();
     };
-    const bool issuer = wq == 0;  // warp-uniform: warp 0 of the group issues (one elected lane)
     auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
         if (issuer) {
             const int su = __shfl_sync(0xffffffffu, s, 0);
@@ -315,9 +339,15 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             mma_commit_elect(bar);
         }
     };
-    auto issue = [&](const TileIO& T, const uint64_t* dl, uint32_t idesc, uint64_t* bar) {
+    // wait for layer l of T, epilogue (ReLU, pack) into A, issue layer l+1
+    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl) {
+        mbar_wait(bar, ph);
+        ph ^= 1u;
+        fence_after();
+        hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
+        sync_group();
         if (issuer) {
-            issue_layer_e<FMT>(T.d, T.a, tC, dl, idesc);
+            issue_layer_e<FMT>(T.d, T.a, tC, dl, id32);
             mma_commit_elect(bar);
         }
     };
@@ -326,82 +356,75 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     float best_y = __int_as_float(0x7fc00000);
     uint64_t wb, we;
     work_range(P.n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
-    Walker W;
-    if (wb < we) walker_begin(P, W, wb, r);
-    for (uint64_t w = wb; w < we; w += 2) {
-        // ---- tile a (slot X) = w, tile b (slot Y) = w + 1 ---------------------
-        if (w != wb) walker_next(P, W, w, r);
-        const uint32_t va[kKMax] = {W.v[0], W.v[1], W.v[2], W.v[3]};
-        const int sa = W.s;
-        const bool valid_a = W.u_end - W.ub > (uint64_t)r;
-        const bool zero_a = walker_is_index0(W, r);
-        const bool has_b = w + 1 < we;
-        if (has_b) walker_next(P, W, w + 1, r);
-        const bool valid_b = has_b && (W.u_end - W.ub > (uint64_t)r);
-
-        store_a1<FMT, SPLIT>(X.a1 + lane_off, va);
-        store_a1<FMT, SPLIT>(Y.a1 + lane_off, W.v);
+    if (wb < we) {
+        Walker W;
+        walker_begin(P, W, wb, r);
+        uint32_t vX[kKMax], vY[kKMax];
+        int sX, sY;
+        bool okX, okY, zX, zY;
+        auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z, uint64_t w) {
+            ok = w < we && (W.u_end - W.ub > (uint64_t)r);
+            z = w < we && walker_is_index0(W, r);
+#pragma unroll
+            for (int j = 0; j < kKMax; j++) v[j] = W.v[j];
+            s = W.s;
+        };
+        auto advance = [&](uint64_t w_next) {
+            if (w_next < we) walker_next(P, W, w_next, r);
+        };
+        // prologue: tiles wb (X) and wb + 1 (Y)
+        take(vX, sX, okX, zX, wb);
+        store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
+        advance(wb + 1);
+        take(vY, sY, okY, zY, wb + 1);
+        store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
         tmem_wait_st();
         sync_group();
-        issue_l1(X, sa, barX);
-        issue_l1(Y, W.s, barY);
-        // layers 2, 3: wait X -> epilogue X -> issue X; then the same for Y
-#pragma unroll 1
-        for (int layer = 0; layer < 2; layer++) {
-            const uint64_t* dl = layer == 0 ? d2 : d3;
+        issue_l1(X, sX, barX);
+        issue_l1(Y, sY, barY);
+
+        for (uint64_t w = wb; w < we; w += 2) {
+            stage(X, barX, phX, d2);
+            stage(Y, barY, phY, d2);
+            stage(X, barX, phX, d3);
+            stage(Y, barY, phY, d3);
+            // X: layer-3 result -> fp32 output layer; start tile w + 2 while Y's layer 3 runs
             mbar_wait(barX, phX);
             phX ^= 1u;
             fence_after();
-            hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
+            const float yX = output_dot(X.d + lane_off, O);
+            const uint32_t fvX[kKMax] = {vX[0], vX[1], vX[2], vX[3]};
+            const int fsX = sX;
+            const bool fokX = okX, fzX = zX;
+            advance(w + 2);
+            take(vX, sX, okX, zX, w + 2);
+            store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
+            tmem_wait_st();
             sync_group();
-            issue(X, dl, id32, barX);
+            issue_l1(X, sX, barX);
+            // Y: the same, next tile w + 3
             mbar_wait(barY, phY);
             phY ^= 1u;
             fence_after();
-            hidden_epilogue<FMT>(Y.d + lane_off, Y.a + lane_off);
+            const float yY = output_dot(Y.d + lane_off, O);
+            const uint32_t fvY[kKMax] = {vY[0], vY[1], vY[2], vY[3]};
+            const int fsY = sY;
+            const bool fokY = okY, fzY = zY;
+            advance(w + 3);
+            take(vY, sY, okY, zY, w + 3);
+            store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+            tmem_wait_st();
             sync_group();
-            issue(Y, dl, id32, barY);
+            issue_l1(Y, sY, barY);
+            // a5: fold the two finished tiles
+            if (fokX && fzX) S->y0 = yX;
+            if (fokY && fzY) S->y0 = yY;
+            if (fokX) fold_tile(P, fsX, fvX, yX, best, best_y);
+            if (fokY) fold_tile(P, fsY, fvY, yY, best, best_y);
         }
-        // layer 3 epilogue -> output MMA (N = 16)
+        // drain the layer-1 MMAs issued for the tiles past the end
         mbar_wait(barX, phX);
-        phX ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
-        sync_group();
-        issue(X, d4, id16, barX);
         mbar_wait(barY, phY);
-        phY ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(Y.d + lane_off, Y.a + lane_off);
-        sync_group();
-        issue(Y, d4, id16, barY);
-        // outputs + a5 fold
-        mbar_wait(barX, phX);
-        phX ^= 1u;
-        fence_after();
-        uint32_t ya, yb;
-        tmem_ld1(X.d + lane_off, ya);
-        mbar_wait(barY, phY);
-        phY ^= 1u;
-        fence_after();
-        tmem_ld1(Y.d + lane_off, yb);
-        if (valid_a && zero_a) S->y0 = __uint_as_float(ya);
-        if (valid_b && walker_is_index0(W, r)) S->y0 = __uint_as_float(yb);
-        {
-            // tile a's segment state (cheap reload: only n_base/t_base/istride)
-            Walker Wa;
-            const SegP& ga = P.seg[sa];
-            Wa.n_base = ga.n_base;
-            Wa.t_base = ga.t_base;
-#pragma unroll
-            for (int j = 0; j < kKMax; j++) {
-                Wa.istride[j] = ga.istride[j];
-                Wa.v[j] = va[j];
-            }
-            fold_candidate(Wa, valid_a, __uint_as_float(ya), P.H, best, best_y);
-        }
-        fold_candidate(W, valid_b, __uint_as_float(yb), P.H, best, best_y);
-        fence_before();
     }
     fence_before();
     __syncthreads();
@@ -598,12 +621,12 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
 // ---------------------------------------------------------------------------
 // launchers
 // ---------------------------------------------------------------------------
-constexpr int kFusedNG = 4;
+constexpr int kFusedNG = 5;
 constexpr int kPredictNG = 4;
 
 template <int FMT, bool SPLIT>
-static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const float* w1b1, Scratch* S, int nsm,
-                                    cudaStream_t st, int* grid_out) {
+static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const OutW& ow, const float* w1b1,
+                                    Scratch* S, int nsm, cudaStream_t st, int* grid_out) {
     using C = TcCfg<FMT>;
     const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG, 0);
     auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
@@ -614,23 +637,26 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     *grid_out = (int)g;
-    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, w1b1, S);
+    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, ow, w1b1, S);
     return cudaGetLastError();
 }
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    OutW ow;
+    for (int j = 0; j < kHidden; j++) ow.w4s[j] = TW.w4s[j];
+    ow.b4 = TW.b4;
     uint32_t maxcnt = 0;
     for (int s = 0; s < P.n_seg; s++)
         for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
     // digits are < cnt: exact unsplit up to 2048 in fp16, 256 in bf16
     if (TW.fmt == 0) {
-        if (maxcnt <= 2049) return launch_fused_fmt<0, false>(P, tp, w1b1, S, nsm, st, grid_out);
-        return launch_fused_fmt<0, true>(P, tp, w1b1, S, nsm, st, grid_out);
+        if (maxcnt <= 2049) return launch_fused_fmt<0, false>(P, tp, ow, w1b1, S, nsm, st, grid_out);
+        return launch_fused_fmt<0, true>(P, tp, ow, w1b1, S, nsm, st, grid_out);
     }
-    if (maxcnt <= 257) return launch_fused_fmt<1, false>(P, tp, w1b1, S, nsm, st, grid_out);
-    return launch_fused_fmt<1, true>(P, tp, w1b1, S, nsm, st, grid_out);
+    if (maxcnt <= 257) return launch_fused_fmt<1, false>(P, tp, ow, w1b1, S, nsm, st, grid_out);
+    return launch_fused_fmt<1, true>(P, tp, ow, w1b1, S, nsm, st, grid_out);
 }
 
 template <int FMT>
