@@ -323,30 +323,42 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     }
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
-    const bool issuer = wq == 0;  // warp 0 of the group issues (one elected lane)
 
-    auto sync_group = [&]() {
+    // Operand hand-off: after writing its 32 rows a warp fences its tcgen05.st
+    // and ARRIVES on the slot's named barrier without blocking; only the
+    // stage's issuing warp SYNCs (waits for all 128 threads), then issues the
+    // MMAs from one elected lane and commits them to the slot's mbarrier.  The
+    // issuer rotates over the group's 4 warps (one per SMSP) stage by stage.
+    // Slots X and Y use different barrier ids, so a warp running ahead can
+    // never arrive in the wrong phase.
+    auto handoff = [&](uint32_t bar_id, uint32_t turn) -> bool {
         fence_before();
-        named_bar_sync(1 + g, 128);
-        fence_after();
-    };
-    auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
-        if (issuer) {
-            const int su = __shfl_sync(0xffffffffu, s, 0);
-            const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
-            mma_ts_elect(T.d, T.a1, db, id32, 0u);
-            if (C::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
-            mma_commit_elect(bar);
+        const bool me = (uint32_t)wq == (turn & 3u);
+        if (me) {
+            named_bar_sync(bar_id, 128);
+            fence_after();
+        } else {
+            named_bar_arrive(bar_id, 128);
         }
+        return me;
     };
-    // wait for layer l of T, epilogue (ReLU, pack) into A, issue layer l+1
-    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl) {
+    const uint32_t idX = 1 + 2 * g, idY = 2 + 2 * g;
+    uint32_t turnX = (uint32_t)g, turnY = (uint32_t)g + 2u;
+    auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
+        const int su = __shfl_sync(0xffffffffu, s, 0);
+        const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
+        mma_ts_elect(T.d, T.a1, db, id32, 0u);
+        if (C::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
+        mma_commit_elect(bar);
+    };
+    // wait for layer l of T, epilogue (ReLU, pack) into A, hand off, issue layer l+1
+    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id,
+                     uint32_t& turn) {
         mbar_wait(bar, ph);
         ph ^= 1u;
         fence_after();
         hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
-        sync_group();
-        if (issuer) {
+        if (handoff(bar_id, turn++)) {
             issue_layer_e<FMT>(T.d, T.a, tC, dl, id32);
             mma_commit_elect(bar);
         }
@@ -379,15 +391,14 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         take(vY, sY, okY, zY, wb + 1);
         store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
         tmem_wait_st();
-        sync_group();
-        issue_l1(X, sX, barX);
-        issue_l1(Y, sY, barY);
+        if (handoff(idX, turnX++)) issue_l1(X, sX, barX);
+        if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
 
         for (uint64_t w = wb; w < we; w += 2) {
-            stage(X, barX, phX, d2);
-            stage(Y, barY, phY, d2);
-            stage(X, barX, phX, d3);
-            stage(Y, barY, phY, d3);
+            stage(X, barX, phX, d2, idX, turnX);
+            stage(Y, barY, phY, d2, idY, turnY);
+            stage(X, barX, phX, d3, idX, turnX);
+            stage(Y, barY, phY, d3, idY, turnY);
             // X: layer-3 result -> fp32 output layer; start tile w + 2 while Y's layer 3 runs
             mbar_wait(barX, phX);
             phX ^= 1u;
@@ -400,8 +411,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             take(vX, sX, okX, zX, w + 2);
             store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
             tmem_wait_st();
-            sync_group();
-            issue_l1(X, sX, barX);
+            if (handoff(idX, turnX++)) issue_l1(X, sX, barX);
             // Y: the same, next tile w + 3
             mbar_wait(barY, phY);
             phY ^= 1u;
@@ -414,8 +424,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             take(vY, sY, okY, zY, w + 3);
             store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
             tmem_wait_st();
-            sync_group();
-            issue_l1(Y, sY, barY);
+            if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
             // a5: fold the two finished tiles
             if (fokX && fzX) S->y0 = yX;
             if (fokY && fzY) S->y0 = yY;
