@@ -311,16 +311,18 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_after();
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    constexpr uint32_t id32 = idesc_f16(FMT, 32);
+    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
     uint64_t* barX = &bars[2 * g];
     uint64_t* barY = &bars[2 * g + 1];
     uint32_t phX = 0, phY = 0;
-    uint64_t d2[C::kNchHid], d3[C::kNchHid];
+    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
 #pragma unroll
     for (int i = 0; i < C::kNchHid; i++) {
         d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
         d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
     }
+#pragma unroll
+    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
 
@@ -353,13 +355,13 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     };
     // wait for layer l of T, epilogue (ReLU, pack) into A, hand off, issue layer l+1
     auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id,
-                     uint32_t& turn) {
+                     uint32_t& turn, uint32_t idesc) {
         mbar_wait(bar, ph);
         ph ^= 1u;
         fence_after();
         hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
         if (handoff(bar_id, turn++)) {
-            issue_layer_e<FMT>(T.d, T.a, tC, dl, id32);
+            issue_layer_e<FMT>(T.d, T.a, tC, dl, idesc);
             mma_commit_elect(bar);
         }
     };
@@ -395,18 +397,23 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
 
         for (uint64_t w = wb; w < we; w += 2) {
-            stage(X, barX, phX, d2, idX, turnX);
-            stage(Y, barY, phY, d2, idY, turnY);
-            stage(X, barX, phX, d3, idX, turnX);
-            stage(Y, barY, phY, d3, idY, turnY);
-            // X: layer-3 result -> fp32 output layer; start tile w + 2 while Y's layer 3 runs
+            stage(X, barX, phX, d2, idX, turnX, id32);
+            stage(Y, barY, phY, d2, idY, turnY, id32);
+            stage(X, barX, phX, d3, idX, turnX, id32);
+            stage(Y, barY, phY, d3, idY, turnY, id32);
+            stage(X, barX, phX, d4, idX, turnX, id16);
+            stage(Y, barY, phY, d4, idY, turnY, id16);
+            // X: output ready -> fold (a5) -> start tile w + 2 while Y's output MMA runs
             mbar_wait(barX, phX);
             phX ^= 1u;
             fence_after();
-            const float yX = output_dot(X.d + lane_off, O);
-            const uint32_t fvX[kKMax] = {vX[0], vX[1], vX[2], vX[3]};
-            const int fsX = sX;
-            const bool fokX = okX, fzX = zX;
+            {
+                uint32_t yb;
+                tmem_ld1(X.d + lane_off, yb);
+                const float y = __uint_as_float(yb);
+                if (okX && zX) S->y0 = y;
+                if (okX) fold_tile(P, sX, vX, y, best, best_y);
+            }
             advance(w + 2);
             take(vX, sX, okX, zX, w + 2);
             store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
@@ -416,20 +423,18 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             mbar_wait(barY, phY);
             phY ^= 1u;
             fence_after();
-            const float yY = output_dot(Y.d + lane_off, O);
-            const uint32_t fvY[kKMax] = {vY[0], vY[1], vY[2], vY[3]};
-            const int fsY = sY;
-            const bool fokY = okY, fzY = zY;
+            {
+                uint32_t yb;
+                tmem_ld1(Y.d + lane_off, yb);
+                const float y = __uint_as_float(yb);
+                if (okY && zY) S->y0 = y;
+                if (okY) fold_tile(P, sY, vY, y, best, best_y);
+            }
             advance(w + 3);
             take(vY, sY, okY, zY, w + 3);
             store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
             tmem_wait_st();
             if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
-            // a5: fold the two finished tiles
-            if (fokX && fzX) S->y0 = yX;
-            if (fokY && fzY) S->y0 = yY;
-            if (fokX) fold_tile(P, fsX, fvX, yX, best, best_y);
-            if (fokY) fold_tile(P, fsY, fvY, yY, best, best_y);
         }
         // drain the layer-1 MMAs issued for the tiles past the end
         mbar_wait(barX, phX);
