@@ -187,13 +187,16 @@ Plan plan_whole_grid(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T) {
     for (int j = 0; j < kKMax; j++) {
         s.cnt[j] = j < g->k ? (uint32_t)P.slot[j].radix : 1u;
         s.pos[j] = -1;
+        s.dpos[j] = j;
     }
     finish_box(s);
     return P;
 }
 
-// number of elements of box `s` (digit sets per slot, see below) with index < a
-uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, uint64_t a) {
+// number of elements of segment box `s` with index < a.  Per SLOT j the box
+// digit set is: present -> [dlo_j, dlo_j + cnt_j), absent -> {0}; elements
+// are ordered lexicographically by slot (index order).
+uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const uint32_t* scnt, uint64_t a) {
     if (a >= P.T) return box_size(s);
     uint32_t dig[kKMax] = {0, 0, 0, 0};
     uint64_t rem = a;
@@ -204,20 +207,40 @@ uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, uint64_
     uint64_t cnt = 0;
     for (int j = 0; j < P.k; j++) {
         const bool present = (s.mask >> j) & 1u;
+        uint64_t after = 1;  // elements per value of slot j's digit
+        for (int i = j + 1; i < P.k; i++)
+            if ((s.mask >> i) & 1u) after *= scnt[i];
         uint64_t below;
         bool inside;
         if (present) {
             const int64_t b = (int64_t)dig[j] - (int64_t)dlo[j];
-            below = (uint64_t)std::min<int64_t>(std::max<int64_t>(b, 0), (int64_t)s.cnt[j]);
-            inside = dig[j] >= dlo[j] && dig[j] < dlo[j] + s.cnt[j];
+            below = (uint64_t)std::min<int64_t>(std::max<int64_t>(b, 0), (int64_t)scnt[j]);
+            inside = dig[j] >= dlo[j] && dig[j] < dlo[j] + scnt[j];
         } else {
             below = dig[j] > 0 ? 1 : 0;
             inside = dig[j] == 0;
         }
-        cnt += below * s.bstride[j];
+        cnt += below * after;
         if (!inside) return cnt;
     }
     return cnt;
+}
+
+// Lay the per-slot box (scnt, sistride) out in digit order: slots with
+// cnt == 1 first, then the varying ones in slot order (common.cuh).
+void order_digits(SegP& s, int k, const uint32_t* scnt, const uint64_t* sistride) {
+    int d = 0;
+    for (int pass = 0; pass < 2; pass++)
+        for (int j = 0; j < kKMax; j++) {
+            const uint32_t cj = j < k ? scnt[j] : 1u;
+            if ((pass == 0) != (cj == 1)) continue;
+            s.dpos[j] = d;
+            s.cnt[d] = cj;
+            s.istride[d] = j < k ? sistride[j] : 0;
+            d++;
+        }
+    finish_box(s);
+    s.fast_carry = s.cnt[kKMax - 1] >= (uint32_t)kTileM ? 1u : 0u;
 }
 
 void set_positions(const Plan& P, SegP& s) {
@@ -259,29 +282,28 @@ Plan plan_grid_segments(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T,
         if (!ok) continue;
         SegP s{};
         s.mask = mask;
-        uint32_t dlo[kKMax] = {0, 0, 0, 0};
+        uint32_t dlo[kKMax] = {0, 0, 0, 0}, scnt[kKMax] = {1, 1, 1, 1};
+        uint64_t sist[kKMax] = {0, 0, 0, 0};
         s.n_base = 0;
         s.t_base = 0;
         for (int j = 0; j < kKMax; j++) {
             const bool present = j < g->k && ((mask >> j) & 1u);
             if (present) {
                 const abacus_slot_t& a = g->slot[j];
-                s.cnt[j] = (uint32_t)(a.end_hi - a.end_lo + 1);
+                scnt[j] = (uint32_t)(a.end_hi - a.end_lo + 1);
                 dlo[j] = a.allow_absent ? 1u : 0u;
                 s.ope0[j] = a.end_lo;
-                s.istride[j] = tstride[j];
+                sist[j] = tstride[j];
                 s.t_base += (uint64_t)dlo[j] * tstride[j];
                 s.n_base += a.end_lo - a.start_op + 1;
             } else {
-                s.cnt[j] = 1;
                 s.ope0[j] = 0;
-                s.istride[j] = 0;
             }
         }
-        finish_box(s);
+        order_digits(s, g->k, scnt, sist);
         set_positions(P, s);
-        s.u_begin = box_count_lt(P, s, dlo, first);
-        s.u_end = box_count_lt(P, s, dlo, last);
+        s.u_begin = box_count_lt(P, s, dlo, scnt, first);
+        s.u_end = box_count_lt(P, s, dlo, scnt, last);
         if (s.u_end <= s.u_begin) continue;
         s.tile0 = tiles;
         tiles += (s.u_end - s.u_begin + kTileM - 1) / kTileM;
@@ -310,11 +332,9 @@ Plan plan_chain(const abacus_ctx* c, const abacus_grid_t* g, float H, uint64_t* 
         SegP s{};
         s.mask = (2u << j) - 1u;
         s.n_base = 0;
-        for (int i = 0; i < kKMax; i++) {
-            s.cnt[i] = 1;
-            s.istride[i] = 0;
-            s.ope0[i] = 0;
-        }
+        uint32_t scnt[kKMax] = {1, 1, 1, 1};
+        uint64_t sist[kKMax] = {0, 0, 0, 0};
+        for (int i = 0; i < kKMax; i++) s.ope0[i] = 0;
         for (int i = 0; i < j; i++) {
             s.ope0[i] = g->slot[i].end_hi;
             s.n_base += g->slot[i].end_hi - g->slot[i].start_op + 1;
@@ -323,14 +343,14 @@ Plan plan_chain(const abacus_ctx* c, const abacus_grid_t* g, float H, uint64_t* 
             s.ope0[0] = g->slot[0].end_hi;
             s.n_base = g->slot[0].end_hi - g->slot[0].start_op + 1;
         } else {
-            s.cnt[j] = (uint32_t)(g->slot[j].end_hi - g->slot[j].start_op + 1);
+            scnt[j] = (uint32_t)(g->slot[j].end_hi - g->slot[j].start_op + 1);
             s.ope0[j] = g->slot[j].start_op;
-            s.istride[j] = 1;
+            sist[j] = 1;
             s.n_base += 1;
         }
+        order_digits(s, g->k, scnt, sist);
         P.chain_cum[j] = cum;
         s.t_base = cum;
-        finish_box(s);
         set_positions(P, s);
         s.u_begin = 0;
         s.u_end = box_size(s);

@@ -6,8 +6,10 @@
 //     ope_j = ope0_j + v_j,  v_j in [0, cnt_j)          (present slots)
 //     index = t_base + sum_j v_j * istride_j             (t for GRID, u for CHAIN)
 //     sum_n = n_base + sum_j v_j                          (reading c12)
-// Box-local ordinal u in [u_begin, u_end) enumerates v in mixed radix with the
-// last slot fastest, so index(u) is increasing in u.  Every candidate of the
+// Box-local ordinal u in [u_begin, u_end) enumerates the digits in mixed radix.
+// The box digit order is: slots with cnt == 1 first, then the varying slots in
+// slot order (dpos[j] = digit of slot j), so index(u) is increasing in u and
+// digit kKMax-1 is always the fastest varying one.  Every candidate of the
 // grid (ABI abacus_grid_t) lies in exactly one
 // segment, and within a segment the Fig.-8 slot positions are
 // uniform: this is what lets a 128-row tile share one layer-1 operand.
@@ -30,15 +32,19 @@ struct SegP {
     uint64_t u_begin, u_end;  // box-local ordinal range of this shard
     uint64_t tile0;           // first work item (tile) of the segment
     uint64_t t_base;          // index of the v = 0 element
-    uint64_t istride[kKMax];  // index stride per slot (0 if absent)
-    uint64_t bstride[kKMax];  // box stride per slot (product of later cnt)
-    double rbstride[kKMax];   // 1.0 / bstride_j (uniform fp64 split of the tile base)
-    FastDiv fd[kKMax];        // divide by cnt_j
-    uint32_t cnt[kKMax];      // box radix per slot (1 if absent)
-    int32_t ope0[kKMax];      // ope at v = 0, 0 if absent
-    int32_t pos[kKMax];       // Fig.-8 position (rank by model id among present), -1 absent
+    // per box DIGIT:
+    uint64_t istride[kKMax];  // index stride (0 if absent)
+    uint64_t bstride[kKMax];  // box stride (product of later cnt)
+    double rbstride[kKMax];   // 1.0 / bstride (uniform fp64 split of the tile base)
+    FastDiv fd[kKMax];        // divide by cnt
+    uint32_t cnt[kKMax];      // box radix (1 if absent / fixed)
+    int32_t ope0[kKMax];      // per SLOT: ope at v = 0, 0 if absent
+    int32_t pos[kKMax];       // per SLOT: Fig.-8 position (rank by model id among present), -1 absent
+    int32_t dpos[kKMax];      // per SLOT: its box digit
     int32_t n_base;           // sum_n at v = 0
     uint32_t mask;            // present slots
+    uint32_t fast_carry;      // 1 if cnt[kKMax-1] >= kTileM (a tile advance carries <= 1)
+    uint32_t pad;
 };
 
 struct SlotP {

@@ -29,6 +29,7 @@ __device__ __forceinline__ int find_segment(const Plan& P, uint64_t w) {
 // segment boundaries.
 // ---------------------------------------------------------------------------
 struct Walker {
+    uint32_t fast;        // segment's fast_carry flag
     uint64_t ub;          // box ordinal of the tile's row 0
     uint64_t u_end;       // segment end (box ordinal)
     uint64_t next_tile0;  // first work item of the next segment
@@ -48,6 +49,7 @@ __device__ __forceinline__ void walker_enter(const Plan& P, Walker& W, int s, ui
     W.next_tile0 = s + 1 < P.n_seg ? P.seg[s + 1].tile0 : ~0ull;
     W.t_base = g.t_base;
     W.n_base = g.n_base;
+    W.fast = g.fast_carry;
 #pragma unroll
     for (int j = 0; j < kKMax; j++) {
         W.istride[j] = g.istride[j];
@@ -69,6 +71,19 @@ __device__ __forceinline__ void walker_next(const Plan& P, Walker& W, uint64_t w
         return;
     }
     W.ub += kTileM;
+    if (W.fast) {
+        // the fastest digit has cnt >= kTileM: every carry is 0 or 1
+        uint32_t x = W.v[kKMax - 1] + kTileM;
+        uint32_t c = x >= W.cnt[kKMax - 1] ? 1u : 0u;
+        W.v[kKMax - 1] = c ? x - W.cnt[kKMax - 1] : x;
+#pragma unroll
+        for (int j = kKMax - 2; j >= 0; j--) {
+            x = W.v[j] + c;
+            c = x >= W.cnt[j] ? 1u : 0u;
+            W.v[j] = c ? x - W.cnt[j] : x;
+        }
+        return;
+    }
     uint32_t carry = kTileM;
 #pragma unroll
     for (int j = kKMax - 1; j >= 0; j--) {

@@ -250,11 +250,9 @@ __device__ void build_l1_tables(const Plan& P, const float* __restrict__ w1b1, f
         const SegP& g = P.seg[s];
         const float* w = w1b1 + i * D;
         float c = b1[i];
+        for (int dg = 0; dg < kKMax; dg++) s_w[(s * kKMax + dg) * kHidden + i] = 0.0f;
         for (int j = 0; j < P.k; j++) {
-            if (!((g.mask >> j) & 1u)) {
-                s_w[(s * kKMax + j) * kHidden + i] = 0.0f;
-                continue;
-            }
+            if (!((g.mask >> j) & 1u)) continue;
             const SlotP& sl = P.slot[j];
             const int f = P.n_models + 4 * g.pos[j];
             c = fmaf(w[sl.model_id - 1], 1.0f, c);
@@ -262,9 +260,8 @@ __device__ void build_l1_tables(const Plan& P, const float* __restrict__ w1b1, f
             c = fmaf(w[f + 1], (float)g.ope0[j], c);
             c = fmaf(w[f + 2], (float)sl.bs, c);
             c = fmaf(w[f + 3], (float)sl.seqlen, c);
-            s_w[(s * kKMax + j) * kHidden + i] = w[f + 1];
+            s_w[(s * kKMax + g.dpos[j]) * kHidden + i] = w[f + 1];  // digit of slot j
         }
-        for (int j = P.k; j < kKMax; j++) s_w[(s * kKMax + j) * kHidden + i] = 0.0f;
         s_c[s * kHidden + i] = c;
     }
 }

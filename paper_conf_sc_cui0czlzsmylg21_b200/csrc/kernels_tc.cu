@@ -72,9 +72,8 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
         const SegP& g = P.seg[s];
         const float* w = w1b1 + n * D;
         float c = b1[n];
-        float wj[kKMax];
+        float wj[kKMax] = {0.0f, 0.0f, 0.0f, 0.0f};  // per box digit
         for (int j = 0; j < kKMax; j++) {
-            wj[j] = 0.0f;
             if (j >= P.k || !((g.mask >> j) & 1u)) continue;
             const SlotP& sl = P.slot[j];
             const int f = P.n_models + 4 * g.pos[j];
@@ -83,7 +82,7 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
             c = fmaf(w[f + 1], (float)g.ope0[j], c);
             c = fmaf(w[f + 2], (float)sl.bs, c);
             c = fmaf(w[f + 3], (float)sl.seqlen, c);
-            wj[j] = w[f + 1] * scale;
+            wj[g.dpos[j]] = w[f + 1] * scale;  // column of slot j's box digit
         }
         c *= scale;
         uint16_t ch, cl;
