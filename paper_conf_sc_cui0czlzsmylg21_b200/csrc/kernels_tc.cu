@@ -332,9 +332,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     // issuer rotates over the group's 4 warps (one per SMSP) stage by stage.
     // Slots X and Y use different barrier ids, so a warp running ahead can
     // never arrive in the wrong phase.
-    auto handoff = [&](uint32_t bar_id, uint32_t turn) -> bool {
+    auto handoff = [&](uint32_t bar_id, bool me) -> bool {
         fence_before();
-        const bool me = (uint32_t)wq == (turn & 3u);
         if (me) {
             named_bar_sync(bar_id, 128);
             fence_after();
@@ -344,7 +343,13 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         return me;
     };
     const uint32_t idX = 1 + 2 * g, idY = 2 + 2 * g;
-    uint32_t turnX = (uint32_t)g, turnY = (uint32_t)g + 2u;
+    // issuer of hand-off position p (0: L2, 1: L3, 2: out, 3: next L1) of slot X / Y
+    bool meX[4], meY[4];
+#pragma unroll
+    for (int p = 0; p < 4; p++) {
+        meX[p] = ((g + p) & 3) == wq;
+        meY[p] = ((g + 2 + p) & 3) == wq;
+    }
     auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
         const int su = __shfl_sync(0xffffffffu, s, 0);
         const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
@@ -353,13 +358,13 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         mma_commit_elect(bar);
     };
     // wait for layer l of T, epilogue (ReLU, pack) into A, hand off, issue layer l+1
-    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id,
-                     uint32_t& turn, uint32_t idesc) {
+    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id, bool me,
+                     uint32_t idesc) {
         mbar_wait(bar, ph);
         ph ^= 1u;
         fence_after();
         hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
-        if (handoff(bar_id, turn++)) {
+        if (handoff(bar_id, me)) {
             issue_layer_e<FMT>(T.d, T.a, tC, dl, idesc);
             mma_commit_elect(bar);
         }
@@ -392,16 +397,16 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         take(vY, sY, okY, zY, wb + 1);
         store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
         tmem_wait_st();
-        if (handoff(idX, turnX++)) issue_l1(X, sX, barX);
-        if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
+        if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
+        if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
 
         for (uint64_t w = wb; w < we; w += 2) {
-            stage(X, barX, phX, d2, idX, turnX, id32);
-            stage(Y, barY, phY, d2, idY, turnY, id32);
-            stage(X, barX, phX, d3, idX, turnX, id32);
-            stage(Y, barY, phY, d3, idY, turnY, id32);
-            stage(X, barX, phX, d4, idX, turnX, id16);
-            stage(Y, barY, phY, d4, idY, turnY, id16);
+            stage(X, barX, phX, d2, idX, meX[0], id32);
+            stage(Y, barY, phY, d2, idY, meY[0], id32);
+            stage(X, barX, phX, d3, idX, meX[1], id32);
+            stage(Y, barY, phY, d3, idY, meY[1], id32);
+            stage(X, barX, phX, d4, idX, meX[2], id16);
+            stage(Y, barY, phY, d4, idY, meY[2], id16);
             // X: output ready -> fold (a5) -> start tile w + 2 while Y's output MMA runs
             mbar_wait(barX, phX);
             phX ^= 1u;
@@ -417,7 +422,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             take(vX, sX, okX, zX, w + 2);
             store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
             tmem_wait_st();
-            if (handoff(idX, turnX++)) issue_l1(X, sX, barX);
+            if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
             // Y: the same, next tile w + 3
             mbar_wait(barY, phY);
             phY ^= 1u;
@@ -433,7 +438,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             take(vY, sY, okY, zY, w + 3);
             store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
             tmem_wait_st();
-            if (handoff(idY, turnY++)) issue_l1(Y, sY, barY);
+            if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
         }
         // drain the layer-1 MMAs issued for the tiles past the end
         mbar_wait(barX, phX);
