@@ -314,3 +314,21 @@ def test_validation_errors():
         assert e.value.code == ab.ABACUS_E_DUP_MODEL
     finally:
         c.close()
+
+
+def test_search_grid_nccl_single_rank(ctx):
+    """a6 through NCCL: a 1-rank communicator (all-gather + finalize kernel)
+    returns the same decision as the local path."""
+    slots = synth.cfg1_grids()[1][1]
+    T = oracle.grid_size(slots)
+    uid = ab.abacus_nccl_unique_id()
+    comm = ab.abacus_nccl_comm_init(ctx.h, 1, 0, uid)
+    try:
+        for prec in PRECS:
+            ctx.load(ctx.params, prec)
+            a = ab.abacus_search_grid(ctx.h, ab.make_grid(slots), 12.5, 0, T)
+            b = ab.abacus_search_grid(ctx.h, ab.make_grid(slots), 12.5, 0, T, comm)
+            assert (a.key, a.pred_ms, a.evaluated, list(a.end_op)) == (b.key, b.pred_ms, b.evaluated, list(b.end_op))
+    finally:
+        ab.abacus_nccl_comm_destroy(comm)
+        ctx.load(ctx.params, ab.ABACUS_FP32)
