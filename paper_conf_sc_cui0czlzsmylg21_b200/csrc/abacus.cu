@@ -13,6 +13,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -35,7 +36,9 @@ struct abacus_ctx {
     cudaStream_t stream = nullptr;      // stream of the blocking calls (default: own_stream)
     cudaStream_t own_stream = nullptr;
     Scratch* S = nullptr;         // device
-    Result* host_result = nullptr;  // pinned
+    Result* host_result = nullptr;  // pinned, host-mapped: the kernels write the decision here
+    Result* dev_result = nullptr;   // device alias of host_result
+    uint32_t seq = 0;
     std::string err;
     uint64_t launches = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -486,6 +489,35 @@ std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, f
 
 cudaStream_t pick_stream(abacus_ctx* c, void* st) { return st ? (cudaStream_t)st : c->stream; }
 
+// Wait until the kernel-side publish of sequence number `seq` is visible in
+// the mapped result (spin; the stream is polled now and then so a failed or
+// finished-without-result launch is reported instead of hanging).
+// sequence numbers are unique per process, so a recycled pinned buffer can
+// never hold a matching stale tag
+std::atomic<uint32_t> g_seq{0};
+uint32_t next_seq(abacus_ctx* c) {
+    uint32_t s = ++g_seq;
+    if (s == 0) s = ++g_seq;
+    c->host_result->seq = 0;  // cleared before the launch that will publish `s`
+    return s;
+}
+
+int wait_result(abacus_ctx* c, uint32_t seq) {
+    volatile uint32_t* s = &c->host_result->seq;
+    for (uint64_t spin = 1;; spin++) {
+        if (*s == seq) break;
+        if ((spin & 1023) == 0) {
+            const cudaError_t e = cudaStreamQuery(c->stream);
+            if (e != cudaSuccess && e != cudaErrorNotReady)
+                return fail(c, ABACUS_E_CUDA, "search kernel failed: %s", cudaGetErrorString(e));
+            if (e == cudaSuccess && *s != seq)
+                return fail(c, ABACUS_E_CUDA, "search finished without publishing its result");
+        }
+    }
+    std::atomic_thread_fence(std::memory_order_acquire);
+    return ABACUS_OK;
+}
+
 int launch_fused(abacus_ctx* c, const Plan& P) {
     int grid = 0;
     cudaError_t e;
@@ -531,13 +563,15 @@ int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, in
     bool ok = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking) == cudaSuccess &&
               cudaMalloc(&c->S, sizeof(Scratch)) == cudaSuccess &&
               cudaMemset(c->S, 0, sizeof(Scratch)) == cudaSuccess &&
-              cudaMallocHost(&c->host_result, sizeof(Result)) == cudaSuccess &&
+              cudaHostAlloc(&c->host_result, sizeof(Result), cudaHostAllocMapped) == cudaSuccess &&
+              cudaHostGetDevicePointer(&c->dev_result, c->host_result, 0) == cudaSuccess &&
               cudaEventCreate(&c->ev0) == cudaSuccess && cudaEventCreate(&c->ev1) == cudaSuccess;
     if (ok) {
         const float nan = NAN;
         ok = cudaMemcpy(&c->S->y0, &nan, sizeof(float), cudaMemcpyHostToDevice) == cudaSuccess;
     }
     c->stream = c->own_stream;
+    if (ok) memset(c->host_result, 0, sizeof(Result));
     if (!ok) {
         abacus_destroy(c);
         return ABACUS_E_CUDA;
@@ -743,12 +777,14 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
         n_eval = P.n_eval;
     }
     P.want_y0 = 1;
+    P.mapped = c->dev_result;
+    P.seq = next_seq(c);
     CUDA_TRY(c, cudaSetDevice(c->device));
     rc = launch_fused(c, P);
     if (rc) return rc;
-    CUDA_TRY(c, cudaMemcpyAsync(c->host_result, &c->S->result, sizeof(Result), cudaMemcpyDeviceToHost, c->stream));
-    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    const Result& R = *c->host_result;
+    rc = wait_result(c, P.seq);
+    if (rc) return rc;
+    const Result R = *c->host_result;
     // a7: decision assembly
     abacus_decision_t d{};
     d.critical = order[0];
@@ -785,6 +821,9 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
     CUDA_TRY(c, cudaSetDevice(c->device));
     Plan P = plan_grid_segments(c, grid, T, first, first + count, headroom_ms);
+    const uint32_t seq = next_seq(c);
+    P.mapped = nccl_comm ? nullptr : c->dev_result;  // with a combine, the finalize kernel publishes
+    P.seq = seq;
     rc = launch_fused(c, P);
     if (rc) return rc;
     if (nccl_comm) {
@@ -795,12 +834,12 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
             return fail(c, ABACUS_E_NCCL, "bad communicator");
         ncclResult_t nr = nccl().AllGather(&c->S->result, c->S->gathered, sizeof(Result), ncclUint8, comm, c->stream);
         if (nr != ncclSuccess) return fail(c, ABACUS_E_NCCL, "ncclAllGather: %s", nccl().GetErrorString(nr));
-        CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->stream));
+        CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->dev_result, seq, c->stream));
         c->launches++;
     }
-    CUDA_TRY(c, cudaMemcpyAsync(c->host_result, &c->S->result, sizeof(Result), cudaMemcpyDeviceToHost, c->stream));
-    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    const Result& R = *c->host_result;
+    rc = wait_result(c, seq);
+    if (rc) return rc;
+    const Result R = *c->host_result;
     abacus_decision_t d{};
     d.critical = 0;
     for (int j = 0; j < 4; j++) d.order[j] = j < grid->k ? j : -1;

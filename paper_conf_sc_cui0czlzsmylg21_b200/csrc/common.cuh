@@ -52,6 +52,19 @@ struct SlotP {
     int32_t end_lo, end_hi, absent, radix;  // grid digit definition (decode of t*)
 };
 
+// result record written by the last CTA (and gathered across ranks)
+struct Result {
+    unsigned long long key;  // best key, 0 = none
+    float y_best;            // y(t*)
+    float y0;                // y(index 0), NaN if not evaluated
+    unsigned long long evaluated;
+    int32_t end_op[kKMax];   // decoded t* per slot (grid order), 0 absent
+    int32_t total_ops;
+    int32_t status;          // 0 OK, 2 NONE (set by host for decisions)
+    uint32_t seq;            // mapped copy: written last, after a system fence
+    uint32_t pad;
+};
+
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
 
 struct Plan {
@@ -64,19 +77,11 @@ struct Plan {
     uint64_t T;             // size of the whole space
     uint64_t n_eval;        // candidates in this plan (this shard)
     uint64_t chain_cum[kKMax + 1];  // CHAIN: first u of block j
+    Result* mapped;         // host-mapped pinned result (device pointer) or null
+    uint32_t seq;           // sequence number the mapped copy is tagged with
+    uint32_t pad2;
     SlotP slot[kKMax];
     SegP seg[kMaxSeg];
-};
-
-// result record written by the last CTA (and gathered across ranks)
-struct Result {
-    unsigned long long key;  // best key, 0 = none
-    float y_best;            // y(t*)
-    float y0;                // y(index 0), NaN if not evaluated
-    unsigned long long evaluated;
-    int32_t end_op[kKMax];   // decoded t* per slot (grid order), 0 absent
-    int32_t total_ops;
-    int32_t status;          // 0 OK, 2 NONE (set by host for decisions)
 };
 
 struct Scratch {             // device scratch owned by the ctx

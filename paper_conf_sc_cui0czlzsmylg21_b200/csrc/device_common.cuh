@@ -169,6 +169,22 @@ __device__ __forceinline__ void decode_index_to_ope(const Plan& P, unsigned long
     }
 }
 
+// copy a result record to host-mapped pinned memory; the sequence number is
+// written last, after a system-scope fence, so a host that sees it sees the
+// whole record
+__device__ __forceinline__ void publish_mapped(const Result& R, Result* M, uint32_t seq) {
+    volatile Result* m = M;
+    m->key = R.key;
+    m->y_best = R.y_best;
+    m->y0 = R.y0;
+    m->evaluated = R.evaluated;
+    for (int j = 0; j < kKMax; j++) m->end_op[j] = R.end_op[j];
+    m->total_ops = R.total_ops;
+    m->status = R.status;
+    __threadfence_system();
+    m->seq = seq;
+}
+
 static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratch* S, unsigned long long key, float y) {
     __shared__ unsigned long long s_key[32];
     __shared__ float s_y[32];
@@ -217,6 +233,7 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
         S->y0 = __int_as_float(0x7fc00000);
         S->counter = 0;
         __threadfence();
+        if (P.mapped) publish_mapped(R, P.mapped, P.seq);
     }
 }
 

@@ -235,6 +235,29 @@ def cfg2_decisions(n: int, seed: int = 12) -> List[Tuple[List[Query], float, flo
     return out
 
 
+def cfg3_decisions(n: int, seed: int = 13, H_range=(10.0, 60.0)) -> List[Tuple[List[Query], float, float]]:
+    """4-way decisions of config 3's services (ResNet-101, ResNet-152, VGG-19,
+    BERT-large; P:2328 with Bert -> BERT-large): s ~ U[1, L], bs ~ U[1, 32],
+    BERT seqlen ~ U{16..512}; the critical headroom ~ U(H_range) ms, the others
+    +U(1, 30) ms (latency benchmarks; the streamed simulator sets real QoS)."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    out = []
+    for _ in range(n):
+        crit = int(rng.integers(0, 4))
+        H = float(rng.uniform(*H_range))
+        now, infl = 100.0, float(rng.uniform(0.0, 5.0))
+        qs = []
+        for j, m in enumerate(cfg3_services()):
+            s = int(rng.integers(1, L(m) + 1))
+            bs = int(rng.integers(1, 33))
+            sl = seqlen_for(m, int(rng.integers(16, 513)))
+            ts = float(rng.uniform(0.0, 80.0))
+            h = H if j == crit else H + float(rng.uniform(1.0, 30.0))
+            qs.append(Query(m, s, bs, sl, h + (now - ts) + infl, ts))
+        out.append((qs, now, infl))
+    return out
+
+
 def cfg3_services(seed: int = 13):
     """Config 3 services: ResNet-101, ResNet-152, VGG-19, BERT-large."""
     return [2, 3, 6, 8]

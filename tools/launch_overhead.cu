@@ -1,0 +1,72 @@
+// launch_overhead.cu -- microbenchmark: host cost of a launch vs. kernel
+// parameter size, cudaFuncSetAttribute, and result read-back styles.
+#include <chrono>
+#include <cstdio>
+#include <cuda_runtime.h>
+
+template <int BYTES>
+struct Blob { unsigned char b[BYTES]; };
+
+template <int BYTES>
+__global__ void k(const __grid_constant__ Blob<BYTES> p, int* out) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) out[0] = p.b[BYTES - 1];
+}
+__global__ void k_mapped(volatile int* host_flag, int seq) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) { __threadfence_system(); host_flag[0] = seq; }
+}
+
+static double now() { return std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now().time_since_epoch()).count(); }
+
+template <int BYTES>
+void run(cudaStream_t s, int* d) {
+    Blob<BYTES> p{};
+    p.b[BYTES - 1] = 7;
+    int* h;
+    cudaMallocHost(&h, 64);
+    double best_launch = 1e9, t_sync = 0;
+    const int N = 2000;
+    double tl = 0, ts = 0, tf = 0;
+    for (int i = 0; i < N; i++) {
+        double t0 = now();
+        k<BYTES><<<148, 128, 0, s>>>(p, d);
+        double t1 = now();
+        cudaMemcpyAsync(h, d, 4, cudaMemcpyDeviceToHost, s);
+        cudaStreamSynchronize(s);
+        double t2 = now();
+        cudaFuncSetAttribute(k<BYTES>, cudaFuncAttributeMaxDynamicSharedMemorySize, 1024);
+        double t3 = now();
+        if (i >= 100) { tl += t1 - t0; ts += t2 - t0; tf += t3 - t2; }
+    }
+    printf("param %6d B: launch call %6.2f us, launch+memcpy+sync %6.2f us, cudaFuncSetAttribute %6.2f us\n",
+           BYTES, tl / (N - 100), ts / (N - 100), tf / (N - 100));
+    cudaFreeHost(h);
+}
+
+int main() {
+    cudaStream_t s;
+    cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    int* d;
+    cudaMalloc(&d, 64);
+    run<64>(s, d);
+    run<1024>(s, d);
+    run<4096>(s, d);
+    run<8192>(s, d);
+    run<16384>(s, d);
+    // mapped pinned flag polling instead of memcpy + sync
+    int* hf;
+    cudaHostAlloc(&hf, 64, cudaHostAllocMapped);
+    int* df;
+    cudaHostGetDevicePointer(&df, hf, 0);
+    double tp = 0;
+    const int N = 2000;
+    for (int i = 1; i <= N; i++) {
+        double t0 = now();
+        k_mapped<<<1, 32, 0, s>>>(df, i);
+        while (*(volatile int*)hf != i) {}
+        double t1 = now();
+        if (i > 100) tp += t1 - t0;
+    }
+    printf("launch + mapped-flag poll: %6.2f us\n", tp / (N - 100));
+    cudaStreamSynchronize(s);
+    return 0;
+}
