@@ -213,17 +213,26 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
     __syncthreads();
     if (!s_last) return;
     __threadfence();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x < 32) {
+        // warp 0 reduces the per-CTA records (independent loads, then shuffles)
         unsigned long long bk = 0;
         float by = __int_as_float(0x7fc00000);
-        for (unsigned int b = 0; b < gridDim.x; b++) {
-            const unsigned long long kk = *((volatile unsigned long long*)&S->cta_key[b]);
-            if (kk > bk) { bk = kk; by = *((volatile float*)&S->cta_y[b]); }
+        for (unsigned int b = threadIdx.x; b < gridDim.x; b += 32) {
+            const unsigned long long kk = __ldcg(&S->cta_key[b]);
+            const float yy = __ldcg(&S->cta_y[b]);
+            if (kk > bk) { bk = kk; by = yy; }
         }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, bk, o);
+            const float y2 = __shfl_xor_sync(0xffffffffu, by, o);
+            if (k2 > bk) { bk = k2; by = y2; }
+        }
+        if (threadIdx.x != 0) return;
         Result& R = S->result;
         R.key = bk;
         R.y_best = by;
-        R.y0 = *((volatile float*)&S->y0);
+        R.y0 = __ldcg(&S->y0);
         R.evaluated = P.n_eval;
         int32_t ope[kKMax];
         decode_index_to_ope(P, bk & ((1ull << 40) - 1), ope);

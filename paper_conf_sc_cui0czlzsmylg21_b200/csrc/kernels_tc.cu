@@ -24,6 +24,8 @@
 #include <cuda_runtime.h>
 #include <math.h>
 
+#include <type_traits>
+
 #include "common.cuh"
 #include "device_common.cuh"
 #include "internal.h"
@@ -209,6 +211,12 @@ __host__ __device__ inline TcSmem tc_smem_layout(int n_l1_tables, uint32_t l1_ta
     return L;
 }
 
+// per-"group" share of the stage area that holds W1 | b1 (fp32) for the table build
+__host__ __device__ inline uint32_t w1_stage_bytes(int D, int ng) {
+    const uint32_t total = (uint32_t)(kHidden * D + kHidden) * 4u;
+    return (total + (uint32_t)ng * 16u - 1u) / ((uint32_t)ng * 16u) * 16u;
+}
+
 // ---------------------------------------------------------------------------
 // fused search
 //
@@ -265,7 +273,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                                                                const float* __restrict__ w1b1, Scratch* S) {
     extern __shared__ __align__(1024) uint8_t smem[];
     using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * NG, 0);
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * NG, w1_stage_bytes(P.D, 2 * NG));
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);  // 2 per group
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
 
@@ -277,8 +285,12 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         const int4* src = reinterpret_cast<const int4*>(TP.blob);
         int4* dst = reinterpret_cast<int4*>(smem);
         for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+        // stage W1 | b1 (fp32) for the layer-1 table build
+        float* s_w1 = reinterpret_cast<float*>(smem + L.stage);
+        for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
     }
-    build_b1_fused<FMT, SPLIT>(P, w1b1, TP.l1_scale, smem + L.b1);
+    __syncthreads();
+    build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1);
     if (tid == 0) {
         for (int i = 0; i < 2 * NG; i++) mbar_init(&bars[i], 1);
         mbar_fence_init();
@@ -380,33 +392,38 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         uint32_t vX[kKMax], vY[kKMax];
         int sX, sY;
         bool okX, okY, zX, zY;
-        auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z, uint64_t w) {
-            ok = w < we && (W.u_end - W.ub > (uint64_t)r);
-            z = w < we && walker_is_index0(W, r);
+        auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z) {
+            ok = W.u_end - W.ub > (uint64_t)r;
+            z = walker_is_index0(W, r);
 #pragma unroll
             for (int j = 0; j < kKMax; j++) v[j] = W.v[j];
             s = W.s;
         };
-        auto advance = [&](uint64_t w_next) {
-            if (w_next < we) walker_next(P, W, w_next, r);
-        };
-        // prologue: tiles wb (X) and wb + 1 (Y)
-        take(vX, sX, okX, zX, wb);
+        // prologue: tile wb in slot X and (if the group has it) wb + 1 in slot Y
+        bool xLive = true, yLive = wb + 1 < we;  // warp-uniform
+        take(vX, sX, okX, zX);
         store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
-        advance(wb + 1);
-        take(vY, sY, okY, zY, wb + 1);
-        store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+        if (yLive) {
+            walker_next(P, W, wb + 1, r);
+            take(vY, sY, okY, zY);
+            store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+        }
         tmem_wait_st();
         if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
-        if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
+        if (yLive && handoff(idY, meY[3])) issue_l1(Y, sY, barY);
 
-        for (uint64_t w = wb; w < we; w += 2) {
+        // one iteration = the remaining layers of the tiles in X and Y, then the
+        // next tiles (w + 2, w + 3) enter the slots.  GUARDED = the tail, where a
+        // slot may be empty or have no successor; the steady state skips the checks.
+        uint64_t w = wb;
+        auto iteration = [&](auto guarded_c) {
+            constexpr bool G = decltype(guarded_c)::value;
             stage(X, barX, phX, d2, idX, meX[0], id32);
-            stage(Y, barY, phY, d2, idY, meY[0], id32);
+            if (!G || yLive) stage(Y, barY, phY, d2, idY, meY[0], id32);
             stage(X, barX, phX, d3, idX, meX[1], id32);
-            stage(Y, barY, phY, d3, idY, meY[1], id32);
+            if (!G || yLive) stage(Y, barY, phY, d3, idY, meY[1], id32);
             stage(X, barX, phX, d4, idX, meX[2], id16);
-            stage(Y, barY, phY, d4, idY, meY[2], id16);
+            if (!G || yLive) stage(Y, barY, phY, d4, idY, meY[2], id16);
             // X: output ready -> fold (a5) -> start tile w + 2 while Y's output MMA runs
             mbar_wait(barX, phX);
             phX ^= 1u;
@@ -418,31 +435,39 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                 if (okX && zX) S->y0 = y;
                 if (okX) fold_tile(P, sX, vX, y, best, best_y);
             }
-            advance(w + 2);
-            take(vX, sX, okX, zX, w + 2);
-            store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
-            tmem_wait_st();
-            if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
-            // Y: the same, next tile w + 3
-            mbar_wait(barY, phY);
-            phY ^= 1u;
-            fence_after();
-            {
-                uint32_t yb;
-                tmem_ld1(Y.d + lane_off, yb);
-                const float y = __uint_as_float(yb);
-                if (okY && zY) S->y0 = y;
-                if (okY) fold_tile(P, sY, vY, y, best, best_y);
+            if (G) xLive = w + 2 < we;
+            if (!G || xLive) {
+                walker_next(P, W, w + 2, r);
+                take(vX, sX, okX, zX);
+                store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
+                tmem_wait_st();
+                if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
             }
-            advance(w + 3);
-            take(vY, sY, okY, zY, w + 3);
-            store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
-            tmem_wait_st();
-            if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
-        }
-        // drain the layer-1 MMAs issued for the tiles past the end
-        mbar_wait(barX, phX);
-        mbar_wait(barY, phY);
+            if (!G || yLive) {
+                // Y: the same, next tile w + 3
+                mbar_wait(barY, phY);
+                phY ^= 1u;
+                fence_after();
+                {
+                    uint32_t yb;
+                    tmem_ld1(Y.d + lane_off, yb);
+                    const float y = __uint_as_float(yb);
+                    if (okY && zY) S->y0 = y;
+                    if (okY) fold_tile(P, sY, vY, y, best, best_y);
+                }
+                if (G) yLive = w + 3 < we;
+                if (!G || yLive) {
+                    walker_next(P, W, w + 3, r);
+                    take(vY, sY, okY, zY);
+                    store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+                    tmem_wait_st();
+                    if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
+                }
+            }
+            w += 2;
+        };
+        while (w + 3 < we) iteration(std::integral_constant<bool, false>{});  // both slots full, both continue
+        while (xLive) iteration(std::integral_constant<bool, true>{});
     }
     fence_before();
     __syncthreads();
@@ -646,12 +671,13 @@ template <int FMT, bool SPLIT>
 static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const OutW& ow, const float* w1b1,
                                     Scratch* S, int nsm, cudaStream_t st, int* grid_out) {
     using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG, 0);
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG,
+                                         w1_stage_bytes(P.D, 2 * kFusedNG));
     auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
-    // two tiles in flight per group: spread the tiles over as many SMs as possible
-    uint64_t g = (P.n_tiles + 2 * kFusedNG - 1) / (2 * kFusedNG);
+    // spread the tiles over as many SMs as possible (one tile per group first)
+    uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     *grid_out = (int)g;

@@ -35,7 +35,7 @@ __global__ void __launch_bounds__(640, 1) kern(const __grid_constant__ P5K p, in
         if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(slot));
     }
     if (threadIdx.x == 0) {
-        out[0] = p.b[4999] + smem[7];
+        out[0] = p.b[4999] + ((VARIANT & 8) ? smem[7] : 0);
         if (VARIANT & 4) { __threadfence_system(); mapped[0] = 1; }
     }
 }
