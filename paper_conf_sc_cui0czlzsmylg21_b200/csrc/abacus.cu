@@ -147,17 +147,29 @@ int validate_grid(abacus_ctx* c, const abacus_grid_t* g, uint64_t* T_out) {
 }
 
 // ---- plans ------------------------------------------------------------------
+void fill_strides(Plan& P) {
+    uint64_t b = 1;
+    for (int j = kKMax - 1; j >= 0; j--) {
+        P.slot[j].tstride = b;
+        P.slot[j].rtstride = 1.0 / (double)b;
+        if (j < P.k) b *= (uint64_t)P.slot[j].radix;
+    }
+}
+
 void fill_slots(Plan& P, const abacus_grid_t* g) {
     for (int j = 0; j < kKMax; j++) {
         SlotP& s = P.slot[j];
         if (j < g->k) {
             const abacus_slot_t& a = g->slot[j];
-            s = SlotP{a.model_id, a.start_op, a.batch, a.seqlen, a.end_lo, a.end_hi, a.allow_absent,
-                      a.allow_absent + a.end_hi - a.end_lo + 1};
+            const int32_t radix = a.allow_absent + a.end_hi - a.end_lo + 1;
+            s = SlotP{a.model_id, a.start_op, a.batch, a.seqlen, a.end_lo, a.end_hi, a.allow_absent, radix,
+                      1.0 / (double)radix};
         } else {
-            s = SlotP{0, 0, 0, 0, 0, 0, 0, 1};
+            s = SlotP{0, 0, 0, 0, 0, 0, 0, 1, 1.0};
         }
     }
+    P.k = g->k;
+    fill_strides(P);
 }
 
 void finish_box(SegP& s) {
@@ -518,7 +530,11 @@ int wait_result(abacus_ctx* c, uint32_t seq) {
     return ABACUS_OK;
 }
 
-int launch_fused(abacus_ctx* c, const Plan& P) {
+unsigned long long* trace_ptr();
+
+int launch_fused(abacus_ctx* c, const Plan& Pin) {
+    Plan P = Pin;
+    P.trace = trace_ptr();
     int grid = 0;
     cudaError_t e;
     if (c->timed) cudaEventRecord(c->ev0, c->stream);
@@ -534,6 +550,11 @@ int launch_fused(abacus_ctx* c, const Plan& P) {
     return ABACUS_OK;
 }
 
+}  // namespace
+
+static unsigned long long* g_trace_ptr = nullptr;
+namespace {
+unsigned long long* trace_ptr() { return g_trace_ptr; }
 }  // namespace
 
 // ============================================================================
@@ -881,6 +902,13 @@ int abacus_nccl_comm_init(abacus_ctx* c, int32_t nranks, int32_t rank, const uin
 
 void abacus_nccl_comm_destroy(void* comm) {
     if (comm && nccl().ok) nccl().CommDestroy((ncclComm_t)comm);
+}
+
+// not in the ABI header (tools/kernel_trace.py): device array of 8 globaltimer
+// stamps the next fused launches write from CTA 0 (null disables)
+int abacus_internal_set_trace(void* d_stamps) {
+    g_trace_ptr = (unsigned long long*)d_stamps;
+    return ABACUS_OK;
 }
 
 int abacus_set_stream(abacus_ctx* c, void* stream) {

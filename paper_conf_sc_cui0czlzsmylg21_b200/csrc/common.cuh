@@ -50,6 +50,9 @@ struct SegP {
 struct SlotP {
     int32_t model_id, ops, bs, seqlen;
     int32_t end_lo, end_hi, absent, radix;  // grid digit definition (decode of t*)
+    double rradix;                           // 1.0 / radix (fp64 quotient in the decode)
+    uint64_t tstride;                        // product of the later radices
+    double rtstride;                         // 1.0 / tstride
 };
 
 // result record written by the last CTA (and gathered across ranks)
@@ -78,6 +81,7 @@ struct Plan {
     uint64_t n_eval;        // candidates in this plan (this shard)
     uint64_t chain_cum[kKMax + 1];  // CHAIN: first u of block j
     Result* mapped;         // host-mapped pinned result (device pointer) or null
+    unsigned long long* trace;  // optional %globaltimer stamps (tools only), null in production
     uint32_t seq;           // sequence number the mapped copy is tagged with
     uint32_t pad2;
     SlotP slot[kKMax];

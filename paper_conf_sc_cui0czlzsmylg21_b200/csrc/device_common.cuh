@@ -146,26 +146,39 @@ __device__ __forceinline__ bool walker_is_index0(const Walker& W, uint32_t r) {
 // Each CTA publishes its best (key, y); the last CTA to arrive reduces them,
 // decodes the winning index into end ops per slot and resets the ticket.
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ void decode_index_to_ope(const Plan& P, unsigned long long idx, int32_t (&ope)[kKMax]) {
-#pragma unroll
-    for (int j = 0; j < kKMax; j++) ope[j] = 0;
+// q = floor(a / b) for a < 2^40 via an fp64 reciprocal (exact after one correction)
+__device__ __forceinline__ unsigned long long div_rcp(unsigned long long a, unsigned long long b, double rb) {
+    unsigned long long q = (unsigned long long)((double)a * rb);
+    const long long rem = (long long)(a - q * b);
+    if (rem < 0) q--;
+    else if (rem >= (long long)b) q++;
+    return q;
+}
+
+// End op of slot `j` of the candidate with index idx (GRID: digit j of the
+// mixed-radix index, computed directly so lanes can decode slots in parallel;
+// CHAIN: block structure).  0 = absent.
+__device__ __forceinline__ int32_t decode_slot_ope(const Plan& P, unsigned long long idx, int j) {
     if (P.mode == kModeGrid) {
-        unsigned long long t = idx;
-        for (int j = P.k - 1; j >= 0; j--) {
-            const unsigned long long r = (unsigned long long)P.slot[j].radix;
-            const uint32_t d = (uint32_t)(t % r);
-            t /= r;
-            ope[j] = digit_to_ope(P.slot[j], d);
-        }
-    } else {
-        int blk = 0;
-        for (int j = 1; j < P.k; j++)
-            if (idx >= P.chain_cum[j]) blk = j;
-        for (int j = 0; j < P.k; j++) {
-            if (j < blk) ope[j] = P.slot[j].end_hi;
-            else if (j == blk) ope[j] = blk == 0 ? P.slot[0].end_hi
-                                                  : P.slot[j].ops + (int32_t)(idx - P.chain_cum[j]);
-        }
+        const SlotP& s = P.slot[j];
+        const unsigned long long q = div_rcp(idx, s.tstride, s.rtstride);
+        const unsigned long long q2 = div_rcp(q, (unsigned long long)s.radix, s.rradix);
+        return digit_to_ope(s, (uint32_t)(q - q2 * (unsigned long long)s.radix));
+    }
+    int blk = 0;
+    for (int i = 1; i < P.k; i++)
+        if (idx >= P.chain_cum[i]) blk = i;
+    if (j < blk) return P.slot[j].end_hi;
+    if (j == blk) return blk == 0 ? P.slot[0].end_hi : P.slot[j].ops + (int32_t)(idx - P.chain_cum[j]);
+    return 0;
+}
+
+// optional timeline stamps (CTA 0, thread 0): tools/kernel_trace.py
+__device__ __forceinline__ void trace_stamp(const Plan& P, int slot) {
+    if (P.trace && blockIdx.x == 0 && threadIdx.x == 0) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        P.trace[slot] = t;
     }
 }
 
@@ -181,8 +194,8 @@ __device__ __forceinline__ void publish_mapped(const Result& R, Result* M, uint3
     for (int j = 0; j < kKMax; j++) m->end_op[j] = R.end_op[j];
     m->total_ops = R.total_ops;
     m->status = R.status;
-    __threadfence_system();
-    m->seq = seq;
+    // release at system scope: the record is visible before the tag
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(&M->seq), "r"(seq) : "memory");
 }
 
 static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratch* S, unsigned long long key, float y) {
@@ -199,50 +212,74 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
     const int warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     if ((threadIdx.x & 31) == 0) { s_key[warp] = key; s_y[warp] = y; }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long bk = 0;
-        float by = __int_as_float(0x7fc00000);
-        for (int w = 0; w < nwarps; w++)
-            if (s_key[w] > bk) { bk = s_key[w]; by = s_y[w]; }
-        S->cta_key[blockIdx.x] = bk;
-        S->cta_y[blockIdx.x] = by;
-        __threadfence();
-        const unsigned int ticket = atomicAdd(&S->counter, 1u);
-        s_last = ticket == gridDim.x - 1;
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
     if (threadIdx.x < 32) {
-        // warp 0 reduces the per-CTA records (independent loads, then shuffles)
-        unsigned long long bk = 0;
-        float by = __int_as_float(0x7fc00000);
-        for (unsigned int b = threadIdx.x; b < gridDim.x; b += 32) {
-            const unsigned long long kk = __ldcg(&S->cta_key[b]);
-            const float yy = __ldcg(&S->cta_y[b]);
-            if (kk > bk) { bk = kk; by = yy; }
-        }
+        unsigned long long bk = threadIdx.x < (unsigned)nwarps ? s_key[threadIdx.x] : 0ull;
+        float by = threadIdx.x < (unsigned)nwarps ? s_y[threadIdx.x] : __int_as_float(0x7fc00000);
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, bk, o);
             const float y2 = __shfl_xor_sync(0xffffffffu, by, o);
             if (k2 > bk) { bk = k2; by = y2; }
         }
+    if (threadIdx.x == 0) {
+        S->cta_key[blockIdx.x] = bk;
+        S->cta_y[blockIdx.x] = by;
+        __threadfence();
+        const unsigned int ticket = atomicAdd(&S->counter, 1u);
+        s_last = ticket == gridDim.x - 1;
+    }
+    }
+    __syncthreads();
+    trace_stamp(P, 5);
+    if (!s_last) return;
+    __threadfence();
+    trace_stamp(P, 8);
+    if (threadIdx.x < 32) {
+        // warp 0 reduces the per-CTA records (independent loads, then shuffles)
+        unsigned long long bk = 0;
+        float by = __int_as_float(0x7fc00000);
+        const float y0 = __ldcg(&S->y0);
+        constexpr int kPer = 16;  // grid <= 512 CTAs: all loads in flight at once
+        unsigned long long kk[kPer];
+        float yy[kPer];
+#pragma unroll
+        for (int i = 0; i < kPer; i++) {
+            const unsigned int b = threadIdx.x + 32u * i;
+            kk[i] = b < gridDim.x ? __ldcg(&S->cta_key[b]) : 0ull;
+            yy[i] = b < gridDim.x ? __ldcg(&S->cta_y[b]) : 0.0f;
+        }
+#pragma unroll
+        for (int i = 0; i < kPer; i++)
+            if (kk[i] > bk) { bk = kk[i]; by = yy[i]; }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, bk, o);
+            const float y2 = __shfl_xor_sync(0xffffffffu, by, o);
+            if (k2 > bk) { bk = k2; by = y2; }
+        }
+        trace_stamp(P, 9);
+        // a7: lane j decodes slot j's end op of t*
+        const int32_t my_ope = (threadIdx.x < (unsigned)P.k && bk)
+                                   ? decode_slot_ope(P, bk & ((1ull << 40) - 1), (int)threadIdx.x)
+                                   : 0;
+        int32_t ope[kKMax];
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) ope[j] = __shfl_sync(0xffffffffu, my_ope, j);
         if (threadIdx.x != 0) return;
+        trace_stamp(P, 10);
         Result& R = S->result;
         R.key = bk;
         R.y_best = by;
-        R.y0 = __ldcg(&S->y0);
+        R.y0 = y0;
         R.evaluated = P.n_eval;
-        int32_t ope[kKMax];
-        decode_index_to_ope(P, bk & ((1ull << 40) - 1), ope);
-        for (int j = 0; j < kKMax; j++) R.end_op[j] = bk ? ope[j] : 0;
+        for (int j = 0; j < kKMax; j++) R.end_op[j] = ope[j];
         R.total_ops = bk ? (int32_t)(bk >> 40) - 1 : 0;
         R.status = bk ? 0 : 2;
         S->y0 = __int_as_float(0x7fc00000);
-        S->counter = 0;
-        __threadfence();
+        S->counter = 0;  // visible to the next launch (kernel boundary)
+        trace_stamp(P, 6);
         if (P.mapped) publish_mapped(R, P.mapped, P.seq);
+        trace_stamp(P, 7);
     }
 }
 

@@ -280,6 +280,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     const int tid = threadIdx.x;
     const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform for the compiler
     const int g = warp >> 2, wq = warp & 3;
+    trace_stamp(P, 0);
 
     {
         const int4* src = reinterpret_cast<const int4*>(TP.blob);
@@ -290,6 +291,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
     }
     __syncthreads();
+    trace_stamp(P, 1);
     build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1);
     if (tid == 0) {
         for (int i = 0; i < 2 * NG; i++) mbar_init(&bars[i], 1);
@@ -304,6 +306,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     __syncthreads();
     fence_after();
     const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
+    trace_stamp(P, 2);
 
     // TMEM: group g owns 96 columns at 96 g: D_X [0,32) D_Y [32,64) A_X [64,80)
     // A_Y [80,96); the layer-1 operand A1 aliases the first 8 columns of A.
@@ -469,10 +472,12 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         while (w + 3 < we) iteration(std::integral_constant<bool, false>{});  // both slots full, both continue
         while (xLive) iteration(std::integral_constant<bool, true>{});
     }
+    trace_stamp(P, 3);
     fence_before();
     __syncthreads();
     fence_after();
     if (warp == 0) tmem_dealloc(tbase, 512);
+    trace_stamp(P, 4);
     cta_publish_and_finish(P, S, best, best_y);
 }
 
