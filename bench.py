@@ -172,7 +172,9 @@ def main():
 
     ctx = ab.abacus_create(local, list(synth.OPS_PER_MODEL))
     ab.abacus_load_predictor(ctx, params, PREC[args.precision])
-    stream = torch.cuda.current_stream()
+    # an explicit (non-legacy) stream shared by the library and the timing events
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     ab.abacus_set_stream(ctx, stream)
     ab.abacus_set_timing(ctx, True)
     comm = ab.nccl_comm_from_process_group(ctx) if world > 1 else None
@@ -219,7 +221,7 @@ def main():
     # ---- per-decision latency (config 2, 3-way; 1 GPU each) -----------------
     dec = None
     if rank == 0 and not args.no_decisions:
-        dec = decision_latency(ab, ctx)
+        dec = decision_latency(ab, ctx, precision=args.precision)
 
     if rank == 0:
         pk, src = peaks()
@@ -267,24 +269,34 @@ def main():
         dist.destroy_process_group()
 
 
-def decision_latency(ab, ctx, n=10_000, warm=100):
-    """Host wall clock around each blocking abacus_search (launch + kernel +
-    decision in host memory), config 2 (3-way), GRID space."""
+def decision_latency(ab, ctx, n=10_000, warm=100, precision="fp16"):
+    """Per-decision latency, host steady clock around each blocking
+    abacus_search: (a) through the C ABI (tools/decision_latency.c, no Python
+    on the path) for config 2 (3-way GRID) and config 3 (4-way: CHAIN, AUTO
+    with two budgets); (b) through the Python binding for config 2."""
+    out = {}
+    try:
+        sys.path.insert(0, os.path.join(ROOT, "tools"))
+        import decision_latency as dl
+        for cfg, space, budget in (("cfg2", "grid", 0), ("cfg3", "chain", 0), ("cfg3", "auto", 1 << 20),
+                                   ("cfg3", "auto", 1 << 22)):
+            key = "%s_%s" % (cfg, space) + ("_%d" % budget if space == "auto" else "")
+            out[key] = dl.run(cfg, space, precision, n, warm, budget or 4_194_304)
+    except Exception as e:  # noqa: BLE001 -- report, do not fail the bench line
+        out["c_abi_error"] = repr(e)
     decs = synth.cfg2_decisions(n + warm)
     lat = []
-    sizes = []
     for i, (qs, now, infl) in enumerate(decs):
         t0 = time.perf_counter()
-        d = ab.abacus_search(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID)
+        ab.abacus_search(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID)
         t1 = time.perf_counter()
         if i >= warm:
             lat.append((t1 - t0) * 1e6)
-            sizes.append(d.evaluated)
     a = np.array(lat)
-    return {"workload": "cfg2 3-way (ResNet-101, Inception-v3, BERT-base), GRID", "decisions": n,
-            "p50_us": float(np.percentile(a, 50)), "p99_us": float(np.percentile(a, 99)),
-            "p999_us": float(np.percentile(a, 99.9)), "grid_p50": float(np.percentile(sizes, 50)),
-            "grid_max": int(max(sizes))}
+    out["cfg2_grid_python"] = {"decisions": n, "p50_us": float(np.percentile(a, 50)),
+                               "p99_us": float(np.percentile(a, 99)), "p999_us": float(np.percentile(a, 99.9)),
+                               "path": "Python binding (ctypes) -> abacus_search"}
+    return out
 
 
 if __name__ == "__main__":

@@ -10,10 +10,25 @@ EPS = {ab.ABACUS_FP32: 1e-4, ab.ABACUS_BF16: 1e-2, ab.ABACUS_FP16: 1e-2}
 NAMES = {ab.ABACUS_FP32: "fp32", ab.ABACUS_BF16: "bf16", ab.ABACUS_FP16: "fp16"}
 
 
+_STREAM = None
+
+
+def stream():
+    """One explicit non-default stream for all GPU tests (the ABI maps a NULL
+    stream to the ctx's own stream, which is not ordered with torch's legacy
+    default stream)."""
+    global _STREAM
+    if _STREAM is None:
+        _STREAM = torch.cuda.Stream()
+        torch.cuda.set_stream(_STREAM)
+    return _STREAM
+
+
 class Ctx:
     def __init__(self, ops=None, params=None, precision=ab.ABACUS_FP32):
         self.ops = list(synth.OPS_PER_MODEL) if ops is None else list(ops)
         self.h = ab.abacus_create(0, self.ops)
+        ab.abacus_set_stream(self.h, stream())
         if params is not None:
             self.load(params, precision)
 
@@ -32,14 +47,14 @@ class Ctx:
     def encode(self, slots, first, count):
         x = torch.full((max(count, 1), self.D), -7, dtype=torch.int16, device="cuda")
         ab.abacus_encode_candidates(self.h, ab.make_grid(slots), first, count, x,
-                                    torch.cuda.current_stream())
+                                    stream())
         torch.cuda.synchronize()
         return x[:count].cpu().numpy()
 
     def predict(self, X):
         x = torch.from_numpy(np.ascontiguousarray(X, dtype=np.int16)).cuda()
         y = torch.full((max(len(X), 1),), float("nan"), dtype=torch.float32, device="cuda")
-        ab.abacus_predict_batch(self.h, x, len(X), y, torch.cuda.current_stream())
+        ab.abacus_predict_batch(self.h, x, len(X), y, stream())
         torch.cuda.synchronize()
         return y[:len(X)].cpu().numpy().astype(np.float64)
 
@@ -48,7 +63,7 @@ class Ctx:
         g = torch.frombuffer(bytearray(raw), dtype=torch.uint8).cuda()
         x = torch.full((max(len(groups), 1), self.D), -7, dtype=torch.int16, device="cuda")
         bad = torch.zeros(1, dtype=torch.int32, device="cuda")
-        ab.abacus_encode_groups(self.h, g, len(groups), x, bad, torch.cuda.current_stream())
+        ab.abacus_encode_groups(self.h, g, len(groups), x, bad, stream())
         torch.cuda.synchronize()
         return x[:len(groups)].cpu().numpy(), int(bad.item())
 
@@ -56,7 +71,7 @@ class Ctx:
         lat = torch.from_numpy(np.ascontiguousarray(y, dtype=np.float32)).cuda()
         best = torch.tensor([init], dtype=torch.int64, device="cuda")
         ab.abacus_select_group(self.h, ab.make_grid(slots), first, len(y), lat, H, best,
-                               torch.cuda.current_stream())
+                               stream())
         torch.cuda.synchronize()
         return int(best.item()) & (2**64 - 1)
 

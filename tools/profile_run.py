@@ -24,6 +24,9 @@ ap.add_argument("--decisions", type=int, default=0)
 a = ap.parse_args()
 prec = {"fp32": 0, "bf16": 1, "fp16": 2}[a.precision]
 ctx = ab.abacus_create(0, list(synth.OPS_PER_MODEL))
+_st = torch.cuda.Stream()
+torch.cuda.set_stream(_st)
+ab.abacus_set_stream(ctx, _st)
 ab.abacus_load_predictor(ctx, synth.weights(1), prec)
 slots = synth.cfg4_grid()
 T = 1
