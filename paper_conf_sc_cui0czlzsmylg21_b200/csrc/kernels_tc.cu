@@ -516,6 +516,12 @@ __device__ void build_b1_predict(const float* __restrict__ w1b1, int D, float sc
     }
 }
 
+// Pipelined like the fused kernel: NG groups x 2 tile slots (X, Y).  Per slot
+// 64 TMEM columns: D [0,32) and an operand region U [32,64) that holds the
+// layer-1 operand (features split 256 hi + lo, 4 K-chunks) and, after the
+// layer-1 MMA, the activations A = U[0,16) plus the bias constant chunk
+// U[16,24) = (1, 1, 0, ...).  Each slot's 128 feature rows are brought into
+// shared memory by a 1-D TMA bulk copy one slot-cycle ahead of use.
 template <int FMT, int NG>
 __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_constant__ TcParams TP,
                                                                  const float* __restrict__ w1b1, int32_t D,
@@ -523,12 +529,17 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
                                                                  float* __restrict__ y) {
     extern __shared__ __align__(1024) uint8_t smem[];
     using C = TcCfg<FMT>;
-    const int nch = (2 * D + 2 + 15) / 16;                 // layer-1 K chunks (A1 columns = 8 nch)
-    const uint32_t stage_bytes = (uint32_t)(kTileM * D * 2 + 15) & ~15u;
-    const TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, NG, stage_bytes);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    const int nch = (2 * D + 2 + 15) / 16;  // layer-1 K chunks (<= 4 for D <= 31)
+    const uint32_t row_bytes = (uint32_t)D * 2u;
+    const uint32_t stage_bytes = (kTileM * row_bytes + 127u) & ~127u;
+    const TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, 2 * NG, stage_bytes);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);  // per group: mma X, mma Y
+    uint64_t* tbars = reinterpret_cast<uint64_t*>(smem + L.tmem_slot + 16);  // per group: tma X, tma Y
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
-    const int tid = threadIdx.x, warp = tid >> 5, g = warp >> 2, wq = warp & 3;
+    const int tid = threadIdx.x;
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+    const int g = warp >> 2, wq = warp & 3;
+    const uint32_t lane = (uint32_t)(tid & 31);
 
     {
         const int4* src = reinterpret_cast<const int4*>(TP.blob);
@@ -537,7 +548,10 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
     }
     build_b1_predict<FMT>(w1b1, D, TP.l1_scale, smem + L.b1, nch);
     if (tid == 0) {
-        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        for (int i = 0; i < 2 * NG; i++) {
+            mbar_init(&bars[i], 1);
+            mbar_init(&tbars[i], 1);
+        }
         mbar_fence_init();
     }
     if (warp == 0) {
@@ -548,47 +562,106 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
     fence_before();
     __syncthreads();
     fence_after();
-    const uint32_t tbase = *tmem_slot;
+    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
 
-    // per group: D 32 cols, A1 8*nch cols (<= 48), A 16 cols, C 8 cols -> 128-column slice
-    const uint32_t col = (uint32_t)g * 128u;
+    const uint32_t col = tbase + (uint32_t)g * 128u;
     const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-    const uint32_t tD = tbase + col, tA1 = tbase + col + 32, tA = tbase + col + 32 + 8 * (uint32_t)nch;
-    const uint32_t tC = tA + 16;
-    {
-        uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
-        tmem_st8(tC + lane_off, c8);
-        tmem_wait_st();
-    }
-    const bool leader = (tid & 127) == 0;
+    const TileIO X{col + 0, col + 32, col + 32}, Y{col + 64, col + 96, col + 96};
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    const uint32_t w2a = sbase + L.w2, w3a = sbase + L.w3, w4a = sbase + L.w4, b1a = sbase + L.b1;
     constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
-    uint64_t* bar = &bars[g];
-    int16_t* stage = reinterpret_cast<int16_t*>(smem + L.stage + (uint32_t)g * stage_bytes);
-    uint32_t phase = 0;
-    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    uint64_t* barX = &bars[2 * g];
+    uint64_t* barY = &bars[2 * g + 1];
+    uint64_t* tbX = &tbars[2 * g];
+    uint64_t* tbY = &tbars[2 * g + 1];
+    uint32_t phX = 0, phY = 0, tphX = 0, tphY = 0;
+    uint8_t* stX = smem + L.stage + (uint32_t)(2 * g) * stage_bytes;
+    uint8_t* stY = stX + stage_bytes;
+    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
+#pragma unroll
+    for (int i = 0; i < C::kNchHid; i++) {
+        d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
+        d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
+    }
+#pragma unroll
+    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
+    const uint64_t d1base = smem_desc(sbase + L.b1);
+    const uint32_t idX = 1 + 2 * g, idY = 2 + 2 * g;
+    bool meX[4], meY[4];
+#pragma unroll
+    for (int p = 0; p < 4; p++) {
+        meX[p] = ((g + p) & 3) == wq;
+        meY[p] = ((g + 2 + p) & 3) == wq;
+    }
+    const bool tma_ok = (row_bytes % 16u) == 0 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0;
 
-    for (uint64_t w = (uint64_t)blockIdx.x * NG + g; w < n_tiles; w += (uint64_t)gridDim.x * NG) {
+    auto handoff = [&](uint32_t bar_id, bool me) -> bool {
+        fence_before();
+        if (me) {
+            named_bar_sync(bar_id, 128);
+            fence_after();
+        } else {
+            named_bar_arrive(bar_id, 128);
+        }
+        return me;
+    };
+    auto issue_l1 = [&](const TileIO& T, uint64_t* bar) {
+        for (int cb = 0; cb < nch; cb++)
+            mma_ts_elect(T.d, T.a1 + 8 * cb, d1base + (uint64_t)(cb * (kChunkBytesN32 >> 4)), id32,
+                         cb > 0 ? 1u : 0u);
+        if (FMT == 1)
+            for (int cb = 0; cb < nch; cb++)
+                mma_ts_elect(T.d, T.a1 + 8 * cb, d1base + (uint64_t)((nch + cb) * (kChunkBytesN32 >> 4)), id32, 1u);
+        mma_commit_elect(bar);
+    };
+    // epilogue: ReLU + pack into A (= U[0,16)); the first hidden layer also
+    // (re)writes the constant chunk U[16,24) over the consumed layer-1 operand
+    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id, bool me,
+                     uint32_t idesc, bool write_const) {
+        mbar_wait(bar, ph);
+        ph ^= 1u;
+        fence_after();
+        {
+            uint32_t rr[32];
+            tmem_ld32(T.d + lane_off, rr);
+            uint32_t h[16];
+#pragma unroll
+            for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(rr[2 * c], rr[2 * c + 1]);
+            tmem_st16(T.a + lane_off, h);
+            if (write_const) {
+                uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
+                tmem_st8(T.a + 16 + lane_off, c8);
+            }
+            tmem_wait_st();
+        }
+        if (handoff(bar_id, me)) {
+            issue_layer_e<FMT>(T.d, T.a, T.a + 16, dl, idesc);
+            mma_commit_elect(bar);
+        }
+    };
+    // feature rows of tile w: TMA bulk copy into the slot's stage (one elected thread)
+    auto fetch = [&](uint64_t w, uint8_t* st, uint64_t* tb) {
+        if (!tma_ok || w >= (count + kTileM - 1) / kTileM) return;
+        if (lane == 0) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of `st`
+            const uint64_t row0 = w * kTileM;
+            const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
+            mbar_arrive_expect_tx(tb, nrows * row_bytes);
+            bulk_g2s(st, x + row0 * (uint64_t)D, nrows * row_bytes, tb);
+        }
+    };
+    // layer-1 operand row from the staged features: [x_hi (D), x_lo (D), 1, 1, 0...]
+    auto encode = [&](const TileIO& T, uint64_t w, uint8_t* st, uint64_t* tb, uint32_t& tph) {
         const uint64_t row0 = w * kTileM;
         const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
-        // stage the tile's rows (contiguous bytes) with 16-byte loads
-        {
-            const uint32_t nbytes = nrows * (uint32_t)D * 2u;
-            const char* src = reinterpret_cast<const char*>(x + row0 * (uint64_t)D);
-            if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
-                for (uint32_t i = r; i < nbytes / 16; i += 128)
-                    reinterpret_cast<int4*>(stage)[i] = __ldg(reinterpret_cast<const int4*>(src) + i);
-                for (uint32_t i = (nbytes / 16) * 16 + r; i < nbytes; i += 128)
-                    reinterpret_cast<char*>(stage)[i] = src[i];
-            } else {
-                for (uint32_t i = r; i < nbytes / 2; i += 128) stage[i] = x[row0 * (uint64_t)D + i];
-            }
+        const int16_t* rowp;
+        if (tma_ok) {
+            mbar_wait(tb, tph);
+            tph ^= 1u;
+            rowp = reinterpret_cast<const int16_t*>(st) + (size_t)min(r, nrows - 1) * D;
+        } else {
+            rowp = x + (row0 + min(r, nrows - 1)) * (uint64_t)D;
         }
-        named_bar_sync(1 + g, 128);
-        // A1 row from the staged features
-        const int16_t* row = stage + (size_t)min(r, nrows - 1) * D;
         for (int cb = 0; cb < nch; cb++) {
             uint32_t a[8];
 #pragma unroll
@@ -598,67 +671,85 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
                 for (int h = 0; h < 2; h++) {
                     const int k = cb * 16 + 2 * i + h;
                     float val = 0.0f;
-                    if (k < D) val = (float)(row[k] >> 8);
-                    else if (k < 2 * D) val = (float)(row[k - D] & 255);
+                    if (k < D) val = (float)(rowp[k] >> 8);
+                    else if (k < 2 * D) val = (float)(rowp[k - D] & 255);
                     else if (k < 2 * D + 2) val = 1.0f;
                     v2[h] = val;
                 }
                 a[i] = pack2<FMT>(v2[0], v2[1]);
             }
-            tmem_st8(tA1 + lane_off + 8 * cb, a);
+            tmem_st8(T.a1 + lane_off + 8 * cb, a);
         }
         tmem_wait_st();
-        fence_before();
-        named_bar_sync(1 + g, 128);  // also: every thread done reading `stage`
-        if (leader) {
-            fence_after();
-            for (int cb = 0; cb < nch; cb++)
-                mma_ts(tD, tA1 + 8 * cb, smem_desc(b1a + cb * kChunkBytesN32), id32, cb > 0 ? 1u : 0u);
-            if (FMT == 1)
-                for (int cb = 0; cb < nch; cb++)
-                    mma_ts(tD, tA1 + 8 * cb, smem_desc(b1a + (nch + cb) * kChunkBytesN32), id32, 1u);
-            mma_commit(bar);
+    };
+
+    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    uint64_t wb, we;
+    work_range(n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
+    if (wb < we) {
+        bool xLive = true, yLive = wb + 1 < we;
+        if (r == 0) {
+            fetch(wb, stX, tbX);
+            if (yLive) fetch(wb + 1, stY, tbY);
         }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            issue_layer<FMT>(tD, tA, tC, w2a, kChunkBytesN32, id32);
-            mma_commit(bar);
+        // the issuing warp waits for all 128 threads (rows of the stage consumed),
+        // then refills the stage with the slot's next tile
+        encode(X, wb, stX, tbX, tphX);
+        if (handoff(idX, meX[3])) {
+            issue_l1(X, barX);
+            fetch(wb + 2 < we ? wb + 2 : ~0ull, stX, tbX);
         }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
-            fence_after();
-            issue_layer<FMT>(tD, tA, tC, w3a, kChunkBytesN32, id32);
-            mma_commit(bar);
+        if (yLive) {
+            encode(Y, wb + 1, stY, tbY, tphY);
+            if (handoff(idY, meY[3])) {
+                issue_l1(Y, barY);
+                fetch(wb + 3 < we ? wb + 3 : ~0ull, stY, tbY);
+            }
         }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        hidden_epilogue<FMT>(tD + lane_off, tA + lane_off);
-        fence_before();
-        named_bar_sync(1 + g, 128);
-        if (leader) {
+        for (uint64_t w = wb; xLive; w += 2) {
+            stage(X, barX, phX, d2, idX, meX[0], id32, true);
+            if (yLive) stage(Y, barY, phY, d2, idY, meY[0], id32, true);
+            stage(X, barX, phX, d3, idX, meX[1], id32, false);
+            if (yLive) stage(Y, barY, phY, d3, idY, meY[1], id32, false);
+            stage(X, barX, phX, d4, idX, meX[2], id16, false);
+            if (yLive) stage(Y, barY, phY, d4, idY, meY[2], id16, false);
+            mbar_wait(barX, phX);
+            phX ^= 1u;
             fence_after();
-            issue_layer<FMT>(tD, tA, tC, w4a, kChunkBytesN16, id16);
-            mma_commit(bar);
+            {
+                uint32_t yb;
+                tmem_ld1(X.d + lane_off, yb);
+                const uint64_t row = w * kTileM + r;
+                if (row < count) y[row] = __uint_as_float(yb);
+            }
+            xLive = w + 2 < we;
+            if (xLive) {
+                encode(X, w + 2, stX, tbX, tphX);
+                if (handoff(idX, meX[3])) {
+                    issue_l1(X, barX);
+                    fetch(w + 4 < we ? w + 4 : ~0ull, stX, tbX);
+                }
+            }
+            if (yLive) {
+                mbar_wait(barY, phY);
+                phY ^= 1u;
+                fence_after();
+                {
+                    uint32_t yb;
+                    tmem_ld1(Y.d + lane_off, yb);
+                    const uint64_t row = (w + 1) * kTileM + r;
+                    if (row < count) y[row] = __uint_as_float(yb);
+                }
+                yLive = w + 3 < we;
+                if (yLive) {
+                    encode(Y, w + 3, stY, tbY, tphY);
+                    if (handoff(idY, meY[3])) {
+                        issue_l1(Y, barY);
+                        fetch(w + 5 < we ? w + 5 : ~0ull, stY, tbY);
+                    }
+                }
+            }
         }
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        uint32_t ybits;
-        tmem_ld1(tD + lane_off, ybits);
-        if (r < nrows) y[row0 + r] = __uint_as_float(ybits);
-        fence_before();
     }
     fence_before();
     __syncthreads();
@@ -712,23 +803,24 @@ template <int FMT>
 static cudaError_t launch_predict_fmt(const TcParams& tp, const float* w1b1, int32_t D, const int16_t* x,
                                       uint64_t count, float* y, int nsm, cudaStream_t st) {
     const int nch = (2 * D + 2 + 15) / 16;
-    const uint32_t stage_bytes = (uint32_t)(kTileM * D * 2 + 15) & ~15u;
-    const TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, kPredictNG, stage_bytes);
+    const uint32_t stage_bytes = (uint32_t)(kTileM * D * 2 + 127) & ~127u;
+    TcSmem L = tc_smem_layout<FMT>(FMT == 0 ? nch : 2 * nch, kChunkBytesN32, 2 * kPredictNG, stage_bytes);
+    const uint32_t total = L.total + 16 + 8 * 2 * kPredictNG;  // + TMA mbarriers after the TMEM slot
     auto kern = predict_tc_kernel<FMT, kPredictNG>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)total);
     if (e != cudaSuccess) return e;
     const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
     uint64_t g = (n_tiles + kPredictNG - 1) / kPredictNG;
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
-    kern<<<(int)g, kPredictNG * 128, L.total, st>>>(tp, w1b1, D, x, count, y);
+    kern<<<(int)g, kPredictNG * 128, total, st>>>(tp, w1b1, D, x, count, y);
     return cudaGetLastError();
 }
 
 cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
                               float* y, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
-    if (D > 40) return cudaErrorInvalidValue;  // A1 slice (8 nch <= 48 columns) of a 128-column group
+    if (D > 31) return cudaErrorInvalidValue;  // layer-1 operand: 4 K-chunks = the 32-column U region
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
     if (TW.fmt == 0) return launch_predict_fmt<0>(tp, w1b1, D, x, count, y, nsm, st);
     return launch_predict_fmt<1>(tp, w1b1, D, x, count, y, nsm, st);
