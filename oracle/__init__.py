@@ -63,6 +63,13 @@ class Decision(C.Structure):
                 ("pred_critical_only_ms", C.c_double), ("h", C.c_double * 4)]
 
 
+class MWay(C.Structure):
+    _fields_ = [("status", C.c_int32), ("rounds", C.c_int32), ("predictions", C.c_int32),
+                ("total_ops", C.c_int32), ("u", C.c_uint64), ("headroom_ms", C.c_double),
+                ("pred_ms", C.c_double), ("pred_critical_only_ms", C.c_double), ("end_op", C.c_int32 * 4),
+                ("order", C.c_int32 * 4)]
+
+
 _lib = None
 
 
@@ -105,6 +112,9 @@ def lib():
         L.orc_search.argtypes = [C.c_int32, C.c_int32, P(C.c_int32), P(C.c_float), P(QueryC),
                                  C.c_int32, C.c_double, C.c_double, C.c_int32, C.c_uint64,
                                  C.c_double, C.c_int32, P(Decision)]
+        L.orc_search_mway.restype = C.c_int32
+        L.orc_search_mway.argtypes = [C.c_int32, C.c_int32, P(C.c_int32), P(C.c_float), P(QueryC), C.c_int32,
+                                      C.c_double, C.c_double, C.c_int32, C.c_int32, P(MWay)]
     return _lib
 
 
@@ -243,6 +253,24 @@ def search(params, queries, now, inflight, space=0, budget=2**40, eps=1e-4, n_mo
                           float(now), float(inflight), space, budget, eps, emu_flags, C.byref(out))
     if rc != 0:
         raise ValueError("orc_search rejected the queries (rc=%d)" % rc)
+    return out
+
+
+def search_mway(params, queries, now, inflight, ways, n_models=8, kmax=4, ops_per_model=None, emu_flags=0):
+    """The paper's multi-way search over the chain (rounds of batched probes)."""
+    if ops_per_model is None:
+        import synth
+        ops_per_model = synth.OPS_PER_MODEL
+    opm = np.ascontiguousarray(ops_per_model, dtype=np.int32)
+    k = len(queries)
+    qa = (QueryC * k)(*[QueryC(q.model_id, q.next_op, q.batch, q.seqlen, q.qos_ms, q.t_start_ms)
+                        for q in queries])
+    p, pp = _f32(params)
+    out = MWay()
+    rc = lib().orc_search_mway(n_models, kmax, opm.ctypes.data_as(C.POINTER(C.c_int32)), pp, qa, k,
+                               float(now), float(inflight), int(ways), emu_flags, C.byref(out))
+    if rc != 0:
+        raise ValueError("orc_search_mway rejected the queries (rc=%d)" % rc)
     return out
 
 

@@ -527,3 +527,152 @@ int32_t orc_search(int32_t n_models, int32_t kmax, const int32_t* ops_per_model,
     for (int32_t j = 0; j < k; j++) out->end_op[order[j]] = ope_best[j];
     return 0;
 }
+
+/* -------------------------------------------------------------------------- */
+/* Multi-way search over the CHAIN (§7.7) */
+/* Round 1 ("between queries"): one batched call predicts u = 0 (drop test)    */
+/* and every block end B_j (queries 1..j fully added); the last fitting block   */
+/* end is lo, the first missing one after it is hi.  Later rounds ("among the   */
+/* operators"): the open interval (lo, hi) of the next query's ops is probed    */
+/* at m points p_i = lo + floor(i (hi - lo) / (m + 1)), i = 1..m (all points    */
+/* when it holds <= m); lo <- last fitting probe, hi <- first missing probe     */
+/* after it (reading c17).  Ends when the interval is empty.  Returns u* = lo.  */
+/* -------------------------------------------------------------------------- */
+typedef struct {
+    int32_t status;      /* 0 OK, 1 DROP */
+    int32_t rounds;      /* batched predictor calls */
+    int32_t predictions; /* candidates predicted */
+    int32_t total_ops;
+    uint64_t u;          /* chosen chain index */
+    double headroom_ms, pred_ms, pred_critical_only_ms;
+    int32_t end_op[4];   /* per caller query */
+    int32_t order[4];
+} orc_mway_t;
+
+static double orc_chain_y(int32_t n_models, int32_t kmax, const float* prm, int32_t emu, int32_t k,
+                          const orc_gslot_t* g, const uint64_t* cum, uint64_t u, int32_t* ope_out,
+                          int32_t* sum_n_out) {
+    orc_present_t pres[ORC_KMAX];
+    int16_t x[64];
+    int32_t ope[ORC_KMAX], n = 0, sum_n = 0, blk = 0;
+    for (int32_t j = 1; j < k; j++)
+        if (u >= cum[j]) blk = j;
+    for (int32_t i = 0; i < k; i++) {
+        if (i < blk) ope[i] = g[i].end_hi;
+        else if (i == blk) ope[i] = blk == 0 ? g[0].end_hi : g[i].start_op + (int32_t)(u - cum[i]);
+        else ope[i] = 0;
+    }
+    for (int32_t i = 0; i < k; i++) {
+        if (ope[i] == 0) continue;
+        pres[n].model_id = g[i].model_id;
+        pres[n].ops = g[i].start_op;
+        pres[n].ope = ope[i];
+        pres[n].bs = g[i].batch;
+        pres[n].seqlen = g[i].seqlen;
+        sum_n += ope[i] - g[i].start_op + 1;
+        n++;
+    }
+    orc_encode(n_models, kmax, n, pres, x);
+    if (ope_out)
+        for (int32_t i = 0; i < k; i++) ope_out[i] = ope[i];
+    if (sum_n_out) *sum_n_out = sum_n;
+    return emu ? orc_mlp64_emu(prm, n_models + 4 * kmax, x, emu) : orc_mlp64(prm, n_models + 4 * kmax, x);
+}
+
+int32_t orc_search_mway(int32_t n_models, int32_t kmax, const int32_t* ops_per_model, const float* prm,
+                        const orc_query_t* q, int32_t k, double now_ms, double inflight_ms, int32_t ways,
+                        int32_t emu_flags, orc_mway_t* out) {
+    double h[ORC_KMAX];
+    int32_t mid[ORC_KMAX], order[ORC_KMAX];
+    orc_gslot_t g[ORC_KMAX];
+    uint64_t cum[ORC_KMAX + 1];
+    if (k < 1 || k > kmax || k > 4 || ways < 1 || ways > 128) return -1;
+    memset(out, 0, sizeof(*out));
+    for (int32_t i = 0; i < k; i++) {
+        if (q[i].model_id < 1 || q[i].model_id > n_models) return -1;
+        for (int32_t j = 0; j < i; j++)
+            if (q[j].model_id == q[i].model_id) return -2;
+        h[i] = orc_headroom(q[i].qos_ms, q[i].t_start_ms, now_ms, inflight_ms);
+        mid[i] = q[i].model_id;
+    }
+    orc_order(k, h, mid, order);
+    for (int32_t j = 0; j < k; j++) out->order[j] = order[j];
+    double H = (double)(float)h[order[0]];
+    out->headroom_ms = H;
+    for (int32_t j = 0; j < k; j++) {
+        const orc_query_t* qq = &q[order[j]];
+        int32_t Lm = ops_per_model[qq->model_id - 1];
+        g[j].model_id = qq->model_id;
+        g[j].start_op = qq->next_op;
+        g[j].batch = qq->batch;
+        g[j].seqlen = qq->seqlen;
+        g[j].end_hi = Lm;
+        g[j].end_lo = j == 0 ? Lm : qq->next_op;
+        g[j].allow_absent = j == 0 ? 0 : 1;
+    }
+    /* chain blocks: u = 0 critical; block j covers [cum[j], cum[j] + R_j) */
+    cum[0] = 0;
+    cum[1] = 1;
+    for (int32_t j = 1; j < k; j++) cum[j + 1] = cum[j] + (uint64_t)(g[j].end_hi - g[j].start_op + 1);
+    /* round 1: u = 0 and the block ends */
+    uint64_t probes[ORC_KMAX + 1];
+    int32_t np = 0;
+    probes[np++] = 0;
+    for (int32_t j = 1; j < k; j++) probes[np++] = cum[j + 1] - 1;
+    uint64_t lo = 0, hi = cum[k];
+    out->rounds = 1;
+    int32_t fit[ORC_KMAX + 1];
+    for (int32_t i = 0; i < np; i++) {
+        double y = orc_chain_y(n_models, kmax, prm, emu_flags, k, g, cum, probes[i], NULL, NULL);
+        out->predictions++;
+        fit[i] = y <= H;
+        if (i == 0) out->pred_critical_only_ms = y;
+    }
+    if (!fit[0]) {
+        out->status = 1;
+        out->pred_ms = out->pred_critical_only_ms;
+        return 0;
+    }
+    int32_t last = 0;
+    for (int32_t i = 1; i < np; i++)
+        if (fit[i]) last = i;
+    lo = probes[last];
+    hi = cum[k];
+    for (int32_t i = last + 1; i < np; i++)
+        if (!fit[i]) { hi = probes[i]; break; }
+    /* later rounds: m-way among the operators of the next query */
+    while (hi - lo > 1) {
+        uint64_t p[128];
+        int32_t n = 0;
+        uint64_t span = hi - lo;
+        if (span - 1 <= (uint64_t)ways) {
+            for (uint64_t v = lo + 1; v < hi; v++) p[n++] = v;
+        } else {
+            for (int32_t i = 1; i <= ways; i++) {
+                uint64_t v = lo + (span * (uint64_t)i) / (uint64_t)(ways + 1);
+                if (v > lo && v < hi && (n == 0 || v > p[n - 1])) p[n++] = v;
+            }
+        }
+        out->rounds++;
+        int32_t f[128];
+        for (int32_t i = 0; i < n; i++) {
+            f[i] = orc_chain_y(n_models, kmax, prm, emu_flags, k, g, cum, p[i], NULL, NULL) <= H;
+            out->predictions++;
+        }
+        int32_t lf = -1;
+        for (int32_t i = 0; i < n; i++)
+            if (f[i]) lf = i;
+        uint64_t nlo = lf >= 0 ? p[lf] : lo, nhi = hi;
+        for (int32_t i = lf + 1; i < n; i++)
+            if (!f[i]) { nhi = p[i]; break; }
+        lo = nlo;
+        hi = nhi;
+    }
+    int32_t ope[ORC_KMAX], sum_n = 0;
+    out->u = lo;
+    out->pred_ms = orc_chain_y(n_models, kmax, prm, emu_flags, k, g, cum, lo, ope, &sum_n);
+    out->total_ops = sum_n;
+    out->status = 0;
+    for (int32_t j = 0; j < k; j++) out->end_op[order[j]] = ope[j];
+    return 0;
+}

@@ -300,3 +300,38 @@ def test_search_invariants():
         a1 = oracle.search(p, qs, now, infl, space=2, budget=T)
         a2 = oracle.search(p, qs, now, infl, space=2, budget=T - 1)
         assert a1.space_used == 0 and a2.space_used == 1
+
+
+# ------------------------------------------------------- multi-way search ---
+def test_fig12_multiway_two_predictions():
+    """P:1349-1355: 3-way search -- first between queries, then among q1's ops;
+    'After two predictions, the query controller completes the exploration'."""
+    f, p, qs = _fig12_setup()
+    m = oracle.search_mway(p, qs, 0.0, 0.0, ways=3, n_models=3, kmax=3, ops_per_model=f["ops_per_model"])
+    names = [q["name"] for q in f["queries"]]
+    assert m.status == 0 and m.rounds == 2
+    assert m.u == f["expected"]["chain_u"] and m.pred_ms == 25.0
+    assert {names[i]: m.end_op[i] for i in range(3)} == f["expected"]["end_op"]
+
+
+def test_multiway_equals_exhaustive_chain_under_monotone_predictor():
+    """With a predictor monotone along the chain (non-negative linear, ReLU-
+    transparent), the m-way search finds the exhaustive CHAIN optimum for every
+    m, in about log_{m+1} steps."""
+    rng = np.random.default_rng(21)
+    for trial in range(40):
+        lp = LinearPredictor(8, 4, c0=2.0, beta=[float(rng.integers(0, 16)) / 4 for _ in range(8)],
+                             a=[float(rng.integers(1, 8)) / 8 for _ in range(4)])
+        p = lp.params()
+        k = int(rng.integers(1, 5))
+        ms = rng.choice(np.arange(1, 9), size=k, replace=False)
+        qs = [synth.Query(int(m), int(rng.integers(1, synth.L(int(m)) + 1)), 8, 0,
+                          float(rng.uniform(5, 200)), 0.0) for m in ms]
+        ex = oracle.search(p, qs, 0.0, 0.0, space=1)
+        for ways in (1, 2, 3, 4, 8, 15):
+            mw = oracle.search_mway(p, qs, 0.0, 0.0, ways)
+            assert mw.status == ex.status
+            if ex.status == 0:
+                assert mw.u == ex.index and list(mw.end_op)[:k] == list(ex.end_op)[:k]
+                R = max(1, ex.evaluated)
+                assert mw.rounds <= 2 + int(np.ceil(np.log(R) / np.log(ways + 1)))
