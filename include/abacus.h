@@ -215,6 +215,19 @@ int abacus_select_group(abacus_ctx* ctx, const abacus_grid_t* grid, uint64_t fir
 int abacus_search(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
                   int32_t space, uint64_t grid_budget, abacus_decision_t* out);
 
+/* The paper's multi-way search (§7.7)
+ * for one scheduling round: same a1 step as abacus_search; candidates are the
+ * CHAIN.  Round 1 is one batched prediction of u = 0 (drop test) and of every
+ * block end (queries fully added, "between queries"); each later round
+ * predicts `ways` evenly spaced points of the open interval (last fit, first
+ * miss) inside the next query's operators (reading c17).  The result is the
+ * last fitting chain position; it equals the exhaustive CHAIN result whenever
+ * the prediction is monotone along the chain.  Predictions use the fp32
+ * arithmetic.  out->evaluated = candidates predicted; *rounds_out (may be
+ * NULL) = batched rounds.  1 <= ways <= 128.  Errors as abacus_search. */
+int abacus_search_mway(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                       int32_t ways, abacus_decision_t* out, int32_t* rounds_out);
+
 /* a2..a6 over a sweep grid: candidates t in [first, first+count) of `grid`
  * (host) under `headroom_ms`; this rank's shard.  With nccl_comm != NULL
  * (an ncclComm_t on this device, e.g. from abacus_nccl_comm_init) the

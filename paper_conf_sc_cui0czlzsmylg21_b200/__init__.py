@@ -27,7 +27,7 @@ K_MAX = 4
 
 EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load_predictor",
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
-            "abacus_select_group", "abacus_search", "abacus_search_grid", "abacus_nccl_unique_id",
+            "abacus_select_group", "abacus_search", "abacus_search_mway", "abacus_search_grid", "abacus_nccl_unique_id",
             "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
             "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version"]
 
@@ -94,6 +94,8 @@ def lib():
         L.abacus_select_group.argtypes = [vp, P(abacus_grid_t), C.c_uint64, C.c_uint64, vp, C.c_float, vp, vp]
         L.abacus_search.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
                                     C.c_uint64, P(abacus_decision_t)]
+        L.abacus_search_mway.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
+                                         P(abacus_decision_t), P(C.c_int32)]
         L.abacus_search_grid.argtypes = [vp, P(abacus_grid_t), C.c_float, C.c_uint64, C.c_uint64, vp,
                                          P(abacus_decision_t)]
         L.abacus_nccl_unique_id.argtypes = [P(C.c_uint8)]
@@ -204,6 +206,18 @@ def abacus_search(ctx, queries, now_ms: float, inflight_pred_ms: float, space: i
     _check(ctx, lib().abacus_search(ctx, qa, k, float(now_ms), float(inflight_pred_ms), space, grid_budget,
                                     C.byref(out)))
     return out
+
+
+def abacus_search_mway(ctx, queries, now_ms: float, inflight_pred_ms: float, ways: int):
+    """Returns (decision, rounds)."""
+    k = len(queries)
+    qa = (abacus_query_t * k)(*[abacus_query_t(q.model_id, q.next_op, q.batch, q.seqlen, q.qos_ms,
+                                               q.t_start_ms) for q in queries])
+    out = abacus_decision_t()
+    rounds = C.c_int32()
+    _check(ctx, lib().abacus_search_mway(ctx, qa, k, float(now_ms), float(inflight_pred_ms), int(ways),
+                                         C.byref(out), C.byref(rounds)))
+    return out, int(rounds.value)
 
 
 def abacus_search_grid(ctx, grid: abacus_grid_t, headroom_ms: float, first: int, count: int,

@@ -530,6 +530,49 @@ int wait_result(abacus_ctx* c, uint32_t seq) {
     return ABACUS_OK;
 }
 
+// a1 (Eq. 2 + Eq. 3, sort) and the decision's slots in headroom order
+int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                   int32_t* order, float* H_out, abacus_grid_t* g_out) {
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (!q) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (k < 1 || k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
+    if (!std::isfinite(now_ms) || !std::isfinite(inflight_pred_ms))
+        return fail(c, ABACUS_E_INVALID, "non-finite time");
+    // a1: Eq. 2 + Eq. 3 headroom per query; ascending order, ties by model id
+    double h[ABACUS_K_MAX];
+    for (int i = 0; i < k; i++) {
+        const abacus_query_t& a = q[i];
+        if (a.model_id < 1 || a.model_id > c->n_models)
+            return fail(c, ABACUS_E_INVALID, "query %d: model_id %d", i, a.model_id);
+        for (int j = 0; j < i; j++)
+            if (q[j].model_id == a.model_id) return fail(c, ABACUS_E_DUP_MODEL, "queries %d, %d share a model", j, i);
+        const int32_t L = c->L[a.model_id - 1];
+        if (a.next_op < 1 || a.next_op > L) return fail(c, ABACUS_E_INVALID, "query %d: next_op %d", i, a.next_op);
+        if (a.batch < 1 || a.batch > 32767 || a.seqlen < 0 || a.seqlen > 32767)
+            return fail(c, ABACUS_E_INVALID, "query %d: batch/seqlen", i);
+        if (!std::isfinite(a.qos_ms) || !std::isfinite(a.t_start_ms))
+            return fail(c, ABACUS_E_INVALID, "query %d: non-finite time", i);
+        h[i] = (a.qos_ms - (now_ms - a.t_start_ms)) - inflight_pred_ms;
+        order[i] = i;
+    }
+    std::stable_sort(order, order + k, [&](int a, int b) {
+        if (h[a] != h[b]) return h[a] < h[b];
+        return q[a].model_id < q[b].model_id;
+    });
+    *H_out = (float)h[order[0]];
+    // a2: slots in headroom order; the critical query is fully included
+    abacus_grid_t& g = *g_out;
+    g = abacus_grid_t{};
+    g.k = k;
+    for (int j = 0; j < k; j++) {
+        const abacus_query_t& a = q[order[j]];
+        const int32_t L = c->L[a.model_id - 1];
+        g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? L : a.next_op, L, j == 0 ? 0 : 1};
+    }
+    uint64_t T = 0;
+    return validate_grid(c, &g, &T);
+}
+
 unsigned long long* trace_ptr();
 
 int launch_fused(abacus_ctx* c, const Plan& Pin) {
@@ -748,45 +791,15 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
                   int32_t space, uint64_t grid_budget, abacus_decision_t* out) {
     if (!c) return ABACUS_E_INVALID;
     c->err.clear();
-    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
-    if (!q || !out) return fail(c, ABACUS_E_INVALID, "NULL argument");
-    if (k < 1 || k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
+    if (!out) return fail(c, ABACUS_E_INVALID, "NULL argument");
     if (space < ABACUS_SPACE_GRID || space > ABACUS_SPACE_AUTO) return fail(c, ABACUS_E_INVALID, "bad space");
-    if (!std::isfinite(now_ms) || !std::isfinite(inflight_pred_ms))
-        return fail(c, ABACUS_E_INVALID, "non-finite time");
-    // a1: Eq. 2 + Eq. 3 headroom per query; ascending order, ties by model id
-    double h[ABACUS_K_MAX];
     int32_t order[ABACUS_K_MAX];
-    for (int i = 0; i < k; i++) {
-        const abacus_query_t& a = q[i];
-        if (a.model_id < 1 || a.model_id > c->n_models)
-            return fail(c, ABACUS_E_INVALID, "query %d: model_id %d", i, a.model_id);
-        for (int j = 0; j < i; j++)
-            if (q[j].model_id == a.model_id) return fail(c, ABACUS_E_DUP_MODEL, "queries %d, %d share a model", j, i);
-        const int32_t L = c->L[a.model_id - 1];
-        if (a.next_op < 1 || a.next_op > L) return fail(c, ABACUS_E_INVALID, "query %d: next_op %d", i, a.next_op);
-        if (a.batch < 1 || a.batch > 32767 || a.seqlen < 0 || a.seqlen > 32767)
-            return fail(c, ABACUS_E_INVALID, "query %d: batch/seqlen", i);
-        if (!std::isfinite(a.qos_ms) || !std::isfinite(a.t_start_ms))
-            return fail(c, ABACUS_E_INVALID, "query %d: non-finite time", i);
-        h[i] = (a.qos_ms - (now_ms - a.t_start_ms)) - inflight_pred_ms;
-        order[i] = i;
-    }
-    std::stable_sort(order, order + k, [&](int a, int b) {
-        if (h[a] != h[b]) return h[a] < h[b];
-        return q[a].model_id < q[b].model_id;
-    });
-    const float H = (float)h[order[0]];
-    // a2: slots in headroom order; the critical query is fully included
+    float H = 0.0f;
     abacus_grid_t g{};
-    g.k = k;
-    for (int j = 0; j < k; j++) {
-        const abacus_query_t& a = q[order[j]];
-        const int32_t L = c->L[a.model_id - 1];
-        g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? L : a.next_op, L, j == 0 ? 0 : 1};
-    }
+    int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g);
+    if (rc) return rc;
     uint64_t T = 0;
-    int rc = validate_grid(c, &g, &T);
+    rc = validate_grid(c, &g, &T);
     if (rc) return rc;
     const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
     Plan P;
@@ -825,6 +838,45 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
         d.total_ops = R.total_ops;
         for (int j = 0; j < k; j++) d.end_op[order[j]] = R.end_op[j];
     }
+    *out = d;
+    return ABACUS_OK;
+}
+
+int abacus_search_mway(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                       int32_t ways, abacus_decision_t* out, int32_t* rounds_out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!out) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (ways < 1 || ways > 128) return fail(c, ABACUS_E_INVALID, "ways=%d outside [1,128]", ways);
+    int32_t order[ABACUS_K_MAX];
+    float H = 0.0f;
+    abacus_grid_t g{};
+    int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g);
+    if (rc) return rc;
+    uint64_t n_chain = 0;
+    Plan P = plan_chain(c, &g, H, &n_chain);
+    P.mapped = c->dev_result;
+    P.seq = next_seq(c);
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    CUDA_TRY(c, launch_mway(P, c->w234, c->d_w1b1, ways, c->S, c->stream));
+    c->launches++;
+    rc = wait_result(c, P.seq);
+    if (rc) return rc;
+    const Result R = *c->host_result;
+    abacus_decision_t d{};
+    d.critical = order[0];
+    for (int j = 0; j < 4; j++) d.order[j] = j < k ? order[j] : -1;
+    d.headroom_ms = H;
+    d.pred_critical_only_ms = R.y0;
+    d.pred_ms = R.y_best;
+    d.evaluated = R.evaluated;
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    d.status = R.status;
+    d.total_ops = R.total_ops;
+    if (R.status == ABACUS_DECIDE_OK)
+        for (int j = 0; j < k; j++) d.end_op[order[j]] = R.end_op[j];
+    if (rounds_out) *rounds_out = (int32_t)R.pad;
     *out = d;
     return ABACUS_OK;
 }

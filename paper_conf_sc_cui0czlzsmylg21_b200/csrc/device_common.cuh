@@ -194,6 +194,7 @@ __device__ __forceinline__ void publish_mapped(const Result& R, Result* M, uint3
     for (int j = 0; j < kKMax; j++) m->end_op[j] = R.end_op[j];
     m->total_ops = R.total_ops;
     m->status = R.status;
+    m->pad = R.pad;
     // release at system scope: the record is visible before the tag
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(&M->seq), "r"(seq) : "memory");
 }

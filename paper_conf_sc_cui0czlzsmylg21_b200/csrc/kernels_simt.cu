@@ -319,6 +319,173 @@ __global__ void finalize_gather_kernel(Scratch* S, int nranks, Result* mapped, u
     if (mapped) publish_mapped(S->result, mapped, seq);
 }
 
+
+// ---------------------------------------------------------------------------
+// NEXT-1: the paper's multi-way search (§7.7) in one
+// CTA.  Round 1 predicts u = 0 (drop test) and the chain's block ends (queries
+// fully added, "between queries"); later rounds probe the open interval
+// (last fit, first miss) of the next query's operators at `ways` points
+// p_i = lo + floor(i (hi - lo) / (ways + 1)) ("among the operators").  Each
+// round is one batched prediction: thread i evaluates probe i with the fp32
+// predictor (layer 1 from shared memory, layers 2-4 from the constant bank).
+// ---------------------------------------------------------------------------
+constexpr int kMwayThreads = 128;
+
+__device__ float chain_candidate_y(const Plan& P, const W234& Wt, const float* s_w1, uint64_t u, int32_t& sum_n) {
+    int32_t ope[kKMax];
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) ope[j] = j < P.k ? decode_slot_ope(P, u, j) : 0;
+    sum_n = 0;
+    float h1[kHidden];
+    const float* b1 = s_w1 + kHidden * P.D;
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) h1[i] = b1[i];
+    // Fig. 8 features applied straight to layer 1: x has at most
+    // 5 non-zeros per present model
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) {
+        if (j >= P.k || ope[j] == 0) continue;
+        int p = 0;
+#pragma unroll
+        for (int i = 0; i < kKMax; i++)
+            if (i < P.k && ope[i] != 0 && P.slot[i].model_id < P.slot[j].model_id) p++;
+        const SlotP& s = P.slot[j];
+        sum_n += ope[j] - s.ops + 1;
+        const int f = P.n_models + 4 * p;
+        const float xo = (float)s.ops, xe = (float)ope[j], xb = (float)s.bs, xs = (float)s.seqlen;
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) {
+            const float* w = s_w1 + i * P.D;
+            float z = h1[i] + w[s.model_id - 1];
+            z = fmaf(w[f + 0], xo, z);
+            z = fmaf(w[f + 1], xe, z);
+            z = fmaf(w[f + 2], xb, z);
+            h1[i] = fmaf(w[f + 3], xs, z);
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) h1[i] = fmaxf(h1[i], 0.0f);
+    float y;
+    mlp_tail_fp32(Wt, h1, y);
+    return y;
+}
+
+__global__ void __launch_bounds__(kMwayThreads, 1) mway_kernel(const __grid_constant__ Plan P,
+                                                                const __grid_constant__ W234 Wt,
+                                                                const float* __restrict__ w1b1, int ways,
+                                                                Scratch* S) {
+    extern __shared__ float s_w1[];  // W1[32][D] | b1[32]
+    __shared__ uint64_t s_probe[kMwayThreads];
+    __shared__ float s_y[kMwayThreads];
+    __shared__ int s_n, s_done, s_rounds, s_preds;
+    __shared__ uint64_t s_lo, s_hi;
+    __shared__ float s_ylo, s_y0;
+    for (int i = threadIdx.x; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = w1b1[i];
+    if (threadIdx.x == 0) {
+        // round 1: u = 0 and the block ends B_j = chain_cum[j + 1] - 1
+        int n = 0;
+        s_probe[n++] = 0;
+        for (int j = 1; j < P.k; j++) s_probe[n++] = P.chain_cum[j + 1] - 1;
+        s_n = n;
+        s_done = 0;
+        s_rounds = 0;
+        s_preds = 0;
+    }
+    __syncthreads();
+    for (int round = 0;; round++) {
+        const int n = s_n;
+        if (threadIdx.x < n) {
+            int32_t sn;
+            s_y[threadIdx.x] = chain_candidate_y(P, Wt, s_w1, s_probe[threadIdx.x], sn);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            s_rounds++;
+            s_preds += n;
+            uint64_t lo, hi;
+            int lf = -1;
+            if (round == 0) {
+                s_y0 = s_y[0];
+                if (!(s_y[0] <= P.H)) {  // drop mechanism
+                    s_done = 2;
+                } else {
+                    lf = 0;
+                    for (int i = 1; i < n; i++)
+                        if (s_y[i] <= P.H) lf = i;
+                    lo = s_probe[lf];
+                    hi = P.chain_cum[P.k];
+                    s_ylo = s_y[lf];
+                }
+            } else {
+                lo = s_lo;
+                hi = s_hi;
+                for (int i = 0; i < n; i++)
+                    if (s_y[i] <= P.H) lf = i;
+                if (lf >= 0) {
+                    lo = s_probe[lf];
+                    s_ylo = s_y[lf];
+                }
+            }
+            if (s_done == 0) {
+                for (int i = lf + 1; i < n; i++)
+                    if (!(s_y[i] <= P.H)) {
+                        hi = s_probe[i];
+                        break;
+                    }
+                s_lo = lo;
+                s_hi = hi;
+                const uint64_t span = hi - lo;
+                if (span <= 1) {
+                    s_done = 1;
+                } else {
+                    int m = 0;
+                    if (span - 1 <= (uint64_t)ways) {
+                        for (uint64_t v = lo + 1; v < hi; v++) s_probe[m++] = v;
+                    } else {
+                        for (int i = 1; i <= ways; i++) {
+                            const uint64_t v = lo + (span * (uint64_t)i) / (uint64_t)(ways + 1);
+                            if (v > lo && v < hi && (m == 0 || v > s_probe[m - 1])) s_probe[m++] = v;
+                        }
+                    }
+                    s_n = m;
+                }
+            }
+        }
+        __syncthreads();
+        if (s_done) break;
+    }
+    if (threadIdx.x < 32) {
+        // a7: decision assembly (lane j decodes slot j)
+        const bool drop = s_done == 2;
+        const uint64_t u = drop ? 0 : s_lo;
+        const int32_t my_ope = threadIdx.x < (unsigned)P.k ? decode_slot_ope(P, u, (int)threadIdx.x) : 0;
+        int32_t ope[kKMax];
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) ope[j] = __shfl_sync(0xffffffffu, my_ope, j);
+        if (threadIdx.x == 0) {
+            int32_t sum_n = 0;
+            for (int j = 0; j < P.k; j++)
+                if (ope[j]) sum_n += ope[j] - P.slot[j].ops + 1;
+            Result& R = S->result;
+            R.key = ((unsigned long long)(sum_n + 1) << 40) | u;
+            R.y_best = drop ? s_y0 : s_ylo;
+            R.y0 = s_y0;
+            R.evaluated = (unsigned long long)s_preds;
+            for (int j = 0; j < kKMax; j++) R.end_op[j] = drop ? 0 : ope[j];
+            R.total_ops = drop ? 0 : sum_n;
+            R.status = drop ? 1 : 0;
+            R.pad = (uint32_t)s_rounds;
+            if (P.mapped) publish_mapped(R, P.mapped, P.seq);
+        }
+    }
+}
+
+cudaError_t launch_mway(const Plan& P, const W234& W, const float* w1b1, int ways, Scratch* S, cudaStream_t st) {
+    const size_t smem = (size_t)(kHidden * P.D + kHidden) * sizeof(float);
+    mway_kernel<<<1, kMwayThreads, smem, st>>>(P, W, w1b1, ways, S);
+    return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------------------
 // launchers
 // ---------------------------------------------------------------------------

@@ -332,3 +332,65 @@ def test_search_grid_nccl_single_rank(ctx):
     finally:
         ab.abacus_nccl_comm_destroy(comm)
         ctx.load(ctx.params, ab.ABACUS_FP32)
+
+
+# ------------------------------------------------------- multi-way search ---
+@pytest.mark.parametrize("ways", [1, 3, 8])
+def test_fig12_multiway_on_gpu(ways):
+    f = load_fig12()
+    p = unit0_params(f["n_models"] + 16, f["unit0"]["bias"], {int(k): v for k, v in f["unit0"]["coef"].items()})
+    c = Ctx(ops=f["ops_per_model"], params=p, precision=ab.ABACUS_FP32)
+    try:
+        qs = [synth.Query(q["model_id"], q["next_op"], 1, 0, q["headroom_ms"], 0.0) for q in f["queries"]]
+        d, rounds = ab.abacus_search_mway(c.h, qs, 0.0, 0.0, ways)
+        o = oracle.search_mway(p, qs, 0.0, 0.0, ways, n_models=3, kmax=4, ops_per_model=f["ops_per_model"])
+        names = [q["name"] for q in f["queries"]]
+        assert d.status == 0 and d.index == f["expected"]["chain_u"] == o.u
+        assert {names[i]: d.end_op[i] for i in range(3)} == f["expected"]["end_op"]
+        assert rounds == o.rounds and d.evaluated == o.predictions and d.pred_ms == 25.0
+        if ways == 3:
+            assert rounds == 2   # "After two predictions"
+    finally:
+        c.close()
+
+
+def test_multiway_gpu_matches_oracle_exactly_on_linear_predictor():
+    """Dyadic linear predictor: fp32 on the GPU is exact, so the whole search
+    path (every probe decision) must match the fp64 oracle."""
+    rng = np.random.default_rng(31)
+    lp = LinearPredictor(8, 4, c0=2.0, beta=[0.5, 1.25, 0.75, 1.0, 0.25, 0.5, 1.5, 2.0], a=[0.125, 0.25, 0.375, 0.5])
+    c = Ctx(params=lp.params(), precision=ab.ABACUS_FP32)
+    try:
+        for trial in range(60):
+            k = int(rng.integers(1, 5))
+            ms = rng.choice(np.arange(1, 9), size=k, replace=False)
+            qs = [synth.Query(int(m), int(rng.integers(1, synth.L(int(m)) + 1)), int(rng.choice([1, 8, 32])),
+                              synth.seqlen_for(int(m), int(rng.integers(8, 513))), float(rng.uniform(5, 400)),
+                              0.0) for m in ms]
+            ways = int(rng.choice([1, 2, 3, 4, 7, 15, 64]))
+            d, rounds = ab.abacus_search_mway(c.h, qs, 0.0, 0.0, ways)
+            o = oracle.search_mway(c.params, qs, 0.0, 0.0, ways)
+            assert d.status == o.status and rounds == o.rounds and d.evaluated == o.predictions
+            if o.status == 0:
+                assert d.index == o.u and list(d.end_op)[:k] == list(o.end_op)[:k]
+                assert d.pred_ms == o.pred_ms
+    finally:
+        c.close()
+
+
+def test_multiway_gpu_vs_oracle_shaped_weights(ctx):
+    agree = 0
+    decs = synth.cfg2_decisions(150)
+    for qs, now, infl in decs:
+        d, rounds = ab.abacus_search_mway(ctx.h, qs, now, infl, 4)
+        o = oracle.search_mway(ctx.params, qs, now, infl, 4)
+        if (d.status, d.index) == (o.status, o.u):
+            agree += 1
+            if o.status == 0:
+                assert abs(d.pred_ms - o.pred_ms) <= 1e-4 * o.pred_ms
+        else:
+            # a probe within the fp32 tolerance of H may flip the path; the
+            # GPU's choice must still fit in fp64 within the tolerance
+            if d.status == 0:
+                assert d.pred_ms <= d.headroom_ms * (1 + 1e-4)
+    assert agree >= 0.97 * len(decs)

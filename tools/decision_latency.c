@@ -55,7 +55,10 @@ int main(int argc, char** argv) {
     for (int i = 0; i < ndec; i++) {
         abacus_decision_t d;
         double t0 = now_us();
-        rc = abacus_search(ctx, &qs[4 * i], ks[i], nows[i], infl[i], space, budget, &d);
+        if (space == 3)  /* multi-way search, budget = ways */
+            rc = abacus_search_mway(ctx, &qs[4 * i], ks[i], nows[i], infl[i], (int32_t)budget, &d, NULL);
+        else
+            rc = abacus_search(ctx, &qs[4 * i], ks[i], nows[i], infl[i], space, budget, &d);
         double t1 = now_us();
         if (rc) { fprintf(stderr, "search failed %s\n", abacus_last_error(ctx)); return 1; }
         lat[i] = t1 - t0;

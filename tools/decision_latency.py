@@ -15,7 +15,7 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 from paper_conf_sc_cui0czlzsmylg21_b200 import _build  # noqa: E402
 
-SPACE = {"grid": 0, "chain": 1, "auto": 2}
+SPACE = {"grid": 0, "chain": 1, "auto": 2, "mway": 3}
 PREC = {"fp32": 0, "bf16": 1, "fp16": 2}
 
 
@@ -50,7 +50,8 @@ def run(config="cfg2", space="grid", precision="fp16", n=10_000, warm=100, budge
     write_input(path, decs, PREC[precision], SPACE[space], budget, warm)
     out = subprocess.check_output([exe, path]).decode()
     d = json.loads(out)
-    d.update({"config": config, "space": space, "precision": precision, "budget": budget if space == "auto" else None,
+    d.update({"config": config, "space": space, "precision": precision,
+              "budget": budget if space == "auto" else None, "ways": budget if space == "mway" else None,
               "path": "C ABI (abacus_search), host steady clock around each call"})
     return d
 
@@ -61,5 +62,6 @@ if __name__ == "__main__":
     ap.add_argument("--space", default="grid")
     ap.add_argument("--precision", default="fp16")
     ap.add_argument("-n", type=int, default=10_000)
+    ap.add_argument("--budget", type=int, default=4_194_304, help="AUTO budget, or the ways of mway")
     a = ap.parse_args()
-    print(json.dumps(run(a.config, a.space, a.precision, a.n)))
+    print(json.dumps(run(a.config, a.space, a.precision, a.n, budget=a.budget)))
