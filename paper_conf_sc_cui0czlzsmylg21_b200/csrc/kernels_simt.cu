@@ -329,19 +329,24 @@ __global__ void finalize_gather_kernel(Scratch* S, int nranks, Result* mapped, u
 // round is one batched prediction: thread i evaluates probe i with the fp32
 // predictor (layer 1 from shared memory, layers 2-4 from the constant bank).
 // ---------------------------------------------------------------------------
-constexpr int kMwayThreads = 128;
+constexpr int kMwayThreads = 512;  // 16 warps: one warp per probe, lane = hidden unit
 
-__device__ float chain_candidate_y(const Plan& P, const W234& Wt, const float* s_w1, uint64_t u, int32_t& sum_n) {
+// y of chain position u, computed by one warp (lane i = hidden unit i; the
+// activations are broadcast with shuffles; weights transposed in shared
+// memory so the lanes read consecutive words).  Returns y in every lane.
+struct MwaySmem {
+    float w1t[80 * kHidden];  // W1^T [D][32]
+    float w2t[kHidden * kHidden], w3t[kHidden * kHidden];
+    float b1[kHidden], b2[kHidden], b3[kHidden], w4[kHidden];
+    float b4;
+};
+
+__device__ float chain_candidate_y_warp(const Plan& P, const MwaySmem& W, uint64_t u, uint32_t lane) {
     int32_t ope[kKMax];
 #pragma unroll
     for (int j = 0; j < kKMax; j++) ope[j] = j < P.k ? decode_slot_ope(P, u, j) : 0;
-    sum_n = 0;
-    float h1[kHidden];
-    const float* b1 = s_w1 + kHidden * P.D;
-#pragma unroll
-    for (int i = 0; i < kHidden; i++) h1[i] = b1[i];
-    // Fig. 8 features applied straight to layer 1: x has at most
-    // 5 non-zeros per present model
+    float z = W.b1[lane];
+    // Fig. 8 features: at most 5 non-zeros per present model
 #pragma unroll
     for (int j = 0; j < kKMax; j++) {
         if (j >= P.k || ope[j] == 0) continue;
@@ -350,37 +355,55 @@ __device__ float chain_candidate_y(const Plan& P, const W234& Wt, const float* s
         for (int i = 0; i < kKMax; i++)
             if (i < P.k && ope[i] != 0 && P.slot[i].model_id < P.slot[j].model_id) p++;
         const SlotP& s = P.slot[j];
-        sum_n += ope[j] - s.ops + 1;
         const int f = P.n_models + 4 * p;
-        const float xo = (float)s.ops, xe = (float)ope[j], xb = (float)s.bs, xs = (float)s.seqlen;
-#pragma unroll
-        for (int i = 0; i < kHidden; i++) {
-            const float* w = s_w1 + i * P.D;
-            float z = h1[i] + w[s.model_id - 1];
-            z = fmaf(w[f + 0], xo, z);
-            z = fmaf(w[f + 1], xe, z);
-            z = fmaf(w[f + 2], xb, z);
-            h1[i] = fmaf(w[f + 3], xs, z);
-        }
+        z += W.w1t[(s.model_id - 1) * kHidden + lane];
+        z = fmaf(W.w1t[(f + 0) * kHidden + lane], (float)s.ops, z);
+        z = fmaf(W.w1t[(f + 1) * kHidden + lane], (float)ope[j], z);
+        z = fmaf(W.w1t[(f + 2) * kHidden + lane], (float)s.bs, z);
+        z = fmaf(W.w1t[(f + 3) * kHidden + lane], (float)s.seqlen, z);
     }
+    float h = fmaxf(z, 0.0f);
+    float acc = W.b2[lane];
 #pragma unroll
-    for (int i = 0; i < kHidden; i++) h1[i] = fmaxf(h1[i], 0.0f);
-    float y;
-    mlp_tail_fp32(Wt, h1, y);
-    return y;
+    for (int j = 0; j < kHidden; j++) acc = fmaf(W.w2t[j * kHidden + lane], __shfl_sync(0xffffffffu, h, j), acc);
+    h = fmaxf(acc, 0.0f);
+    acc = W.b3[lane];
+#pragma unroll
+    for (int j = 0; j < kHidden; j++) acc = fmaf(W.w3t[j * kHidden + lane], __shfl_sync(0xffffffffu, h, j), acc);
+    h = fmaxf(acc, 0.0f);
+    float y = W.w4[lane] * h;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
+    return y + W.b4;
 }
 
 __global__ void __launch_bounds__(kMwayThreads, 1) mway_kernel(const __grid_constant__ Plan P,
                                                                 const __grid_constant__ W234 Wt,
                                                                 const float* __restrict__ w1b1, int ways,
                                                                 Scratch* S) {
-    extern __shared__ float s_w1[];  // W1[32][D] | b1[32]
-    __shared__ uint64_t s_probe[kMwayThreads];
-    __shared__ float s_y[kMwayThreads];
+    __shared__ MwaySmem W;
+    __shared__ uint64_t s_probe[128];
+    __shared__ float s_y[128];
     __shared__ int s_n, s_done, s_rounds, s_preds;
     __shared__ uint64_t s_lo, s_hi;
     __shared__ float s_ylo, s_y0;
-    for (int i = threadIdx.x; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = w1b1[i];
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    for (int i = threadIdx.x; i < kHidden * P.D; i += blockDim.x) {
+        const int o = i / P.D, c = i % P.D;
+        W.w1t[c * kHidden + o] = w1b1[i];
+    }
+    for (int i = threadIdx.x; i < kHidden * kHidden; i += blockDim.x) {
+        const int o = i / kHidden, c = i % kHidden;
+        W.w2t[c * kHidden + o] = Wt.W2[o][c];
+        W.w3t[c * kHidden + o] = Wt.W3[o][c];
+    }
+    if (threadIdx.x < kHidden) {
+        W.b1[threadIdx.x] = w1b1[kHidden * P.D + threadIdx.x];
+        W.b2[threadIdx.x] = Wt.b2[threadIdx.x];
+        W.b3[threadIdx.x] = Wt.b3[threadIdx.x];
+        W.w4[threadIdx.x] = Wt.w4[threadIdx.x];
+    }
+    if (threadIdx.x == 0) W.b4 = Wt.b4;
     if (threadIdx.x == 0) {
         // round 1: u = 0 and the block ends B_j = chain_cum[j + 1] - 1
         int n = 0;
@@ -394,9 +417,9 @@ __global__ void __launch_bounds__(kMwayThreads, 1) mway_kernel(const __grid_cons
     __syncthreads();
     for (int round = 0;; round++) {
         const int n = s_n;
-        if (threadIdx.x < n) {
-            int32_t sn;
-            s_y[threadIdx.x] = chain_candidate_y(P, Wt, s_w1, s_probe[threadIdx.x], sn);
+        for (int pi = (int)warp; pi < n; pi += (int)nwarps) {
+            const float yv = chain_candidate_y_warp(P, W, s_probe[pi], lane);
+            if (lane == 0) s_y[pi] = yv;
         }
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -434,17 +457,23 @@ __global__ void __launch_bounds__(kMwayThreads, 1) mway_kernel(const __grid_cons
                     }
                 s_lo = lo;
                 s_hi = hi;
-                const uint64_t span = hi - lo;
+                // a chain holds < 2^17 positions: 32-bit probe arithmetic
+                const uint32_t span = (uint32_t)(hi - lo);
                 if (span <= 1) {
                     s_done = 1;
                 } else {
                     int m = 0;
-                    if (span - 1 <= (uint64_t)ways) {
-                        for (uint64_t v = lo + 1; v < hi; v++) s_probe[m++] = v;
+                    if (span - 1 <= (uint32_t)ways) {
+                        for (uint32_t v = 1; v < span; v++) s_probe[m++] = lo + v;
                     } else {
+                        const uint32_t den = (uint32_t)ways + 1u;
+                        uint32_t prev = 0;
                         for (int i = 1; i <= ways; i++) {
-                            const uint64_t v = lo + (span * (uint64_t)i) / (uint64_t)(ways + 1);
-                            if (v > lo && v < hi && (m == 0 || v > s_probe[m - 1])) s_probe[m++] = v;
+                            const uint32_t v = (span * (uint32_t)i) / den;
+                            if (v > prev && v < span) {
+                                s_probe[m++] = lo + v;
+                                prev = v;
+                            }
                         }
                     }
                     s_n = m;
@@ -481,8 +510,8 @@ __global__ void __launch_bounds__(kMwayThreads, 1) mway_kernel(const __grid_cons
 }
 
 cudaError_t launch_mway(const Plan& P, const W234& W, const float* w1b1, int ways, Scratch* S, cudaStream_t st) {
-    const size_t smem = (size_t)(kHidden * P.D + kHidden) * sizeof(float);
-    mway_kernel<<<1, kMwayThreads, smem, st>>>(P, W, w1b1, ways, S);
+    if (P.D > 80) return cudaErrorInvalidValue;
+    mway_kernel<<<1, kMwayThreads, 0, st>>>(P, W, w1b1, ways, S);
     return cudaGetLastError();
 }
 
