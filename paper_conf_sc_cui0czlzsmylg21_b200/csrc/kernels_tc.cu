@@ -325,18 +325,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_after();
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
+    constexpr uint32_t id32 = idesc_f16(FMT, 32);
     uint64_t* barX = &bars[2 * g];
     uint64_t* barY = &bars[2 * g + 1];
     uint32_t phX = 0, phY = 0;
-    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
-#pragma unroll
-    for (int i = 0; i < C::kNchHid; i++) {
-        d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
-        d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
-    }
-#pragma unroll
-    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
+    const uint64_t db2 = smem_desc(sbase + L.w2), db3 = smem_desc(sbase + L.w3), db4 = smem_desc(sbase + L.w4);
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
 
@@ -373,17 +366,22 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         mma_commit_elect(bar);
     };
     // wait for layer l of T, epilogue (ReLU, pack) into A, hand off, issue layer l+1
-    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id, bool me,
-                     uint32_t idesc) {
+    // LAYER: 0 = layer 2, 1 = layer 3, 2 = output (N = 16)
+    auto stage = [&](auto layer_c, const TileIO& T, uint64_t* bar, uint32_t& ph, uint32_t bar_id, bool me) {
+        constexpr int LAYER = decltype(layer_c)::value;
         mbar_wait(bar, ph);
         ph ^= 1u;
         fence_after();
         hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
         if (handoff(bar_id, me)) {
-            issue_layer_e<FMT>(T.d, T.a, tC, dl, idesc);
-            mma_commit_elect(bar);
+            if (LAYER == 0) issue_layer_asm<FMT, idesc_f16(FMT, 32), kChunkBytesN32>(T.d, T.a, tC, db2, bar);
+            else if (LAYER == 1) issue_layer_asm<FMT, idesc_f16(FMT, 32), kChunkBytesN32>(T.d, T.a, tC, db3, bar);
+            else issue_layer_asm<FMT, idesc_f16(FMT, 16), kChunkBytesN16>(T.d, T.a, tC, db4, bar);
         }
     };
+    using L0 = std::integral_constant<int, 0>;
+    using L1 = std::integral_constant<int, 1>;
+    using L2 = std::integral_constant<int, 2>;
 
     unsigned long long best = 0;
     float best_y = __int_as_float(0x7fc00000);
@@ -421,12 +419,12 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         uint64_t w = wb;
         auto iteration = [&](auto guarded_c) {
             constexpr bool G = decltype(guarded_c)::value;
-            stage(X, barX, phX, d2, idX, meX[0], id32);
-            if (!G || yLive) stage(Y, barY, phY, d2, idY, meY[0], id32);
-            stage(X, barX, phX, d3, idX, meX[1], id32);
-            if (!G || yLive) stage(Y, barY, phY, d3, idY, meY[1], id32);
-            stage(X, barX, phX, d4, idX, meX[2], id16);
-            if (!G || yLive) stage(Y, barY, phY, d4, idY, meY[2], id16);
+            stage(L0{}, X, barX, phX, idX, meX[0]);
+            if (!G || yLive) stage(L0{}, Y, barY, phY, idY, meY[0]);
+            stage(L1{}, X, barX, phX, idX, meX[1]);
+            if (!G || yLive) stage(L1{}, Y, barY, phY, idY, meY[1]);
+            stage(L2{}, X, barX, phX, idX, meX[2]);
+            if (!G || yLive) stage(L2{}, Y, barY, phY, idY, meY[2]);
             // X: output ready -> fold (a5) -> start tile w + 2 while Y's output MMA runs
             mbar_wait(barX, phX);
             phX ^= 1u;

@@ -146,6 +146,64 @@ __device__ __forceinline__ void mma_commit_elect(uint64_t* bar) {
         : "memory");
 }
 
+// One whole layer in one asm block (called by all lanes of the issuing warp):
+// chunk descriptors are derived from the layer's base descriptor by 64-bit
+// adds (a chunk = CHUNK bytes = CHUNK >> 4 descriptor units; no carry out of
+// the 14-bit start-address field), the instruction descriptor is an
+// immediate, one elected lane issues the MMAs and the commit.
+//   FMT 0 (fp16):  D  = A[0:8) W_c0 + A[8:16) W_c1 + C bias
+//   FMT 1 (bf16):  D  = A[0:8) Whi_c0 + A[8:16) Whi_c1 + A[0:8) Wlo_c0 + A[8:16) Wlo_c1 + C bias
+template <int FMT, uint32_t IDESC, uint32_t CHUNK>
+__device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32_t tC, uint64_t dbase,
+                                                uint64_t* bar) {
+    constexpr uint32_t U = CHUNK >> 4;
+    if (FMT == 0) {
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1, d2;\n\t"
+            ".reg .b32 a8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %3, %5;\n\t"
+            "add.s64 d2, %3, %6;\n\t"
+            "add.u32 a8, %1, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %3, %7, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d1, %7, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], d2, %7, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t"
+            "}" ::"r"(tD),
+            "r"(tA), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(2 * U)),
+            "n"(IDESC)
+            : "memory");
+    } else {
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1, d2, d3, d4;\n\t"
+            ".reg .b32 a8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %3, %5;\n\t"
+            "add.s64 d2, %3, %6;\n\t"
+            "add.s64 d3, %3, %7;\n\t"
+            "add.s64 d4, %3, %8;\n\t"
+            "add.u32 a8, %1, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %3, %9, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d1, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d3, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], d4, %9, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t"
+            "}" ::"r"(tD),
+            "r"(tA), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(2 * U)),
+            "n"((uint64_t)(3 * U)), "n"((uint64_t)(4 * U)), "n"(IDESC)
+            : "memory");
+    }
+}
+
 // predicated forms: every lane of the issuing warps executes the instruction
 // stream, only `pred != 0` issues (no divergent branch around the issue)
 __device__ __forceinline__ void mma_ts_p(uint32_t pred, uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc,
