@@ -199,10 +199,12 @@ Plan plan_whole_grid(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T) {
     fill_slots(P, g);
     P.n_seg = 1;
     SegP& s = P.seg[0];
+    // slots right-aligned in the digits: digit kKMax-1 is the last (fastest) slot
+    const int off = kKMax - g->k;
+    for (int d = 0; d < kKMax; d++) s.cnt[d] = d < off ? 1u : (uint32_t)P.slot[d - off].radix;
     for (int j = 0; j < kKMax; j++) {
-        s.cnt[j] = j < g->k ? (uint32_t)P.slot[j].radix : 1u;
         s.pos[j] = -1;
-        s.dpos[j] = j;
+        s.dpos[j] = j < g->k ? off + j : -1;
     }
     finish_box(s);
     return P;

@@ -21,22 +21,24 @@ namespace abacus {
 // shared device helpers
 // ---------------------------------------------------------------------------
 
-// Fig. 8 row for one candidate whose slot j is present with end op ope[j]
-// (ope[j] == 0: absent).  Positions: present slots in ascending model id.
-__device__ __forceinline__ void write_fig8_row(const Plan& P, const int32_t (&ope)[kKMax], int16_t* row) {
+// Fig. 8 row for one candidate.  opeD[d] is the end op of the slot in digit d
+// (slots right-aligned: slot j = d - (kKMax - k)); 0 = absent.  Positions:
+// present slots in ascending model id.
+__device__ __forceinline__ void write_fig8_row(const Plan& P, const int32_t (&opeD)[kKMax], int16_t* row) {
     for (int i = 0; i < P.D; i++) row[i] = 0;
+    const int off = kKMax - P.k;
 #pragma unroll
-    for (int j = 0; j < kKMax; j++) {
-        if (j >= P.k || ope[j] == 0) continue;
+    for (int d = 0; d < kKMax; d++) {
+        if (d < off || opeD[d] == 0) continue;
+        const SlotP& s = P.slot[d - off];
         int p = 0;
 #pragma unroll
-        for (int i = 0; i < kKMax; i++)
-            if (i < P.k && ope[i] != 0 && P.slot[i].model_id < P.slot[j].model_id) p++;
-        const SlotP& s = P.slot[j];
+        for (int e = 0; e < kKMax; e++)
+            if (e >= off && opeD[e] != 0 && P.slot[e - off].model_id < s.model_id) p++;
         row[s.model_id - 1] = 1;
         int16_t* f = row + P.n_models + 4 * p;
         f[0] = (int16_t)s.ops;
-        f[1] = (int16_t)ope[j];
+        f[1] = (int16_t)opeD[d];
         f[2] = (int16_t)s.bs;
         f[3] = (int16_t)s.seqlen;
     }
@@ -75,10 +77,11 @@ __global__ void __launch_bounds__(kEncThreads) encode_grid_kernel(const __grid_c
         const uint64_t idx = base + threadIdx.x;
         uint32_t v[kKMax];
         decode_box<kKMax>(g, first + base, threadIdx.x, v);
-        int32_t ope[kKMax];
+        int32_t opeD[kKMax];
+        const int off = kKMax - P.k;
 #pragma unroll
-        for (int j = 0; j < kKMax; j++) ope[j] = j < P.k ? digit_to_ope(P.slot[j], v[j]) : 0;
-        if (idx < count) write_fig8_row(P, ope, s_rows + threadIdx.x * P.D);
+        for (int d = 0; d < kKMax; d++) opeD[d] = d >= off ? digit_to_ope(P.slot[d - off], v[d]) : 0;
+        if (idx < count) write_fig8_row(P, opeD, s_rows + threadIdx.x * P.D);
         __syncthreads();
         const uint64_t nrows = min((uint64_t)kEncThreads, count - base);
         store_rows(s_rows, out + base * P.D, nrows * P.D * 2);
@@ -191,32 +194,82 @@ __global__ void __launch_bounds__(kPredThreads) predict_fp32_kernel(const __grid
 }
 
 // ---------------------------------------------------------------------------
-// a5: headroom mask + largest-group key over a grid range.  One thread per t;
-// warp shuffle max -> shared -> one atomicMax(u64) per block.
+// a5: headroom mask + largest-group key over a grid range.  Each thread walks
+// kSelPer consecutive candidates (two 16-byte loads of y), decoding only the
+// first index; the following ones advance the fastest digit with a carry
+// check.  Warp shuffle max -> shared -> one atomicMax(u64) per block.
+// plan.seg[0] is the whole grid with the slots right-aligned in the digits
+// (digit 3 = last slot), see plan_whole_grid.
 // ---------------------------------------------------------------------------
 constexpr int kSelThreads = 256;
+constexpr int kSelPer = 32;
 
 __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_constant__ Plan P, uint64_t first,
                                                              uint64_t count, const float* __restrict__ lat,
                                                              float H, unsigned long long* best) {
     __shared__ unsigned long long s_max[kSelThreads / 32];
     const SegP& g = P.seg[0];
-    unsigned long long mx = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kSelThreads; base < count;
-         base += (uint64_t)gridDim.x * kSelThreads) {
-        const uint64_t idx = base + threadIdx.x;
-        if (idx >= count) break;
-        uint32_t v[kKMax];
-        decode_box<kKMax>(g, first + base, threadIdx.x, v);
-        int32_t sum_n = 0;
+    const int off = kKMax - P.k;  // digit of slot j = off + j
+    // n of slot j at digit value d: 0 if absent (d == 0 and absent allowed), else nb_j + d
+    int32_t nb[kKMax];
+    bool ab[kKMax];
 #pragma unroll
-        for (int j = 0; j < kKMax; j++) {
-            if (j >= P.k) continue;
-            const int32_t e = digit_to_ope(P.slot[j], v[j]);
-            if (e != 0) sum_n += e - P.slot[j].ops + 1;
+    for (int d = 0; d < kKMax; d++) {
+        const int j = d - off;
+        if (j < 0) {
+            nb[d] = 0;
+            ab[d] = true;
+            continue;
         }
-        const float yv = lat[idx];
-        if (yv <= H) mx = umax64(mx, ((unsigned long long)(sum_n + 1) << 40) | (first + idx));
+        const SlotP& s = P.slot[j];
+        ab[d] = s.absent != 0;
+        nb[d] = s.end_lo - s.ops + 1 - s.absent;
+    }
+    const uint32_t cnt3 = g.cnt[kKMax - 1];
+    unsigned long long mx = 0;
+    const uint64_t chunk = (uint64_t)kSelThreads * kSelPer;
+    for (uint64_t base = (uint64_t)blockIdx.x * chunk; base < count; base += (uint64_t)gridDim.x * chunk) {
+        const uint64_t i0 = base + (uint64_t)threadIdx.x * kSelPer;
+        if (i0 >= count) continue;
+        float y[kSelPer];
+        const float* src = lat + i0;
+        if (i0 + kSelPer <= count && (reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+#pragma unroll
+            for (int q = 0; q < kSelPer / 4; q++) {
+                const float4 a = __ldcs(reinterpret_cast<const float4*>(src) + q);
+                y[4 * q] = a.x; y[4 * q + 1] = a.y; y[4 * q + 2] = a.z; y[4 * q + 3] = a.w;
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < kSelPer; q++) y[q] = i0 + q < count ? src[q] : __int_as_float(0x7fc00000);
+        }
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, first + base, threadIdx.x * kSelPer, v);
+        auto nsum_rest = [&]() {
+            int32_t r = 0;
+#pragma unroll
+            for (int d = 0; d < kKMax - 1; d++) r += (ab[d] && v[d] == 0) ? 0 : nb[d] + (int32_t)v[d];
+            return r;
+        };
+        int32_t rest = nsum_rest();
+        const uint64_t t0 = first + i0;
+#pragma unroll
+        for (int q = 0; q < kSelPer; q++) {
+            if (y[q] <= H) {
+                const int32_t n3 = (ab[kKMax - 1] && v[kKMax - 1] == 0) ? 0 : nb[kKMax - 1] + (int32_t)v[kKMax - 1];
+                mx = umax64(mx, ((unsigned long long)(rest + n3 + 1) << 40) | (t0 + q));
+            }
+            // advance to t + 1
+            if (++v[kKMax - 1] == cnt3) {
+                v[kKMax - 1] = 0;
+#pragma unroll
+                for (int d = kKMax - 2; d >= 0; d--) {
+                    if (++v[d] < g.cnt[d]) break;
+                    v[d] = 0;
+                }
+                rest = nsum_rest();
+            }
+        }
     }
     mx = warp_max_u64(mx);
     if ((threadIdx.x & 31) == 0) s_max[threadIdx.x >> 5] = mx;
@@ -552,7 +605,7 @@ cudaError_t launch_predict_fp32(const W234& W, const float* w1b1, int32_t D, con
 cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const float* lat, float H,
                           unsigned long long* best, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
-    const uint64_t blocks = (count + kSelThreads - 1) / kSelThreads;
+    const uint64_t blocks = (count + kSelThreads * kSelPer - 1) / (kSelThreads * kSelPer);
     const int grid = (int)(blocks < (uint64_t)nsm * 8 ? blocks : (uint64_t)nsm * 8);
     select_kernel<<<grid, kSelThreads, 0, st>>>(P, first, count, lat, H, best);
     return cudaGetLastError();
