@@ -484,6 +484,79 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
 //   A1 row = [x_hi (D values), x_lo (D values), 1, 1, 0...], x = 256 x_hi + x_lo
 //   B1     = [256 W1 | W1 | b1_hi | b1_lo]  (bf16: second set of chunks = lo halves)
 // ---------------------------------------------------------------------------
+// Fast layer-1 layout for even D (here D = 24): x = 2^S hi + lo with
+// lo in [0, 2^S) entered as the exact value 2^S0 + lo built by bit operations
+// (fp16: S = 10, 1024 + lo = bits 0x6400 | lo; bf16: S = 7, 128 + lo = bits
+// 0x4300 | lo) and hi converted exactly.  B columns: lo -> w, hi -> 2^S w; the
+// constant offset 2^S0 sum_j w_j of the lo entries is removed from the bias.
+template <int FMT>
+struct Split {
+    static constexpr int S = FMT == 0 ? 10 : 7;
+    static constexpr uint32_t LOMASK2 = FMT == 0 ? 0x03FF03FFu : 0x007F007Fu;
+    static constexpr uint32_t MAGIC2 = FMT == 0 ? 0x64006400u : 0x43004300u;
+    static constexpr float OFFSET = FMT == 0 ? 1024.0f : 128.0f;
+};
+
+template <int FMT>
+__device__ void build_b1_predict_fast(const float* __restrict__ w1b1, int D, float scale, uint8_t* s_b1, int nch) {
+    const float* b1 = w1b1 + kHidden * D;
+    const int K = nch * 16;
+    for (int e = threadIdx.x; e < kHidden * K; e += blockDim.x) {
+        const int n = e / K, k = e % K;
+        uint16_t v0 = 0, v1 = 0;
+        if (k < 2 * D) {
+            const float w = w1b1[n * D + (k % D)] * scale;
+            const float m = k < D ? 1.0f : (float)(1 << Split<FMT>::S);
+            uint16_t h, l;
+            split16<FMT>(w, h, l);
+            if (FMT == 0) {
+                v0 = to16<FMT>(w * m);
+            } else {
+                v0 = to16<FMT>(from16<FMT>(h) * m);
+                v1 = to16<FMT>(from16<FMT>(l) * m);
+            }
+        } else if (k < 2 * D + 2) {
+            // bias minus the lo offsets (computed with the weights as the MMA sees them)
+            double off = 0.0;
+            for (int j = 0; j < D; j++) {
+                const float w = w1b1[n * D + j] * scale;
+                double wq;
+                if (FMT == 0) {
+                    wq = (double)from16<FMT>(to16<FMT>(w));
+                } else {
+                    uint16_t h, l;
+                    split16<FMT>(w, h, l);
+                    wq = (double)from16<FMT>(h) + (double)from16<FMT>(l);
+                }
+                off += wq * (double)Split<FMT>::OFFSET;
+            }
+            const float bb = (float)((double)b1[n] * (double)scale - off);
+            uint16_t h, l;
+            split16<FMT>(bb, h, l);
+            v0 = k == 2 * D ? h : l;
+        }
+        const int ch = k >> 4, kk = k & 15;
+        *reinterpret_cast<uint16_t*>(s_b1 + (size_t)ch * kChunkBytesN32 + b_offset(n, kk)) = v0;
+        if (FMT == 1)
+            *reinterpret_cast<uint16_t*>(s_b1 + (size_t)(nch + ch) * kChunkBytesN32 + b_offset(n, kk)) = v1;
+    }
+}
+
+// layer-1 operand row for D = 24 from the 12 packed int16 pairs of a row
+template <int FMT>
+__device__ __forceinline__ void encode_row24(const uint32_t (&w)[12], uint32_t (&a)[32]) {
+#pragma unroll
+    for (int i = 0; i < 12; i++) {
+        a[i] = (w[i] & Split<FMT>::LOMASK2) | Split<FMT>::MAGIC2;        // lo pair, exact 2^S0 + lo
+        const int32_t x0 = (int32_t)(w[i] << 16) >> (16 + Split<FMT>::S);  // sign-extended hi parts
+        const int32_t x1 = (int32_t)w[i] >> (16 + Split<FMT>::S);
+        a[12 + i] = pack2<FMT>((float)x0, (float)x1);
+    }
+    a[24] = TcCfg<FMT>::kOne2;
+#pragma unroll
+    for (int i = 25; i < 32; i++) a[i] = 0;
+}
+
 template <int FMT>
 __device__ void build_b1_predict(const float* __restrict__ w1b1, int D, float scale, uint8_t* s_b1, int nch) {
     const float* b1 = w1b1 + kHidden * D;
@@ -544,7 +617,9 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
         int4* dst = reinterpret_cast<int4*>(smem);
         for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
     }
-    build_b1_predict<FMT>(w1b1, D, TP.l1_scale, smem + L.b1, nch);
+    const bool fast24 = D == 24;  // magic-number layer-1 layout (encode_row24)
+    if (fast24) build_b1_predict_fast<FMT>(w1b1, D, TP.l1_scale, smem + L.b1, nch);
+    else build_b1_predict<FMT>(w1b1, D, TP.l1_scale, smem + L.b1, nch);
     if (tid == 0) {
         for (int i = 0; i < 2 * NG; i++) {
             mbar_init(&bars[i], 1);
@@ -659,6 +734,32 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
             rowp = reinterpret_cast<const int16_t*>(st) + (size_t)min(r, nrows - 1) * D;
         } else {
             rowp = x + (row0 + min(r, nrows - 1)) * (uint64_t)D;
+        }
+        if (fast24) {
+            uint32_t wv[12];
+            const uint4* rp = reinterpret_cast<const uint4*>(rowp);
+            const bool al = (reinterpret_cast<uintptr_t>(rowp) & 15u) == 0;
+#pragma unroll
+            for (int q = 0; q < 3; q++) {
+                uint4 v4;
+                if (al) v4 = rp[q];
+                else {
+                    const uint32_t* r32 = reinterpret_cast<const uint32_t*>(rowp) + 4 * q;
+                    v4 = make_uint4(r32[0], r32[1], r32[2], r32[3]);
+                }
+                wv[4 * q] = v4.x; wv[4 * q + 1] = v4.y; wv[4 * q + 2] = v4.z; wv[4 * q + 3] = v4.w;
+            }
+            uint32_t av[32];
+            encode_row24<FMT>(wv, av);
+#pragma unroll
+            for (int cb = 0; cb < 4; cb++) {
+                uint32_t a8[8];
+#pragma unroll
+                for (int i = 0; i < 8; i++) a8[i] = av[8 * cb + i];
+                tmem_st8(T.a1 + lane_off + 8 * cb, a8);
+            }
+            tmem_wait_st();
+            return;
         }
         for (int cb = 0; cb < nch; cb++) {
             uint32_t a[8];
