@@ -89,6 +89,100 @@ __global__ void __launch_bounds__(kEncThreads) encode_grid_kernel(const __grid_c
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// a2 + a3 fast path for D = 24 (N = 8): per block 1024 consecutive candidates,
+// thread t builds rows t, t + 128, ... in a shared-memory stage (3 x 16-byte
+// stores for the bitmap and zeros, then 2 x 4-byte stores per present model at
+// its Fig.-8 position, read from a per-presence-pattern table), and one thread
+// writes the whole 48 KB stage to HBM with a TMA bulk store (double-buffered).
+// ---------------------------------------------------------------------------
+constexpr int kEnc24Threads = 128;
+constexpr int kEnc24Rows = 1024;
+
+__global__ void __launch_bounds__(kEnc24Threads) encode_grid24_kernel(const __grid_constant__ Plan P, uint64_t first,
+                                                                      uint64_t count, int16_t* __restrict__ out) {
+    extern __shared__ __align__(128) uint8_t s_enc[];
+    uint4* stage = reinterpret_cast<uint4*>(s_enc);                  // 2 x 1024 rows x 3 uint4
+    uint4* s_bm = stage + 2 * kEnc24Rows * 3;                          // [16] bitmap words per mask
+    int8_t* s_pos = reinterpret_cast<int8_t*>(s_bm + 16);              // [16][4] Fig.-8 position per digit
+    const SegP& g = P.seg[0];
+    const int off = kKMax - P.k;
+    if (threadIdx.x < 16) {
+        const uint32_t mask = threadIdx.x;  // bit d: digit d present
+        uint32_t w[4] = {0, 0, 0, 0};
+        for (int d = 0; d < kKMax; d++) {
+            int8_t p = -1;
+            if (d >= off && ((mask >> d) & 1u)) {
+                const int m = P.slot[d - off].model_id;
+                w[(m - 1) >> 1] |= 1u << (16 * ((m - 1) & 1));
+                p = 0;
+                for (int e = off; e < kKMax; e++)
+                    if (((mask >> e) & 1u) && P.slot[e - off].model_id < m) p++;
+            }
+            s_pos[threadIdx.x * 4 + d] = p;
+        }
+        s_bm[threadIdx.x] = make_uint4(w[0], w[1], w[2], w[3]);
+    }
+    // per digit: (ops | ope0 << 16) base word and the constant (bs | seqlen << 16) word
+    uint32_t opsw[kKMax], bsw[kKMax];
+    int32_t elo[kKMax];
+    bool abs_[kKMax];
+#pragma unroll
+    for (int d = 0; d < kKMax; d++) {
+        if (d < off) {
+            opsw[d] = bsw[d] = 0;
+            elo[d] = 0;
+            abs_[d] = true;
+            continue;
+        }
+        const SlotP& s = P.slot[d - off];
+        opsw[d] = (uint32_t)(uint16_t)s.ops;
+        bsw[d] = (uint32_t)(uint16_t)s.bs | ((uint32_t)(uint16_t)s.seqlen << 16);
+        elo[d] = s.end_lo - s.absent;  // ope = elo + digit (for a present digit)
+        abs_[d] = s.absent != 0;
+    }
+    __syncthreads();
+    int it = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kEnc24Rows; base < count;
+         base += (uint64_t)gridDim.x * kEnc24Rows, it++) {
+        uint4* st = stage + (it & 1) * kEnc24Rows * 3;
+        if (it >= 2 && threadIdx.x == 0)
+            asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // stage reused two rounds later
+        __syncthreads();
+        const uint32_t nrows = (uint32_t)min((uint64_t)kEnc24Rows, count - base);
+        for (uint32_t r = threadIdx.x; r < nrows; r += kEnc24Threads) {
+            uint32_t v[kKMax];
+            decode_box<kKMax>(g, first + base, r, v);
+            uint32_t mask = 0;
+#pragma unroll
+            for (int d = 0; d < kKMax; d++)
+                if (d >= off && !(abs_[d] && v[d] == 0)) mask |= 1u << d;
+            uint4* row = st + r * 3;
+            row[0] = s_bm[mask];
+            row[1] = make_uint4(0, 0, 0, 0);
+            row[2] = make_uint4(0, 0, 0, 0);
+            uint32_t* rw = reinterpret_cast<uint32_t*>(row);
+#pragma unroll
+            for (int d = 0; d < kKMax; d++) {
+                const int p = s_pos[mask * 4 + d];
+                if (p < 0) continue;
+                rw[4 + 2 * p] = opsw[d] | ((uint32_t)(elo[d] + (int32_t)v[d]) << 16);
+                rw[5 + 2 * p] = bsw[d];
+            }
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(out + base * 24),
+                         "r"((uint32_t)__cvta_generic_to_shared(st)), "r"(nrows * 48u)
+                         : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
 // ---------------------------------------------------------------------------
 // a3 for explicit groups (config-5 instance samples)
 // ---------------------------------------------------------------------------
@@ -574,6 +668,16 @@ cudaError_t launch_mway(const Plan& P, const W234& W, const float* w1b1, int way
 cudaError_t launch_encode_grid(const Plan& P, uint64_t first, uint64_t count, int16_t* out, int nsm,
                                cudaStream_t st) {
     if (count == 0) return cudaSuccess;
+    if (P.D == 24 && (reinterpret_cast<uintptr_t>(out) & 15u) == 0) {
+        const size_t smem = 2 * kEnc24Rows * 3 * sizeof(uint4) + 16 * sizeof(uint4) + 64;
+        cudaError_t e = cudaFuncSetAttribute(encode_grid24_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)smem);
+        if (e != cudaSuccess) return e;
+        const uint64_t blocks = (count + kEnc24Rows - 1) / kEnc24Rows;
+        const int grid = (int)(blocks < (uint64_t)nsm * 2 ? blocks : (uint64_t)nsm * 2);
+        encode_grid24_kernel<<<grid, kEnc24Threads, smem, st>>>(P, first, count, out);
+        return cudaGetLastError();
+    }
     const uint64_t blocks = (count + kEncThreads - 1) / kEncThreads;
     const int grid = (int)(blocks < (uint64_t)nsm * 16 ? blocks : (uint64_t)nsm * 16);
     const size_t smem = (size_t)kEncThreads * P.D * sizeof(int16_t);
