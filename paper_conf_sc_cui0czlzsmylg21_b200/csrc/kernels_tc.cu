@@ -266,7 +266,7 @@ __device__ __forceinline__ float output_dot(uint32_t tD_lane, const OutW& O) {
     return acc0 + acc1;
 }
 
-template <int FMT, bool SPLIT, int NG>
+template <int FMT, bool SPLIT, int NG, bool TRACE>
 __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
                                                                const __grid_constant__ TcParams TP,
                                                                const __grid_constant__ OutW O,
@@ -326,21 +326,24 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
     constexpr uint32_t id32 = idesc_f16(FMT, 32);
-    uint64_t* barX = &bars[2 * g];
-    uint64_t* barY = &bars[2 * g + 1];
-    uint32_t phX = 0, phY = 0;
+    constexpr uint32_t id16 = idesc_f16(FMT, 16);
+    uint64_t* bar = &bars[g];
+    uint32_t ph = 0;
     const uint64_t db2 = smem_desc(sbase + L.w2), db3 = smem_desc(sbase + L.w3), db4 = smem_desc(sbase + L.w4);
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
 
+    // The group's two tiles (slots X and Y) move through the layers in lock
+    // step: one MMA commit covers both, so each stage costs ONE mbarrier wait,
+    // two overlapped TMEM loads, one tcgen05.st wait and ONE hand-off for two
+    // tiles; the other groups of the CTA keep the tensor pipe busy meanwhile.
     // Operand hand-off: after writing its 32 rows a warp fences its tcgen05.st
-    // and ARRIVES on the slot's named barrier without blocking; only the
+    // and ARRIVES on the group's named barrier without blocking; only the
     // stage's issuing warp SYNCs (waits for all 128 threads), then issues the
-    // MMAs from one elected lane and commits them to the slot's mbarrier.  The
-    // issuer rotates over the group's 4 warps (one per SMSP) stage by stage.
-    // Slots X and Y use different barrier ids, so a warp running ahead can
-    // never arrive in the wrong phase.
-    auto handoff = [&](uint32_t bar_id, bool me) -> bool {
+    // MMAs from one elected lane and commits them to the group's mbarrier.
+    // The issuer rotates over the group's 4 warps (one per SMSP) stage by stage.
+    const uint32_t bar_id = 1 + g;
+    auto handoff = [&](bool me) -> bool {
         fence_before();
         if (me) {
             named_bar_sync(bar_id, 128);
@@ -350,38 +353,86 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         }
         return me;
     };
-    const uint32_t idX = 1 + 2 * g, idY = 2 + 2 * g;
-    // issuer of hand-off position p (0: L2, 1: L3, 2: out, 3: next L1) of slot X / Y
-    bool meX[4], meY[4];
+    // issuer of hand-off position p (0: L2, 1: L3, 2: out, 3: next L1)
+    bool me[4];
 #pragma unroll
-    for (int p = 0; p < 4; p++) {
-        meX[p] = ((g + p) & 3) == wq;
-        meY[p] = ((g + 2 + p) & 3) == wq;
-    }
-    auto issue_l1 = [&](const TileIO& T, int s, uint64_t* bar) {
+    for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
+    auto issue_l1 = [&](const TileIO& T, int s) {
         const int su = __shfl_sync(0xffffffffu, s, 0);
         const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
         mma_ts_elect(T.d, T.a1, db, id32, 0u);
         if (C::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
-        mma_commit_elect(bar);
     };
-    // wait for layer l of T, epilogue (ReLU, pack) into A, hand off, issue layer l+1
-    // LAYER: 0 = layer 2, 1 = layer 3, 2 = output (N = 16)
-    auto stage = [&](auto layer_c, const TileIO& T, uint64_t* bar, uint32_t& ph, uint32_t bar_id, bool me) {
+    // layer LAYER (0: layer 2, 1: layer 3, 2: output) of X (and Y), one commit
+    auto issue_next = [&](auto layer_c, auto two_c) {
         constexpr int LAYER = decltype(layer_c)::value;
+        constexpr bool TWO = decltype(two_c)::value;
+        constexpr uint32_t CH = LAYER == 2 ? kChunkBytesN16 : kChunkBytesN32;
+        constexpr uint32_t ID = LAYER == 2 ? id16 : id32;
+        const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
+        if (FMT == 0 && TWO) {
+            issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tC, db, bar);
+        } else if (!TWO) {
+            issue_layer_asm<FMT, ID, CH>(X.d, X.a, tC, db, bar);
+        } else {
+            uint64_t d[5];
+#pragma unroll
+            for (int i = 0; i < 5; i++) d[i] = db + (uint64_t)(i * (CH >> 4));
+            issue_layer_e<FMT>(X.d, X.a, tC, d, ID);
+            issue_layer_e<FMT>(Y.d, Y.a, tC, d, ID);
+            mma_commit_elect(bar);
+        }
+    };
+    // debug timeline (tools/stage_trace.py): CTA 0, group 0, lane 0 of each warp, 12 stages
+    const bool tr = TRACE && P.trace != nullptr && blockIdx.x == 0 && g == 0 && (tid & 31) == 0;
+    int trn = 0;
+    constexpr int kTr0 = 40;  // first traced stage (steady state)
+    auto tstamp = [&](int slot) {
+        if (TRACE && tr && trn >= kTr0 && trn < kTr0 + 12) {
+            long long c;
+            asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
+            P.trace[16 + (wq * 12 + trn - kTr0) * 6 + slot] = (unsigned long long)c;
+        }
+    };
+    auto tnext = [&](bool mine) {
+        if (TRACE && tr) {
+            if (trn >= kTr0 && trn < kTr0 + 12) P.trace[16 + (wq * 12 + trn - kTr0) * 6 + 5] = mine ? 1ull : 0ull;
+            trn++;
+        }
+    };
+    // wait for layer LAYER-1's MMAs, epilogue (ReLU, pack) into A, hand off, issue layer LAYER
+    auto stage = [&](auto layer_c, auto two_c) {
+        constexpr bool TWO = decltype(two_c)::value;
+        tstamp(0);
         mbar_wait(bar, ph);
         ph ^= 1u;
         fence_after();
-        hidden_epilogue<FMT>(T.d + lane_off, T.a + lane_off);
-        if (handoff(bar_id, me)) {
-            if (LAYER == 0) issue_layer_asm<FMT, idesc_f16(FMT, 32), kChunkBytesN32>(T.d, T.a, tC, db2, bar);
-            else if (LAYER == 1) issue_layer_asm<FMT, idesc_f16(FMT, 32), kChunkBytesN32>(T.d, T.a, tC, db3, bar);
-            else issue_layer_asm<FMT, idesc_f16(FMT, 16), kChunkBytesN16>(T.d, T.a, tC, db4, bar);
+        tstamp(1);
+        if (TWO) {
+            uint32_t a[32], b[32], h[16];
+            tmem_ld32x2(X.d + lane_off, Y.d + lane_off, a, b);
+#pragma unroll
+            for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(a[2 * c], a[2 * c + 1]);
+            tmem_st16(X.a + lane_off, h);
+#pragma unroll
+            for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(b[2 * c], b[2 * c + 1]);
+            tmem_st16(Y.a + lane_off, h);
+            tmem_wait_st();
+        } else {
+            hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
         }
+        tstamp(2);
+        const bool mine = handoff(me[decltype(layer_c)::value]);
+        tstamp(3);
+        if (mine) issue_next(layer_c, two_c);
+        tstamp(4);
+        tnext(mine);
     };
     using L0 = std::integral_constant<int, 0>;
     using L1 = std::integral_constant<int, 1>;
     using L2 = std::integral_constant<int, 2>;
+    using T1 = std::integral_constant<bool, false>;
+    using T2 = std::integral_constant<bool, true>;
 
     unsigned long long best = 0;
     float best_y = __int_as_float(0x7fc00000);
@@ -391,8 +442,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         Walker W;
         walker_begin(P, W, wb, r);
         uint32_t vX[kKMax], vY[kKMax];
-        int sX, sY;
-        bool okX, okY, zX, zY;
+        int sX = 0, sY = 0;
+        bool okX = false, okY = false, zX = false, zY = false;
         auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z) {
             ok = W.u_end - W.ub > (uint64_t)r;
             z = walker_is_index0(W, r);
@@ -400,8 +451,13 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             for (int j = 0; j < kKMax; j++) v[j] = W.v[j];
             s = W.s;
         };
+        auto fold = [&](uint32_t yb, int s, const uint32_t (&v)[kKMax], bool ok, bool z) {
+            const float y = __uint_as_float(yb);
+            if (ok && z) S->y0 = y;
+            if (ok) fold_tile(P, s, v, y, best, best_y);
+        };
         // prologue: tile wb in slot X and (if the group has it) wb + 1 in slot Y
-        bool xLive = true, yLive = wb + 1 < we;  // warp-uniform
+        const bool yLive = wb + 1 < we;  // warp-uniform
         take(vX, sX, okX, zX);
         store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
         if (yLive) {
@@ -410,65 +466,61 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
         }
         tmem_wait_st();
-        if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
-        if (yLive && handoff(idY, meY[3])) issue_l1(Y, sY, barY);
+        if (handoff(me[3])) {
+            issue_l1(X, sX);
+            if (yLive) issue_l1(Y, sY);
+            mma_commit_elect(bar);
+        }
 
-        // one iteration = the remaining layers of the tiles in X and Y, then the
-        // next tiles (w + 2, w + 3) enter the slots.  GUARDED = the tail, where a
-        // slot may be empty or have no successor; the steady state skips the checks.
+        // one iteration = layers 2, 3, out of the tiles in X (and Y), fold (a5),
+        // then tiles w + 2 (and w + 3) enter the slots.  The steady state has
+        // both slots full before and after; the tail handles a lone X.
         uint64_t w = wb;
-        auto iteration = [&](auto guarded_c) {
-            constexpr bool G = decltype(guarded_c)::value;
-            stage(L0{}, X, barX, phX, idX, meX[0]);
-            if (!G || yLive) stage(L0{}, Y, barY, phY, idY, meY[0]);
-            stage(L1{}, X, barX, phX, idX, meX[1]);
-            if (!G || yLive) stage(L1{}, Y, barY, phY, idY, meY[1]);
-            stage(L2{}, X, barX, phX, idX, meX[2]);
-            if (!G || yLive) stage(L2{}, Y, barY, phY, idY, meY[2]);
-            // X: output ready -> fold (a5) -> start tile w + 2 while Y's output MMA runs
-            mbar_wait(barX, phX);
-            phX ^= 1u;
+        auto iteration = [&](auto two_c, auto next_two_c) {
+            constexpr bool TWO = decltype(two_c)::value;
+            constexpr bool NTWO = decltype(next_two_c)::value;
+            stage(L0{}, two_c);
+            stage(L1{}, two_c);
+            stage(L2{}, two_c);
+            tstamp(0);
+            mbar_wait(bar, ph);
+            ph ^= 1u;
             fence_after();
-            {
-                uint32_t yb;
-                tmem_ld1(X.d + lane_off, yb);
-                const float y = __uint_as_float(yb);
-                if (okX && zX) S->y0 = y;
-                if (okX) fold_tile(P, sX, vX, y, best, best_y);
+            tstamp(1);
+            uint32_t ybx, yby = 0;
+            if (TWO) {
+                tmem_ld1x2(X.d + lane_off, Y.d + lane_off, ybx, yby);
+            } else {
+                tmem_ld1(X.d + lane_off, ybx);
             }
-            if (G) xLive = w + 2 < we;
-            if (!G || xLive) {
+            fold(ybx, sX, vX, okX, zX);
+            if (TWO) fold(yby, sY, vY, okY, zY);
+            tstamp(2);
+            if (w + 2 < we) {
                 walker_next(P, W, w + 2, r);
                 take(vX, sX, okX, zX);
                 store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
-                tmem_wait_st();
-                if (handoff(idX, meX[3])) issue_l1(X, sX, barX);
-            }
-            if (!G || yLive) {
-                // Y: the same, next tile w + 3
-                mbar_wait(barY, phY);
-                phY ^= 1u;
-                fence_after();
-                {
-                    uint32_t yb;
-                    tmem_ld1(Y.d + lane_off, yb);
-                    const float y = __uint_as_float(yb);
-                    if (okY && zY) S->y0 = y;
-                    if (okY) fold_tile(P, sY, vY, y, best, best_y);
-                }
-                if (G) yLive = w + 3 < we;
-                if (!G || yLive) {
+                if (NTWO) {
                     walker_next(P, W, w + 3, r);
                     take(vY, sY, okY, zY);
                     store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
-                    tmem_wait_st();
-                    if (handoff(idY, meY[3])) issue_l1(Y, sY, barY);
                 }
+                tmem_wait_st();
+                tstamp(3);
+                const bool mine = handoff(me[3]);
+                if (mine) {
+                    issue_l1(X, sX);
+                    if (NTWO) issue_l1(Y, sY);
+                    mma_commit_elect(bar);
+                }
+                tstamp(4);
+                tnext(mine);
             }
             w += 2;
         };
-        while (w + 3 < we) iteration(std::integral_constant<bool, false>{});  // both slots full, both continue
-        while (xLive) iteration(std::integral_constant<bool, true>{});
+        while (w + 3 < we) iteration(T2{}, T2{});  // both slots full, both continue
+        if (w + 1 < we) iteration(T2{}, T1{});    // both full; at most X gets a successor
+        if (w < we) iteration(T1{}, T1{});        // X alone
     }
     trace_stamp(P, 3);
     fence_before();
@@ -868,7 +920,7 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const Out
     using C = TcCfg<FMT>;
     const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG,
                                          w1_stage_bytes(P.D, 2 * kFusedNG));
-    auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
+    auto kern = P.trace ? fused_tc_kernel<FMT, SPLIT, kFusedNG, true> : fused_tc_kernel<FMT, SPLIT, kFusedNG, false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
     // spread the tiles over as many SMs as possible (one tile per group first)

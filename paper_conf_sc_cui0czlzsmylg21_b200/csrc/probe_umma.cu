@@ -8,6 +8,8 @@
 // variant 1: descriptor fields swapped (LBO=256, SBO=128)
 // variant 2: as 0 but A at column 40 (A address not 32-aligned)
 // variant 3: as 0, and the same A/B issued twice with accumulate (D = 2 A B^T)
+// variant 4: as 0 with an f16 accumulator (idesc c_format = F16); raw D words
+// variant 5: as 4, issued twice with accumulate
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -53,9 +55,10 @@ __global__ void probe_kernel(int fmt, int variant, int N, const uint32_t* __rest
         fence_after();
         const uint32_t saddr = smem_u32(sb);
         const uint64_t desc = variant == 1 ? smem_desc(saddr, 256, 128) : smem_desc(saddr, 128, 256);
-        const uint32_t id = idesc_f16(fmt, N);
+        uint32_t id = idesc_f16(fmt, N);
+        if (variant >= 4) id &= ~(3u << 4);  // D format F16
         mma_ts(tb, tb + acol, desc, id, 0u);
-        if (variant == 3) mma_ts(tb, tb + acol, desc, id, 1u);
+        if (variant == 3 || variant == 5) mma_ts(tb, tb + acol, desc, id, 1u);
         mma_commit(&bar);
     }
     mbar_wait(&bar, 0);

@@ -204,6 +204,37 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
     }
 }
 
+// the MMAs of one layer for TWO tiles (same B operand) and ONE commit
+template <int FMT, uint32_t IDESC, uint32_t CHUNK>
+__device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
+                                                 uint32_t tC, uint64_t dbase, uint64_t* bar) {
+    static_assert(FMT == 0, "lock-step pair issue: fp16 layout");
+    constexpr uint32_t U = CHUNK >> 4;
+    asm volatile(
+        "{\n\t"
+        ".reg .pred e, pf, pt;\n\t"
+        ".reg .b64 d1, d2;\n\t"
+        ".reg .b32 ax8, ay8;\n\t"
+        "setp.ne.b32 pf, 0, 0;\n\t"
+        "setp.eq.b32 pt, 0, 0;\n\t"
+        "add.s64 d1, %5, %7;\n\t"
+        "add.s64 d2, %5, %8;\n\t"
+        "add.u32 ax8, %1, 8;\n\t"
+        "add.u32 ay8, %3, 8;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %5, %9, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d1, %9, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%4], d2, %9, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %5, %9, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %9, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%4], d2, %9, pt;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t"
+        "}" ::"r"(tDx),
+        "r"(tAx), "r"(tDy), "r"(tAy), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
+        "n"((uint64_t)(2 * U)), "n"(IDESC)
+        : "memory");
+}
+
 // predicated forms: every lane of the issuing warps executes the instruction
 // stream, only `pred != 0` issues (no divergent branch around the issue)
 __device__ __forceinline__ void mma_ts_p(uint32_t pred, uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc,
@@ -248,6 +279,37 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
           "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]),
           "=r"(r[30]), "=r"(r[31])
         : "r"(taddr)
+        : "memory");
+}
+// two 32-column loads (e.g. two tiles) with a single wait: the latencies overlap
+__device__ __forceinline__ void tmem_ld32x2(uint32_t ta, uint32_t tb, uint32_t (&a)[32], uint32_t (&b)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%64];\n\t"
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%32,%33,%34,%35,%36,%37,%38,%39,%40,%41,%42,%43,%44,%45,%46,%47,"
+        "%48,%49,%50,%51,%52,%53,%54,%55,%56,%57,%58,%59,%60,%61,%62,%63}, [%65];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(a[0]), "=r"(a[1]), "=r"(a[2]), "=r"(a[3]), "=r"(a[4]), "=r"(a[5]), "=r"(a[6]), "=r"(a[7]),
+          "=r"(a[8]), "=r"(a[9]), "=r"(a[10]), "=r"(a[11]), "=r"(a[12]), "=r"(a[13]), "=r"(a[14]), "=r"(a[15]),
+          "=r"(a[16]), "=r"(a[17]), "=r"(a[18]), "=r"(a[19]), "=r"(a[20]), "=r"(a[21]), "=r"(a[22]),
+          "=r"(a[23]), "=r"(a[24]), "=r"(a[25]), "=r"(a[26]), "=r"(a[27]), "=r"(a[28]), "=r"(a[29]),
+          "=r"(a[30]), "=r"(a[31]), "=r"(b[0]), "=r"(b[1]), "=r"(b[2]), "=r"(b[3]), "=r"(b[4]), "=r"(b[5]),
+          "=r"(b[6]), "=r"(b[7]), "=r"(b[8]), "=r"(b[9]), "=r"(b[10]), "=r"(b[11]), "=r"(b[12]), "=r"(b[13]),
+          "=r"(b[14]), "=r"(b[15]), "=r"(b[16]), "=r"(b[17]), "=r"(b[18]), "=r"(b[19]), "=r"(b[20]),
+          "=r"(b[21]), "=r"(b[22]), "=r"(b[23]), "=r"(b[24]), "=r"(b[25]), "=r"(b[26]), "=r"(b[27]),
+          "=r"(b[28]), "=r"(b[29]), "=r"(b[30]), "=r"(b[31])
+        : "r"(ta), "r"(tb)
+        : "memory");
+}
+__device__ __forceinline__ void tmem_ld1x2(uint32_t ta, uint32_t tb, uint32_t& a, uint32_t& b) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%2];\n\t"
+        "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%1}, [%3];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(a), "=r"(b)
+        : "r"(ta), "r"(tb)
         : "memory");
 }
 __device__ __forceinline__ void tmem_ld1(uint32_t taddr, uint32_t& r) {
