@@ -48,7 +48,8 @@ extern "C" {
 
 #define ABACUS_K_MAX 4
 #define ABACUS_HIDDEN 32
-#define ABACUS_ABI_VERSION 1
+#define ABACUS_ABI_VERSION 2
+#define ABACUS_BATCH_MAX (1 << 20) /* decisions per abacus_search_batch call */
 
 /* status codes */
 enum {
@@ -214,6 +215,21 @@ int abacus_select_group(abacus_ctx* ctx, const abacus_grid_t* grid, uint64_t fir
  * E_CUDA. */
 int abacus_search(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
                   int32_t space, uint64_t grid_budget, abacus_decision_t* out);
+
+/* Many independent scheduling rounds in one call (
+ * the paper runs one round at a time): decision i is exactly
+ * abacus_search(q + 4 i, k[i], now_ms[i], inflight_pred_ms[i], space,
+ * grid_budget).  q: host array of 4 n query records (decision i uses
+ * q[4i .. 4i + k[i] - 1]; the rest are ignored); k, now_ms,
+ * inflight_pred_ms: host arrays of n; out: host array of n decisions.
+ * 1 <= n <= ABACUS_BATCH_MAX.  fp16 / bf16: one batched tensor-core launch
+ * (plus a decode kernel) for all n; fp32: one fused launch per decision.
+ * The ctx grows its batch buffers on the first call with a larger n.
+ * Errors: as abacus_search (the message names the failing decision; no
+ * output is written on error). */
+int abacus_search_batch(abacus_ctx* ctx, const abacus_query_t* q, const int32_t* k, const double* now_ms,
+                        const double* inflight_pred_ms, int32_t n, int32_t space, uint64_t grid_budget,
+                        abacus_decision_t* out);
 
 /* The paper's multi-way search (§7.7)
  * for one scheduling round: same a1 step as abacus_search; candidates are the

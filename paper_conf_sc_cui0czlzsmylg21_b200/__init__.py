@@ -27,7 +27,7 @@ K_MAX = 4
 
 EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load_predictor",
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
-            "abacus_select_group", "abacus_search", "abacus_search_mway", "abacus_search_grid", "abacus_nccl_unique_id",
+            "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_nccl_unique_id",
             "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
             "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version"]
 
@@ -94,6 +94,8 @@ def lib():
         L.abacus_select_group.argtypes = [vp, P(abacus_grid_t), C.c_uint64, C.c_uint64, vp, C.c_float, vp, vp]
         L.abacus_search.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
                                     C.c_uint64, P(abacus_decision_t)]
+        L.abacus_search_batch.argtypes = [vp, P(abacus_query_t), P(C.c_int32), P(C.c_double), P(C.c_double),
+                                          C.c_int32, C.c_int32, C.c_uint64, P(abacus_decision_t)]
         L.abacus_search_mway.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
                                          P(abacus_decision_t), P(C.c_int32)]
         L.abacus_search_grid.argtypes = [vp, P(abacus_grid_t), C.c_float, C.c_uint64, C.c_uint64, vp,
@@ -206,6 +208,24 @@ def abacus_search(ctx, queries, now_ms: float, inflight_pred_ms: float, space: i
     _check(ctx, lib().abacus_search(ctx, qa, k, float(now_ms), float(inflight_pred_ms), space, grid_budget,
                                     C.byref(out)))
     return out
+
+
+def abacus_search_batch(ctx, decisions, space: int = ABACUS_SPACE_GRID, grid_budget: int = 2**40):
+    """decisions: sequence of (queries, now_ms, inflight_pred_ms); returns a list of decisions."""
+    n = len(decisions)
+    qa = (abacus_query_t * (4 * n))()
+    ka = (C.c_int32 * n)()
+    now = (C.c_double * n)()
+    inf = (C.c_double * n)()
+    for i, (queries, now_ms, inflight) in enumerate(decisions):
+        ka[i] = len(queries)
+        now[i] = float(now_ms)
+        inf[i] = float(inflight)
+        for j, q in enumerate(queries):
+            qa[4 * i + j] = abacus_query_t(q.model_id, q.next_op, q.batch, q.seqlen, q.qos_ms, q.t_start_ms)
+    out = (abacus_decision_t * n)()
+    _check(ctx, lib().abacus_search_batch(ctx, qa, ka, now, inf, n, space, grid_budget, out))
+    return list(out)
 
 
 def abacus_search_mway(ctx, queries, now_ms: float, inflight_pred_ms: float, ways: int):

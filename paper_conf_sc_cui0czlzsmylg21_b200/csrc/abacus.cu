@@ -51,6 +51,18 @@ struct abacus_ctx {
     W234 w234{};
     uint8_t* d_blob[2] = {nullptr, nullptr};  // tensor-core weight blobs (fp16, bf16)
     TcWeights tw[2]{};
+    // batched decisions: staging and device buffers, grown on demand (first call of a larger batch)
+    int32_t batch_cap = 0;
+    BatchDec* h_decs = nullptr;  // pinned
+    SegP* h_segs = nullptr;      // pinned, kMaxSegBatch per decision
+    Result* h_out = nullptr;     // pinned
+    BatchDec* d_decs = nullptr;
+    SegP* d_segs = nullptr;
+    BatchAcc* d_acc = nullptr;
+    float* d_y0 = nullptr;
+    Result* d_out = nullptr;
+    std::vector<int32_t> b_order;  // [4 n] headroom order per decision
+    std::vector<float> b_H;
 };
 
 namespace {
@@ -605,6 +617,67 @@ unsigned long long* trace_ptr() { return g_trace_ptr; }
 // ============================================================================
 // C ABI
 // ============================================================================
+namespace {
+int grow_batch(abacus_ctx* c, int32_t n) {
+    if (n <= c->batch_cap) return ABACUS_OK;
+    int32_t cap = c->batch_cap ? c->batch_cap : 256;
+    while (cap < n) cap *= 2;
+    if (c->h_decs) cudaFreeHost(c->h_decs);
+    if (c->h_segs) cudaFreeHost(c->h_segs);
+    if (c->h_out) cudaFreeHost(c->h_out);
+    cudaFree(c->d_decs);
+    cudaFree(c->d_segs);
+    cudaFree(c->d_acc);
+    cudaFree(c->d_y0);
+    cudaFree(c->d_out);
+    c->h_decs = nullptr;
+    c->h_segs = nullptr;
+    c->h_out = nullptr;
+    c->d_decs = nullptr;
+    c->d_segs = nullptr;
+    c->d_acc = nullptr;
+    c->d_y0 = nullptr;
+    c->d_out = nullptr;
+    c->batch_cap = 0;
+    const size_t nd = (size_t)cap, ns = (size_t)cap * kMaxSegBatch;
+    CUDA_TRY(c, cudaHostAlloc(&c->h_decs, nd * sizeof(BatchDec), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_segs, ns * sizeof(SegP), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_out, nd * sizeof(Result), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaMalloc(&c->d_decs, nd * sizeof(BatchDec)));
+    CUDA_TRY(c, cudaMalloc(&c->d_segs, ns * sizeof(SegP)));
+    CUDA_TRY(c, cudaMalloc(&c->d_acc, nd * sizeof(BatchAcc)));
+    CUDA_TRY(c, cudaMalloc(&c->d_y0, nd * sizeof(float)));
+    CUDA_TRY(c, cudaMalloc(&c->d_out, nd * sizeof(Result)));
+    c->b_order.resize(4 * nd);
+    c->b_H.resize(nd);
+    c->batch_cap = cap;
+    return ABACUS_OK;
+}
+
+// a7 for one decision from its result record (shared by the single and batched searches)
+abacus_decision_t assemble_decision(const Result& R, const int32_t* order, int32_t k, float H, uint64_t n_eval) {
+    abacus_decision_t d{};
+    d.critical = order[0];
+    for (int j = 0; j < 4; j++) d.order[j] = j < k ? order[j] : -1;
+    d.headroom_ms = H;
+    d.pred_critical_only_ms = R.y0;
+    d.evaluated = n_eval;
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    if (!(R.y0 <= H)) {  // drop mechanism (P:1293-1298)
+        d.status = ABACUS_DECIDE_DROP;
+        d.pred_ms = R.y0;
+        d.total_ops = 0;
+    } else {
+        d.status = ABACUS_DECIDE_OK;
+        d.pred_ms = R.y_best;
+        d.total_ops = R.total_ops;
+        for (int j = 0; j < k; j++) d.end_op[order[j]] = R.end_op[j];
+    }
+    return d;
+}
+}  // namespace
+
 extern "C" {
 
 int abacus_abi_version(void) { return ABACUS_ABI_VERSION; }
@@ -656,6 +729,14 @@ void abacus_destroy(abacus_ctx* c) {
     cudaFree(c->d_blob[0]);
     cudaFree(c->d_blob[1]);
     if (c->host_result) cudaFreeHost(c->host_result);
+    if (c->h_decs) cudaFreeHost(c->h_decs);
+    if (c->h_segs) cudaFreeHost(c->h_segs);
+    if (c->h_out) cudaFreeHost(c->h_out);
+    cudaFree(c->d_decs);
+    cudaFree(c->d_segs);
+    cudaFree(c->d_acc);
+    cudaFree(c->d_y0);
+    cudaFree(c->d_out);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->own_stream) cudaStreamDestroy(c->own_stream);
@@ -820,27 +901,81 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
     if (rc) return rc;
     rc = wait_result(c, P.seq);
     if (rc) return rc;
-    const Result R = *c->host_result;
-    // a7: decision assembly
-    abacus_decision_t d{};
-    d.critical = order[0];
-    for (int j = 0; j < 4; j++) d.order[j] = j < k ? order[j] : -1;
-    d.headroom_ms = H;
-    d.pred_critical_only_ms = R.y0;
-    d.evaluated = n_eval;
-    d.key = R.key;
-    d.index = R.key & ((1ull << 40) - 1);
-    if (!(R.y0 <= H)) {  // drop mechanism (P:1293-1298)
-        d.status = ABACUS_DECIDE_DROP;
-        d.pred_ms = R.y0;
-        d.total_ops = 0;
-    } else {
-        d.status = ABACUS_DECIDE_OK;
-        d.pred_ms = R.y_best;
-        d.total_ops = R.total_ops;
-        for (int j = 0; j < k; j++) d.end_op[order[j]] = R.end_op[j];
+    *out = assemble_decision(*c->host_result, order, k, H, n_eval);
+    return ABACUS_OK;
+}
+
+
+int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k, const double* now_ms,
+                        const double* inflight_pred_ms, int32_t n, int32_t space, uint64_t grid_budget,
+                        abacus_decision_t* out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!q || !k || !now_ms || !inflight_pred_ms || !out) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (n < 1 || n > ABACUS_BATCH_MAX) return fail(c, ABACUS_E_INVALID, "n=%d outside [1,%d]", n, ABACUS_BATCH_MAX);
+    if (space < ABACUS_SPACE_GRID || space > ABACUS_SPACE_AUTO) return fail(c, ABACUS_E_INVALID, "bad space");
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (c->precision == ABACUS_FP32) {
+        // the fp32 SIMT path has no batched kernel: one fused launch per decision
+        for (int32_t i = 0; i < n; i++) {
+            const int rc = abacus_search(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], space,
+                                         grid_budget, &out[i]);
+            if (rc) return rc;
+        }
+        return ABACUS_OK;
     }
-    *out = d;
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    int rc = grow_batch(c, n);
+    if (rc) return rc;
+    uint64_t pair = 0;
+    uint32_t seg = 0, maxcnt = 0;
+    for (int32_t i = 0; i < n; i++) {
+        int32_t* order = &c->b_order[4 * (size_t)i];
+        abacus_grid_t g{};
+        rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], order, &c->b_H[i], &g);
+        if (rc) {
+            c->err = "decision " + std::to_string(i) + ": " + c->err;
+            return rc;
+        }
+        uint64_t T = 0;
+        validate_grid(c, &g, &T);
+        const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
+        uint64_t n_eval = 0;
+        Plan P = chain ? plan_chain(c, &g, c->b_H[i], &n_eval) : plan_grid_segments(c, &g, T, 0, T, c->b_H[i]);
+        if (!chain) n_eval = P.n_eval;
+        if (P.n_seg > kMaxSegBatch) return fail(c, ABACUS_E_INVALID, "decision %d: %d segments", i, P.n_seg);
+        BatchDec& bd = c->h_decs[i];
+        bd.h = static_cast<const PlanHdr&>(P);
+        bd.h.want_y0 = 1;
+        bd.h.n_eval = n_eval;
+        bd.h.mapped = nullptr;
+        bd.h.trace = nullptr;
+        bd.pair0 = pair;
+        bd.seg0 = seg;
+        for (int s = 0; s < P.n_seg; s++) {
+            c->h_segs[seg + s] = P.seg[s];
+            for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
+        }
+        seg += (uint32_t)P.n_seg;
+        pair += (P.n_tiles + 1) / 2;
+    }
+    cudaStream_t st = c->stream;
+    CUDA_TRY(c, cudaMemcpyAsync(c->d_decs, c->h_decs, (size_t)n * sizeof(BatchDec), cudaMemcpyHostToDevice, st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->d_segs, c->h_segs, (size_t)seg * sizeof(SegP), cudaMemcpyHostToDevice, st));
+    CUDA_TRY(c, cudaMemsetAsync(c->d_acc, 0, (size_t)n * sizeof(BatchAcc), st));
+    CUDA_TRY(c, cudaMemsetAsync(c->d_y0, 0xFF, (size_t)n * sizeof(float), st));  // NaN
+    if (c->timed) cudaEventRecord(c->ev0, st);
+    const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
+    cudaError_t e = launch_batch_tc(c->d_decs, c->d_segs, n, pair, maxcnt, c->D, c->tw[fmt], c->d_w1b1, c->d_acc,
+                                    c->d_y0, c->d_out, c->nsm, st);
+    if (c->timed) cudaEventRecord(c->ev1, st);
+    if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "batched search launch: %s", cudaGetErrorString(e));
+    c->launches += 2;
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_out, c->d_out, (size_t)n * sizeof(Result), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(c, cudaStreamSynchronize(st));
+    for (int32_t i = 0; i < n; i++)
+        out[i] = assemble_decision(c->h_out[i], &c->b_order[4 * (size_t)i], k[i], c->b_H[i],
+                                   c->h_decs[i].h.n_eval);
     return ABACUS_OK;
 }
 

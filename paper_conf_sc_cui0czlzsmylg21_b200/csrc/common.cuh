@@ -70,7 +70,8 @@ struct Result {
 
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
 
-struct Plan {
+// header of a plan: everything but the segment table (decode of t*, a7)
+struct PlanHdr {
     int32_t k, n_seg, n_models, D;
     int32_t mode;           // kModeGrid (t) or kModeChain (u)
     int32_t want_y0;        // 1 if index 0 is in range (decision drop test)
@@ -85,7 +86,28 @@ struct Plan {
     uint32_t seq;           // sequence number the mapped copy is tagged with
     uint32_t pad2;
     SlotP slot[kKMax];
+};
+
+struct Plan : PlanHdr {
     SegP seg[kMaxSeg];
+};
+
+// ---- batched decisions (NEXT-4): many independent decisions in one launch ----
+// Decision d owns tiles [2 pair0, 2 pair0 + n_tiles) of the launch (n_tiles
+// rounded up to even, so a group's two lock-step tiles never straddle two
+// decisions); its segments are segs[seg0 .. seg0 + h.n_seg).
+constexpr int kMaxSegBatch = 8;  // decision mode: <= 2^(k-1) presence patterns
+struct BatchDec {
+    PlanHdr h;
+    uint64_t pair0;
+    uint32_t seg0;
+    uint32_t pad;
+};
+// per-decision running result, updated with a 128-bit compare-and-swap
+struct __align__(16) BatchAcc {
+    unsigned long long key;
+    float y;   // y(t*) of the key
+    float y0;  // y(index 0), written by the owner of the decision's first row
 };
 
 struct Scratch {             // device scratch owned by the ctx

@@ -158,7 +158,7 @@ __device__ __forceinline__ unsigned long long div_rcp(unsigned long long a, unsi
 // End op of slot `j` of the candidate with index idx (GRID: digit j of the
 // mixed-radix index, computed directly so lanes can decode slots in parallel;
 // CHAIN: block structure).  0 = absent.
-__device__ __forceinline__ int32_t decode_slot_ope(const Plan& P, unsigned long long idx, int j) {
+__device__ __forceinline__ int32_t decode_slot_ope(const PlanHdr& P, unsigned long long idx, int j) {
     if (P.mode == kModeGrid) {
         const SlotP& s = P.slot[j];
         const unsigned long long q = div_rcp(idx, s.tstride, s.rtstride);
@@ -174,7 +174,7 @@ __device__ __forceinline__ int32_t decode_slot_ope(const Plan& P, unsigned long 
 }
 
 // optional timeline stamps (CTA 0, thread 0): tools/kernel_trace.py
-__device__ __forceinline__ void trace_stamp(const Plan& P, int slot) {
+__device__ __forceinline__ void trace_stamp(const PlanHdr& P, int slot) {
     if (P.trace && blockIdx.x == 0 && threadIdx.x == 0) {
         unsigned long long t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

@@ -45,6 +45,10 @@ cudaError_t launch_finalize_gather(Scratch* S, int nranks, Result* mapped, uint3
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out);
+// batched decisions: d_decs[n_dec] and d_segs on the device; acc/y0s zeroed / NaN-filled by the caller
+cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, uint64_t n_pairs,
+                            uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1, BatchAcc* acc,
+                            float* y0s, Result* out, int nsm, cudaStream_t st);
 cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
                               float* y, int nsm, cudaStream_t st);
 

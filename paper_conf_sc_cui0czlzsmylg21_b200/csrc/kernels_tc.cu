@@ -65,11 +65,12 @@ __device__ __forceinline__ void split16(float v, uint16_t& hi, uint16_t& lo) {
 // c = b1 + W1 x0 (Fig.-8 vector of the segment's v = 0 group), w_j = the
 // W1 column of slot j's ope at its Fig.-8 position.
 template <int FMT, bool SPLIT>
-__device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, float scale, uint8_t* s_b1) {
+__device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, float scale, uint8_t* s_b1, int t0,
+                               int nt) {
     constexpr int NCH = TcCfg<FMT>::kNchL1;
     const int D = P.D;
     const float* b1 = w1b1 + kHidden * D;
-    for (int e = threadIdx.x; e < P.n_seg * kHidden; e += blockDim.x) {
+    for (int e = t0; e < P.n_seg * kHidden; e += nt) {
         const int s = e / kHidden, n = e % kHidden;
         const SegP& g = P.seg[s];
         const float* w = w1b1 + n * D;
@@ -220,11 +221,14 @@ __host__ __device__ inline uint32_t w1_stage_bytes(int D, int ng) {
 // ---------------------------------------------------------------------------
 // fused search
 //
-// Each group keeps TWO tiles in flight (TMEM slots X and Y) and interleaves
-// them stage by stage: while the tensor core runs layer l of one tile, the
-// group's warps run the epilogue of the other.  Per group TMEM (128 columns):
-//   X: D [0,32)  A1 [32,40)  A [40,56)     Y: D [64,96)  A1 [96,104)  A [104,120)
-//   constant chunk [56,64) = (1, 1, 0, ...) for the bias columns
+// A group (4 warps = the 128 TMEM lanes, warp q reaching lanes 32q..32q+31)
+// keeps TWO tiles in flight (TMEM slots X and Y) that move through the layers
+// in lock step: one MMA commit covers both, so a stage costs one mbarrier
+// wait, two overlapped tcgen05.ld, one tcgen05.st wait and one hand-off for
+// two tiles, while the CTA's other groups keep the tensor pipe fed.
+// Per group 96 TMEM columns: D_X [0,32) D_Y [32,64) A_X [64,80) A_Y [80,96);
+// the layer-1 operand A1 aliases the first 8 columns of A.  One constant
+// chunk (1, 1, 0, ...) at column 480 supplies the bias rows of every B operand.
 // ---------------------------------------------------------------------------
 struct TileIO {
     uint32_t d, a1, a;  // TMEM addresses (column part; lane 0)
@@ -246,129 +250,64 @@ __device__ __forceinline__ void store_a1(uint32_t taddr, const uint32_t (&v)[kKM
     tmem_st8(taddr, a);
 }
 
-// output layer in fp32 on the SIMT pipes: y = b4 + sum_j w4s_j relu(z3_j)
-// (w4s = w4 * 2^s3 undoes the fp16 layer scaling; kernel parameter -> FFMA
-// with a constant-bank operand)
-struct OutW {
-    float w4s[kHidden];
-    float b4;
-};
+// The MMA pipeline of one group.  Operand hand-off: after writing its 32 rows
+// a warp fences its tcgen05.st and ARRIVES on the group's named barrier
+// without blocking; only the stage's issuing warp SYNCs (waits for all 128
+// threads), then issues the MMAs from one elected lane and commits them to the
+// group's mbarrier.  The issuer rotates over the group's 4 warps (one per
+// SMSP): hand-off position p = 0 (issue layer 2), 1 (layer 3), 2 (output),
+// 3 (layer 1 of the next tiles).
+template <int FMT>
+struct TcPipe {
+    TileIO X, Y;
+    uint32_t tC, lane_off, bar_id, ph;
+    uint64_t* bar;
+    uint64_t db2, db3, db4;
+    bool me[4];
 
-__device__ __forceinline__ float output_dot(uint32_t tD_lane, const OutW& O) {
-    uint32_t z[32];
-    tmem_ld32(tD_lane, z);
-    float acc0 = O.b4, acc1 = 0.0f;
+    __device__ __forceinline__ void init(uint32_t tbase, int g, int wq, uint64_t* mbar, uint64_t d2, uint64_t d3,
+                                         uint64_t d4) {
+        const uint32_t col = tbase + (uint32_t)g * 96u;
+        X = TileIO{col + 0, col + 64, col + 64};
+        Y = TileIO{col + 32, col + 80, col + 80};
+        tC = tbase + 480;
+        lane_off = (uint32_t)(wq * 32) << 16;
+        bar_id = 1 + (uint32_t)g;
+        ph = 0;
+        bar = mbar;
+        db2 = d2;
+        db3 = d3;
+        db4 = d4;
 #pragma unroll
-    for (int j = 0; j < kHidden; j += 2) {
-        acc0 = fmaf(O.w4s[j], fmaxf(__uint_as_float(z[j]), 0.0f), acc0);
-        acc1 = fmaf(O.w4s[j + 1], fmaxf(__uint_as_float(z[j + 1]), 0.0f), acc1);
+        for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
     }
-    return acc0 + acc1;
-}
-
-template <int FMT, bool SPLIT, int NG, bool TRACE>
-__global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
-                                                               const __grid_constant__ TcParams TP,
-                                                               const __grid_constant__ OutW O,
-                                                               const float* __restrict__ w1b1, Scratch* S) {
-    extern __shared__ __align__(1024) uint8_t smem[];
-    using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * NG, w1_stage_bytes(P.D, 2 * NG));
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);  // 2 per group
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
-
-    const int tid = threadIdx.x;
-    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform for the compiler
-    const int g = warp >> 2, wq = warp & 3;
-    trace_stamp(P, 0);
-
-    {
-        const int4* src = reinterpret_cast<const int4*>(TP.blob);
-        int4* dst = reinterpret_cast<int4*>(smem);
-        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
-        // stage W1 | b1 (fp32) for the layer-1 table build
-        float* s_w1 = reinterpret_cast<float*>(smem + L.stage);
-        for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
-    }
-    __syncthreads();
-    trace_stamp(P, 1);
-    build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1);
-    if (tid == 0) {
-        for (int i = 0; i < 2 * NG; i++) mbar_init(&bars[i], 1);
-        mbar_fence_init();
-    }
-    if (warp == 0) {
-        tmem_alloc(tmem_slot, 512);
-        tmem_relinquish();
-    }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    fence_before();
-    __syncthreads();
-    fence_after();
-    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
-    trace_stamp(P, 2);
-
-    // TMEM: group g owns 96 columns at 96 g: D_X [0,32) D_Y [32,64) A_X [64,80)
-    // A_Y [80,96); the layer-1 operand A1 aliases the first 8 columns of A.
-    // One constant chunk (1, 1, 0, ...) for the bias columns at 480.
-    const uint32_t col = tbase + (uint32_t)g * 96u;
-    const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-    const TileIO X{col + 0, col + 64, col + 64}, Y{col + 32, col + 80, col + 80};
-    const uint32_t tC = tbase + 480;
-    if (g == 0) {
-        uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
-        tmem_st8(tC + lane_off, c8);
-        tmem_wait_st();
-    }
-    fence_before();
-    __syncthreads();
-    fence_after();
-    const uint32_t r = (uint32_t)(tid & 127);
-    const uint32_t sbase = smem_u32(smem);
-    constexpr uint32_t id32 = idesc_f16(FMT, 32);
-    constexpr uint32_t id16 = idesc_f16(FMT, 16);
-    uint64_t* bar = &bars[g];
-    uint32_t ph = 0;
-    const uint64_t db2 = smem_desc(sbase + L.w2), db3 = smem_desc(sbase + L.w3), db4 = smem_desc(sbase + L.w4);
-    const uint64_t d1base = smem_desc(sbase + L.b1);
-    constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
-
-    // The group's two tiles (slots X and Y) move through the layers in lock
-    // step: one MMA commit covers both, so each stage costs ONE mbarrier wait,
-    // two overlapped TMEM loads, one tcgen05.st wait and ONE hand-off for two
-    // tiles; the other groups of the CTA keep the tensor pipe busy meanwhile.
-    // Operand hand-off: after writing its 32 rows a warp fences its tcgen05.st
-    // and ARRIVES on the group's named barrier without blocking; only the
-    // stage's issuing warp SYNCs (waits for all 128 threads), then issues the
-    // MMAs from one elected lane and commits them to the group's mbarrier.
-    // The issuer rotates over the group's 4 warps (one per SMSP) stage by stage.
-    const uint32_t bar_id = 1 + g;
-    auto handoff = [&](bool me) -> bool {
+    __device__ __forceinline__ bool handoff(bool mine) const {
         fence_before();
-        if (me) {
+        if (mine) {
             named_bar_sync(bar_id, 128);
             fence_after();
         } else {
             named_bar_arrive(bar_id, 128);
         }
-        return me;
-    };
-    // issuer of hand-off position p (0: L2, 1: L3, 2: out, 3: next L1)
-    bool me[4];
-#pragma unroll
-    for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
-    auto issue_l1 = [&](const TileIO& T, int s) {
-        const int su = __shfl_sync(0xffffffffu, s, 0);
-        const uint64_t db = d1base + (uint64_t)((uint32_t)su * kSegStep);
+        return mine;
+    }
+    __device__ __forceinline__ void wait() {
+        mbar_wait(bar, ph);
+        ph ^= 1u;
+        fence_after();
+    }
+    // layer-1 MMA(s) of one tile against its segment's B operand (no commit)
+    __device__ __forceinline__ void issue_l1(const TileIO& T, uint64_t db) const {
+        constexpr uint32_t id32 = idesc_f16(FMT, 32);
         mma_ts_elect(T.d, T.a1, db, id32, 0u);
-        if (C::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
-    };
+        if (TcCfg<FMT>::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
+    }
+    __device__ __forceinline__ void commit() const { mma_commit_elect(bar); }
     // layer LAYER (0: layer 2, 1: layer 3, 2: output) of X (and Y), one commit
-    auto issue_next = [&](auto layer_c, auto two_c) {
-        constexpr int LAYER = decltype(layer_c)::value;
-        constexpr bool TWO = decltype(two_c)::value;
+    template <int LAYER, bool TWO>
+    __device__ __forceinline__ void issue_next() const {
         constexpr uint32_t CH = LAYER == 2 ? kChunkBytesN16 : kChunkBytesN32;
-        constexpr uint32_t ID = LAYER == 2 ? id16 : id32;
+        constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 0 && TWO) {
             issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tC, db, bar);
@@ -382,32 +321,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             issue_layer_e<FMT>(Y.d, Y.a, tC, d, ID);
             mma_commit_elect(bar);
         }
-    };
-    // debug timeline (tools/stage_trace.py): CTA 0, group 0, lane 0 of each warp, 12 stages
-    const bool tr = TRACE && P.trace != nullptr && blockIdx.x == 0 && g == 0 && (tid & 31) == 0;
-    int trn = 0;
-    constexpr int kTr0 = 40;  // first traced stage (steady state)
-    auto tstamp = [&](int slot) {
-        if (TRACE && tr && trn >= kTr0 && trn < kTr0 + 12) {
-            long long c;
-            asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
-            P.trace[16 + (wq * 12 + trn - kTr0) * 6 + slot] = (unsigned long long)c;
-        }
-    };
-    auto tnext = [&](bool mine) {
-        if (TRACE && tr) {
-            if (trn >= kTr0 && trn < kTr0 + 12) P.trace[16 + (wq * 12 + trn - kTr0) * 6 + 5] = mine ? 1ull : 0ull;
-            trn++;
-        }
-    };
-    // wait for layer LAYER-1's MMAs, epilogue (ReLU, pack) into A, hand off, issue layer LAYER
-    auto stage = [&](auto layer_c, auto two_c) {
-        constexpr bool TWO = decltype(two_c)::value;
-        tstamp(0);
-        mbar_wait(bar, ph);
-        ph ^= 1u;
-        fence_after();
-        tstamp(1);
+    }
+    // wait for the previous layer's MMAs, ReLU + pack into A, hand off, issue layer LAYER
+    template <int LAYER, bool TWO>
+    __device__ __forceinline__ void stage() {
+        wait();
         if (TWO) {
             uint32_t a[32], b[32], h[16];
             tmem_ld32x2(X.d + lane_off, Y.d + lane_off, a, b);
@@ -421,16 +339,87 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         } else {
             hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
         }
-        tstamp(2);
-        const bool mine = handoff(me[decltype(layer_c)::value]);
-        tstamp(3);
-        if (mine) issue_next(layer_c, two_c);
-        tstamp(4);
-        tnext(mine);
+        if (handoff(me[LAYER])) issue_next<LAYER, TWO>();
+    }
+    // the three hidden stages, then wait for the output MMA and read y (column 0 of D)
+    template <bool TWO>
+    __device__ __forceinline__ void run_layers(uint32_t& yx, uint32_t& yy) {
+        stage<0, TWO>();
+        stage<1, TWO>();
+        stage<2, TWO>();
+        wait();
+        if (TWO) tmem_ld1x2(X.d + lane_off, Y.d + lane_off, yx, yy);
+        else tmem_ld1(X.d + lane_off, yx);
+    }
+};
+
+// CTA prologue common to both fused kernels: weights -> smem, mbarriers,
+// TMEM allocation, the constant chunk
+template <int FMT, int NG>
+__device__ __forceinline__ uint32_t fused_prologue_tmem(uint64_t* bars, uint32_t* tmem_slot, int warp, int g, int wq) {
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        mbar_fence_init();
+    }
+    if (warp == 0) {
+        tmem_alloc(tmem_slot, 512);
+        tmem_relinquish();
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
+    if (g == 0) {
+        uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
+        tmem_st8(tbase + 480 + ((uint32_t)(wq * 32) << 16), c8);
+        tmem_wait_st();
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    return tbase;
+}
+
+template <int FMT, bool SPLIT, int NG>
+__global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
+                                                               const __grid_constant__ TcParams TP,
+                                                               const float* __restrict__ w1b1, Scratch* S) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    using C = TcCfg<FMT>;
+    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, NG, w1_stage_bytes(P.D, NG));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);  // one per group
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
+
+    const int tid = threadIdx.x;
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform for the compiler
+    const int g = warp >> 2, wq = warp & 3;
+    trace_stamp(P, 0);
+    {
+        const int4* src = reinterpret_cast<const int4*>(TP.blob);
+        int4* dst = reinterpret_cast<int4*>(smem);
+        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+        // stage W1 | b1 (fp32) for the layer-1 table build
+        float* s_w1 = reinterpret_cast<float*>(smem + L.stage);
+        for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
+    }
+    __syncthreads();
+    trace_stamp(P, 1);
+    build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
+                               blockDim.x);
+    const uint32_t tbase = fused_prologue_tmem<FMT, NG>(bars, tmem_slot, warp, g, wq);
+    trace_stamp(P, 2);
+
+    const uint32_t r = (uint32_t)(tid & 127);
+    const uint32_t sbase = smem_u32(smem);
+    TcPipe<FMT> pp;
+    pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    const uint64_t d1base = smem_desc(sbase + L.b1);
+    constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
+    auto issue_l1 = [&](const TileIO& T, int s) {
+        const int su = __shfl_sync(0xffffffffu, s, 0);
+        pp.issue_l1(T, d1base + (uint64_t)((uint32_t)su * kSegStep));
     };
-    using L0 = std::integral_constant<int, 0>;
-    using L1 = std::integral_constant<int, 1>;
-    using L2 = std::integral_constant<int, 2>;
     using T1 = std::integral_constant<bool, false>;
     using T2 = std::integral_constant<bool, true>;
 
@@ -459,19 +448,18 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         // prologue: tile wb in slot X and (if the group has it) wb + 1 in slot Y
         const bool yLive = wb + 1 < we;  // warp-uniform
         take(vX, sX, okX, zX);
-        store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
+        store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
         if (yLive) {
             walker_next(P, W, wb + 1, r);
             take(vY, sY, okY, zY);
-            store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+            store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
         }
         tmem_wait_st();
-        if (handoff(me[3])) {
-            issue_l1(X, sX);
-            if (yLive) issue_l1(Y, sY);
-            mma_commit_elect(bar);
+        if (pp.handoff(pp.me[3])) {
+            issue_l1(pp.X, sX);
+            if (yLive) issue_l1(pp.Y, sY);
+            pp.commit();
         }
-
         // one iteration = layers 2, 3, out of the tiles in X (and Y), fold (a5),
         // then tiles w + 2 (and w + 3) enter the slots.  The steady state has
         // both slots full before and after; the tail handles a lone X.
@@ -479,42 +467,25 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         auto iteration = [&](auto two_c, auto next_two_c) {
             constexpr bool TWO = decltype(two_c)::value;
             constexpr bool NTWO = decltype(next_two_c)::value;
-            stage(L0{}, two_c);
-            stage(L1{}, two_c);
-            stage(L2{}, two_c);
-            tstamp(0);
-            mbar_wait(bar, ph);
-            ph ^= 1u;
-            fence_after();
-            tstamp(1);
             uint32_t ybx, yby = 0;
-            if (TWO) {
-                tmem_ld1x2(X.d + lane_off, Y.d + lane_off, ybx, yby);
-            } else {
-                tmem_ld1(X.d + lane_off, ybx);
-            }
+            pp.template run_layers<TWO>(ybx, yby);
             fold(ybx, sX, vX, okX, zX);
             if (TWO) fold(yby, sY, vY, okY, zY);
-            tstamp(2);
             if (w + 2 < we) {
                 walker_next(P, W, w + 2, r);
                 take(vX, sX, okX, zX);
-                store_a1<FMT, SPLIT>(X.a1 + lane_off, vX);
+                store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
                 if (NTWO) {
                     walker_next(P, W, w + 3, r);
                     take(vY, sY, okY, zY);
-                    store_a1<FMT, SPLIT>(Y.a1 + lane_off, vY);
+                    store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
                 }
                 tmem_wait_st();
-                tstamp(3);
-                const bool mine = handoff(me[3]);
-                if (mine) {
-                    issue_l1(X, sX);
-                    if (NTWO) issue_l1(Y, sY);
-                    mma_commit_elect(bar);
+                if (pp.handoff(pp.me[3])) {
+                    issue_l1(pp.X, sX);
+                    if (NTWO) issue_l1(pp.Y, sY);
+                    pp.commit();
                 }
-                tstamp(4);
-                tnext(mine);
             }
             w += 2;
         };
@@ -529,6 +500,219 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     if (warp == 0) tmem_dealloc(tbase, 512);
     trace_stamp(P, 4);
     cta_publish_and_finish(P, S, best, best_y);
+}
+
+// ---------------------------------------------------------------------------
+// batched decisions (NEXT-4): one launch searches many independent decisions.
+// The launch's tile PAIRS are split contiguously over all groups; a group
+// walks its pairs decision by decision.  On entering a decision it copies the
+// decision's plan (header + segments) into its own shared-memory slot and
+// builds that decision's layer-1 B operands into its own table region (all
+// of the group's MMAs have completed at that point), so the five groups of a
+// CTA can be in five different decisions.  On leaving a decision it folds its
+// best (key, y) into the decision's accumulator with a 128-bit CAS.
+// ---------------------------------------------------------------------------
+constexpr uint32_t kPlanBatchBytes =
+    (uint32_t)((sizeof(Plan) - kMaxSeg * sizeof(SegP) + kMaxSegBatch * sizeof(SegP) + 15) & ~size_t(15));
+
+__device__ __forceinline__ void acc_fold(BatchAcc* a, unsigned long long key, float y) {
+    unsigned long long ok = a->key, oy = __float_as_uint(a->y);
+    while (key > ok) {
+        unsigned long long rk, ry;
+        const unsigned long long ny = __float_as_uint(y);
+        asm volatile(
+            "{\n\t"
+            ".reg .b128 d, c, n;\n\t"
+            "mov.b128 c, {%2, %3};\n\t"
+            "mov.b128 n, {%4, %5};\n\t"
+            "atom.global.cas.b128 d, [%6], c, n;\n\t"
+            "mov.b128 {%0, %1}, d;\n\t"
+            "}"
+            : "=l"(rk), "=l"(ry)
+            : "l"(ok), "l"(oy), "l"(key), "l"(ny), "l"(a)
+            : "memory");
+        if (rk == ok && ry == oy) return;
+        ok = rk;
+        oy = ry;
+    }
+}
+
+template <int FMT>
+__host__ __device__ inline TcSmem batch_smem_layout(int D, int ng, uint32_t* plans_off) {
+    TcSmem L = tc_smem_layout<FMT>(ng * kMaxSegBatch, TcCfg<FMT>::kNchL1 * kChunkBytesN32, ng,
+                                   w1_stage_bytes(D, ng));
+    *plans_off = (L.total + 15u) & ~15u;
+    L.total = *plans_off + (uint32_t)ng * kPlanBatchBytes;
+    return L;
+}
+
+template <int FMT, bool SPLIT, int NG>
+__global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const BatchDec* __restrict__ decs,
+                                                                     const SegP* __restrict__ segs, int32_t n_dec,
+                                                                     uint64_t n_pairs, int32_t D,
+                                                                     const __grid_constant__ TcParams TP,
+                                                                     const float* __restrict__ w1b1, BatchAcc* acc,
+                                                                     float* y0s) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    using C = TcCfg<FMT>;
+    uint32_t plans_off;
+    const TcSmem L = batch_smem_layout<FMT>(D, NG, &plans_off);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
+    const int tid = threadIdx.x;
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+    const int g = warp >> 2, wq = warp & 3;
+    const float* s_w1 = reinterpret_cast<const float*>(smem + L.stage);
+    {
+        const int4* src = reinterpret_cast<const int4*>(TP.blob);
+        int4* dst = reinterpret_cast<int4*>(smem);
+        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+        float* w = reinterpret_cast<float*>(smem + L.stage);
+        for (int i = tid; i < kHidden * D + kHidden; i += blockDim.x) w[i] = __ldg(w1b1 + i);
+    }
+    __syncthreads();
+    const uint32_t tbase = fused_prologue_tmem<FMT, NG>(bars, tmem_slot, warp, g, wq);
+
+    const uint32_t r = (uint32_t)(tid & 127);
+    const uint32_t sbase = smem_u32(smem);
+    TcPipe<FMT> pp;
+    pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    constexpr uint32_t kTable = C::kNchL1 * kChunkBytesN32;
+    uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegBatch * kTable;
+    const uint64_t d1base = smem_desc(sbase + L.b1 + (uint32_t)g * kMaxSegBatch * kTable);
+    constexpr uint32_t kSegStep = kTable >> 4;
+    Plan& P = *reinterpret_cast<Plan*>(smem + plans_off + (size_t)g * kPlanBatchBytes);
+    auto issue_l1 = [&](const TileIO& T, int s) {
+        const int su = __shfl_sync(0xffffffffu, s, 0);
+        pp.issue_l1(T, d1base + (uint64_t)((uint32_t)su * kSegStep));
+    };
+
+    uint64_t pb, pe;
+    work_range(n_pairs, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, pb, pe);
+    if (pb < pe) {
+        // decision holding pair pb: the last d with pair0 <= pb
+        int d = 0;
+        {
+            int lo = 0, hi = n_dec - 1;
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (decs[mid].pair0 <= pb) lo = mid;
+                else hi = mid - 1;
+            }
+            d = lo;
+        }
+        uint64_t dec_pair0 = 0, dec_pair_end = 0;
+        // plan + layer-1 tables of decision d into this group's slots
+        auto load_decision = [&]() {
+            named_bar_sync(pp.bar_id, 128);  // every warp is done with the previous plan
+            const BatchDec& bd = decs[d];
+            const int n_seg = bd.h.n_seg;
+            const uint32_t* src = reinterpret_cast<const uint32_t*>(&bd.h);
+            uint32_t* dst = reinterpret_cast<uint32_t*>(&P);
+            for (uint32_t i = r; i < sizeof(PlanHdr) / 4; i += 128) dst[i] = src[i];
+            const uint32_t* ss = reinterpret_cast<const uint32_t*>(segs + bd.seg0);
+            uint32_t* sd = reinterpret_cast<uint32_t*>(&P.seg[0]);
+            for (uint32_t i = r; i < (uint32_t)n_seg * (sizeof(SegP) / 4); i += 128) sd[i] = ss[i];
+            dec_pair0 = bd.pair0;
+            dec_pair_end = d + 1 < n_dec ? decs[d + 1].pair0 : n_pairs;
+            named_bar_sync(pp.bar_id, 128);
+            build_b1_fused<FMT, SPLIT>(P, s_w1, TP.l1_scale, my_b1, (int)r, 128);
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            named_bar_sync(pp.bar_id, 128);
+        };
+        unsigned long long best = 0;
+        float best_y = __int_as_float(0x7fc00000);
+        auto flush = [&]() {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, best, o);
+                const float y2 = __shfl_xor_sync(0xffffffffu, best_y, o);
+                if (k2 > best) { best = k2; best_y = y2; }
+            }
+            if ((tid & 31) == 0 && best) acc_fold(&acc[d], best, best_y);
+            best = 0;
+        };
+        Walker W{};
+        uint32_t vX[kKMax], vY[kKMax];
+        int sX = 0, sY = 0;
+        bool okX = false, okY = false, zX = false, zY = false;
+        auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z) {
+            ok = W.u_end - W.ub > (uint64_t)r;
+            z = walker_is_index0(W, r);
+#pragma unroll
+            for (int j = 0; j < kKMax; j++) v[j] = W.v[j];
+            s = W.s;
+        };
+        auto fold = [&](uint32_t yb, int s, const uint32_t (&v)[kKMax], bool ok, bool z) {
+            const float y = __uint_as_float(yb);
+            if (ok && z) y0s[d] = y;
+            if (ok) fold_tile(P, s, v, y, best, best_y);
+        };
+        // the pair p's two tiles enter the slots (local tiles of decision d)
+        auto enter_pair = [&](uint64_t p, bool fresh) {
+            const uint64_t lt = 2 * (p - dec_pair0);
+            if (fresh) walker_begin(P, W, lt, r);
+            else walker_next(P, W, lt, r);
+            take(vX, sX, okX, zX);
+            store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
+            walker_next(P, W, lt + 1, r);
+            take(vY, sY, okY, zY);
+            store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
+            tmem_wait_st();
+            if (pp.handoff(pp.me[3])) {
+                issue_l1(pp.X, sX);
+                issue_l1(pp.Y, sY);
+                pp.commit();
+            }
+        };
+        load_decision();
+        enter_pair(pb, true);
+        for (uint64_t p = pb; p < pe; p++) {
+            uint32_t ybx, yby;
+            pp.template run_layers<true>(ybx, yby);
+            fold(ybx, sX, vX, okX, zX);
+            fold(yby, sY, vY, okY, zY);
+            if (p + 1 == dec_pair_end) {  // leaving decision d
+                flush();
+                if (p + 1 < pe) {
+                    d++;
+                    load_decision();
+                    enter_pair(p + 1, true);
+                }
+            } else if (p + 1 < pe) {
+                enter_pair(p + 1, false);
+            }
+        }
+        flush();  // the last decision of the range (a no-op if it was flushed at its end)
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    if (warp == 0) tmem_dealloc(tbase, 512);
+}
+
+// a7 for a batch: one warp per decision, lane j decodes slot j of t*
+__global__ void batch_finalize_kernel(const BatchDec* __restrict__ decs, const BatchAcc* __restrict__ acc,
+                                      const float* __restrict__ y0s, int32_t n_dec, Result* out) {
+    const int d = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (d >= n_dec) return;
+    const PlanHdr& h = decs[d].h;
+    const unsigned long long key = acc[d].key;
+    const int32_t my = (lane < h.k && key) ? decode_slot_ope(h, key & ((1ull << 40) - 1), lane) : 0;
+    int32_t ope[kKMax];
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) ope[j] = __shfl_sync(0xffffffffu, my, j);
+    if (lane) return;
+    Result R{};
+    R.key = key;
+    R.y_best = key ? acc[d].y : __int_as_float(0x7fc00000);
+    R.y0 = y0s[d];
+    R.evaluated = h.n_eval;
+    for (int j = 0; j < kKMax; j++) R.end_op[j] = ope[j];
+    R.total_ops = key ? (int32_t)(key >> 40) - 1 : 0;
+    R.status = key ? 0 : 2;
+    out[d] = R;
 }
 
 // ---------------------------------------------------------------------------
@@ -915,12 +1099,12 @@ constexpr int kFusedNG = 5;
 constexpr int kPredictNG = 4;
 
 template <int FMT, bool SPLIT>
-static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const OutW& ow, const float* w1b1,
-                                    Scratch* S, int nsm, cudaStream_t st, int* grid_out) {
+static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const float* w1b1, Scratch* S, int nsm,
+                                    cudaStream_t st, int* grid_out) {
     using C = TcCfg<FMT>;
-    const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, 2 * kFusedNG,
-                                         w1_stage_bytes(P.D, 2 * kFusedNG));
-    auto kern = P.trace ? fused_tc_kernel<FMT, SPLIT, kFusedNG, true> : fused_tc_kernel<FMT, SPLIT, kFusedNG, false>;
+    const TcSmem L =
+        tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, kFusedNG, w1_stage_bytes(P.D, kFusedNG));
+    auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
     // spread the tiles over as many SMs as possible (one tile per group first)
@@ -928,26 +1112,61 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const Out
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     *grid_out = (int)g;
-    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, ow, w1b1, S);
+    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, w1b1, S);
     return cudaGetLastError();
 }
+
+// digits are < cnt: exact unsplit up to 2048 in fp16, 256 in bf16
+static bool need_split(int fmt, uint32_t maxcnt) { return fmt == 0 ? maxcnt > 2049 : maxcnt > 257; }
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
-    OutW ow;
-    for (int j = 0; j < kHidden; j++) ow.w4s[j] = TW.w4s[j];
-    ow.b4 = TW.b4;
     uint32_t maxcnt = 0;
     for (int s = 0; s < P.n_seg; s++)
         for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
-    // digits are < cnt: exact unsplit up to 2048 in fp16, 256 in bf16
+    const bool split = need_split(TW.fmt, maxcnt);
     if (TW.fmt == 0) {
-        if (maxcnt <= 2049) return launch_fused_fmt<0, false>(P, tp, ow, w1b1, S, nsm, st, grid_out);
-        return launch_fused_fmt<0, true>(P, tp, ow, w1b1, S, nsm, st, grid_out);
+        if (!split) return launch_fused_fmt<0, false>(P, tp, w1b1, S, nsm, st, grid_out);
+        return launch_fused_fmt<0, true>(P, tp, w1b1, S, nsm, st, grid_out);
     }
-    if (maxcnt <= 257) return launch_fused_fmt<1, false>(P, tp, ow, w1b1, S, nsm, st, grid_out);
-    return launch_fused_fmt<1, true>(P, tp, ow, w1b1, S, nsm, st, grid_out);
+    if (!split) return launch_fused_fmt<1, false>(P, tp, w1b1, S, nsm, st, grid_out);
+    return launch_fused_fmt<1, true>(P, tp, w1b1, S, nsm, st, grid_out);
+}
+
+template <int FMT, bool SPLIT>
+static cudaError_t launch_batch_fmt(const BatchDec* decs, const SegP* segs, int32_t n_dec, uint64_t n_pairs,
+                                    int32_t D, const TcParams& tp, const float* w1b1, BatchAcc* acc, float* y0s,
+                                    int nsm, cudaStream_t st) {
+    uint32_t plans_off;
+    const TcSmem L = batch_smem_layout<FMT>(D, kFusedNG, &plans_off);
+    auto kern = fused_batch_tc_kernel<FMT, SPLIT, kFusedNG>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    if (e != cudaSuccess) return e;
+    uint64_t g = (n_pairs + kFusedNG - 1) / kFusedNG;
+    if (g > (uint64_t)nsm) g = (uint64_t)nsm;
+    if (g < 1) g = 1;
+    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(decs, segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, uint64_t n_pairs,
+                            uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1, BatchAcc* acc,
+                            float* y0s, Result* out, int nsm, cudaStream_t st) {
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    const bool split = need_split(TW.fmt, maxcnt);
+    cudaError_t e;
+    if (TW.fmt == 0)
+        e = split ? launch_batch_fmt<0, true>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st)
+                  : launch_batch_fmt<0, false>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st);
+    else
+        e = split ? launch_batch_fmt<1, true>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st)
+                  : launch_batch_fmt<1, false>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st);
+    if (e != cudaSuccess) return e;
+    const int threads = 256;
+    const int blocks = (int)(((int64_t)n_dec * 32 + threads - 1) / threads);
+    batch_finalize_kernel<<<blocks, threads, 0, st>>>(d_decs, acc, y0s, n_dec, out);
+    return cudaGetLastError();
 }
 
 template <int FMT>

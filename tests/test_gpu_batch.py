@@ -1,0 +1,146 @@
+"""NEXT-4: many independent scheduling rounds in one
+abacus_search_batch call.  Decision i of a batch must be exactly the
+single-round abacus_search of the same inputs (the same per-row arithmetic on
+the tensor cores, so bit-identical), and within the oracle's acceptance window
+(reading c18) like every other search."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+import paper_conf_sc_cui0czlzsmylg21_b200 as ab
+from gpu_util import EPS, Ctx, accept_key
+from oracle_helpers import load_fig12, unit0_params
+
+pytestmark = pytest.mark.gpu
+TC = [ab.ABACUS_FP16, ab.ABACUS_BF16]
+SPACES = [ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN, ab.ABACUS_SPACE_AUTO]
+
+
+def _same(a, b):
+    fields = ["status", "critical", "key", "index", "evaluated", "total_ops"]
+    for f in fields:
+        assert getattr(a, f) == getattr(b, f), f
+    assert list(a.order) == list(b.order) and list(a.end_op) == list(b.end_op)
+    for f in ["headroom_ms", "pred_ms", "pred_critical_only_ms"]:
+        x, y = getattr(a, f), getattr(b, f)
+        assert (np.isnan(x) and np.isnan(y)) or x == y, f
+
+
+def _mixed(n, seed=5):
+    """cfg2 (3-way) and cfg3 (4-way) rounds, plus k = 1 and k = 2 rounds cut from them."""
+    rng = np.random.default_rng(seed)
+    d2 = synth.cfg2_decisions(n)
+    d3 = synth.cfg3_decisions(n, seed=31)
+    out = []
+    for i in range(n):
+        qs, now, infl = (d2 if i % 2 else d3)[i]
+        kk = int(rng.integers(1, len(qs) + 1))
+        out.append((qs[:kk], now, infl))
+    return out
+
+
+@pytest.mark.parametrize("prec", TC)
+@pytest.mark.parametrize("space", SPACES)
+def test_batch_equals_single_rounds(prec, space):
+    c = Ctx(params=synth.weights(1), precision=prec)
+    try:
+        decs = _mixed(96)
+        got = ab.abacus_search_batch(c.h, decs, space, 200_000)
+        for (qs, now, infl), g in zip(decs, got):
+            _same(g, ab.abacus_search(c.h, qs, now, infl, space, 200_000))
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", TC)
+@pytest.mark.parametrize("space", [ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN])
+def test_batch_cfg2_vs_oracle(prec, space):
+    c = Ctx(params=synth.weights(1), precision=prec)
+    eps = EPS[prec]
+    try:
+        decs = synth.cfg2_decisions(40)
+        got = ab.abacus_search_batch(c.h, decs, space)
+        for (qs, now, infl), d in zip(decs, got):
+            od = oracle.search(c.params, qs, now, infl, space=space, budget=2**40, eps=eps)
+            assert d.critical == od.critical and list(d.order)[:3] == list(od.order)[:3]
+            assert d.headroom_ms == np.float32(od.headroom_ms)
+            assert d.evaluated == od.evaluated
+            assert abs(d.pred_critical_only_ms - od.pred_critical_only_ms) <= eps * abs(od.pred_critical_only_ms)
+            if abs(od.pred_critical_only_ms - od.headroom_ms) > eps * abs(od.headroom_ms):
+                assert d.status == od.status
+            if d.status == ab.ABACUS_DECIDE_OK and od.status == ab.ABACUS_DECIDE_OK:
+                assert accept_key(d.key, od.maxkey_strict, od.maxkey_loose)
+                assert d.total_ops == (d.key >> 40) - 1
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", TC)
+def test_batch_fig12_among_other_rounds(prec):
+    """The Fig. 12 replay at several positions of a batch."""
+    f = load_fig12()
+    d_feat = f["n_models"] + 16
+    p = unit0_params(d_feat, f["unit0"]["bias"], {int(k): v for k, v in f["unit0"]["coef"].items()})
+    c = Ctx(ops=f["ops_per_model"], params=p, precision=prec)
+    try:
+        fig = [synth.Query(q["model_id"], q["next_op"], 1, 0, q["headroom_ms"], 0.0) for q in f["queries"]]
+        other = [synth.Query(1, 2, 1, 0, 40.0, 0.0), synth.Query(3, 1, 1, 0, 30.0, 0.0)]
+        decs = [(fig, 0.0, 0.0) if i % 3 == 0 else (other[: 1 + i % 2], 0.0, 0.0) for i in range(10)]
+        names = [q["name"] for q in f["queries"]]
+        for space in (ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN):
+            got = ab.abacus_search_batch(c.h, decs, space)
+            for i, d in enumerate(got):
+                if i % 3:
+                    continue
+                assert d.status == ab.ABACUS_DECIDE_OK
+                assert names[d.critical] == f["expected"]["critical"]
+                assert {names[j]: d.end_op[j] for j in range(3)} == f["expected"]["end_op"]
+                assert d.pred_ms == f["expected"]["pred_ms"]
+                assert d.index == (f["expected"]["grid_t"] if space == 0 else f["expected"]["chain_u"])
+    finally:
+        c.close()
+
+
+def test_batch_large_and_regrow():
+    """Batches of growing size (buffers regrow), one decision repeated: every copy identical."""
+    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_FP16)
+    try:
+        qs, now, infl = synth.cfg3_decisions(1, seed=7)[0]
+        ref = ab.abacus_search(c.h, qs, now, infl, ab.ABACUS_SPACE_AUTO, 1_000_000)
+        for n in (1, 300, 2000):
+            got = ab.abacus_search_batch(c.h, [(qs, now, infl)] * n, ab.ABACUS_SPACE_AUTO, 1_000_000)
+            for g in got:
+                _same(g, ref)
+    finally:
+        c.close()
+
+
+def test_batch_fp32_is_per_round():
+    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_FP32)
+    try:
+        decs = synth.cfg2_decisions(12)
+        got = ab.abacus_search_batch(c.h, decs, ab.ABACUS_SPACE_GRID)
+        for (qs, now, infl), g in zip(decs, got):
+            _same(g, ab.abacus_search(c.h, qs, now, infl, ab.ABACUS_SPACE_GRID))
+    finally:
+        c.close()
+
+
+def test_batch_errors_name_the_decision():
+    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_FP16)
+    try:
+        decs = synth.cfg2_decisions(5)
+        bad = list(decs)
+        qs = list(bad[3][0])
+        qs[1] = synth.Query(qs[0].model_id, 1, 4, 0, 50.0, 0.0)  # duplicate model
+        bad[3] = (qs, bad[3][1], bad[3][2])
+        with pytest.raises(ab.AbacusError) as e:
+            ab.abacus_search_batch(c.h, bad)
+        assert e.value.code == ab.ABACUS_E_DUP_MODEL and "decision 3" in str(e.value)
+        with pytest.raises(ab.AbacusError):
+            ab.abacus_search_batch(c.h, [])
+        # still usable after an error
+        assert len(ab.abacus_search_batch(c.h, decs)) == 5
+    finally:
+        c.close()
