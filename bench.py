@@ -286,6 +286,12 @@ def decision_latency(ab, ctx, n=10_000, warm=100, precision="fp16"):
                                    ("cfg3", "auto", 1 << 22)):
             key = "%s_%s" % (cfg, space) + ("_%d" % budget if space == "auto" else "")
             out[key] = dl.run(cfg, space, precision, n, warm, budget or 4_194_304)
+        # NEXT-4: many rounds per call (abacus_search_batch), decisions/s
+        out["batched"] = {
+            "cfg2_grid_b4096": dl.run("cfg2", "grid", precision, 16_384, warm, 4_194_304, batch=4096),
+            "cfg3_chain_b4096": dl.run("cfg3", "chain", precision, 16_384, warm, 4_194_304, batch=4096),
+            "cfg3_auto_4194304_b1024": dl.run("cfg3", "auto", precision, 4096, warm, 4_194_304, batch=1024),
+        }
     except Exception as e:  # noqa: BLE001 -- report, do not fail the bench line
         out["c_abi_error"] = repr(e)
     decs = synth.cfg2_decisions(n + warm)

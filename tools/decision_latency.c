@@ -4,6 +4,9 @@
  *   int32 precision, int32 space, uint64 budget, int32 n_dec, int32 warm,
  *   n_dec x { int32 k, double now, double inflight, k x abacus_query_t }
  * Output: one line of JSON with p50/p99/p99.9 (us) and the grid-size spread.
+ * With a second argument B > 0: abacus_search_batch over consecutive batches
+ * of B decisions (the first `warm` decisions warm up); reports per-call
+ * latency, decisions/s and the kernel share (CUDA events around the launch).
  */
 #include <stdio.h>
 #include <stdlib.h>
@@ -49,6 +52,39 @@ int main(int argc, char** argv) {
     if (rc) { fprintf(stderr, "create failed %d\n", rc); return 1; }
     rc = abacus_load_predictor(ctx, prm, np, prec);
     if (rc) { fprintf(stderr, "load failed %s\n", abacus_last_error(ctx)); return 1; }
+    int B = argc > 2 ? atoi(argv[2]) : 0;
+    if (B > 0) {
+        abacus_decision_t* out = malloc(sizeof(abacus_decision_t) * B);
+        abacus_set_timing(ctx, 1);
+        /* warm-up: one call of the same size (grows the ctx buffers) */
+        if (ndec < B) { fprintf(stderr, "need >= B decisions\n"); return 2; }
+        rc = abacus_search_batch(ctx, qs, ks, nows, infl, B, space, budget, out);
+        if (rc) { fprintf(stderr, "batch failed %s\n", abacus_last_error(ctx)); return 1; }
+        int calls = (ndec - warm) / B;
+        double* cl = malloc(8 * calls);
+        double kms = 0.0, tsum = 0.0;
+        uint64_t evsum = 0;
+        int ndrop = 0;
+        for (int c = 0; c < calls; c++) {
+            const int i0 = warm + c * B;
+            double t0 = now_us();
+            rc = abacus_search_batch(ctx, &qs[4 * i0], &ks[i0], &nows[i0], &infl[i0], B, space, budget, out);
+            double t1 = now_us();
+            if (rc) { fprintf(stderr, "batch failed %s\n", abacus_last_error(ctx)); return 1; }
+            cl[c] = t1 - t0;
+            tsum += cl[c];
+            kms += abacus_last_kernel_ms(ctx);
+            for (int i = 0; i < B; i++) { evsum += out[i].evaluated; ndrop += out[i].status == ABACUS_DECIDE_DROP; }
+        }
+        qsort(cl, calls, sizeof(double), cmpd);
+        printf("{\"batch\": %d, \"calls\": %d, \"call_p50_us\": %.1f, \"call_p99_us\": %.1f, "
+               "\"decisions_per_s\": %.1f, \"kernel_us_mean\": %.1f, \"evaluated_mean\": %.1f, "
+               "\"candidates_per_s\": %.4g, \"drops\": %d}\n",
+               B, calls, cl[calls / 2], cl[(int)(0.99 * calls)], (double)calls * B / (tsum * 1e-6),
+               kms * 1e3 / calls, (double)evsum / ((double)calls * B), (double)evsum / (tsum * 1e-6), ndrop);
+        abacus_destroy(ctx);
+        return 0;
+    }
     double* lat = malloc(8 * ndec);
     uint64_t* ev = malloc(8 * ndec);
     int ndrop = 0;

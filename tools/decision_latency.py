@@ -43,16 +43,17 @@ def write_input(path, decs, precision, space, budget, warm):
                 f.write(struct.pack("<iiiidd", q.model_id, q.next_op, q.batch, q.seqlen, q.qos_ms, q.t_start_ms))
 
 
-def run(config="cfg2", space="grid", precision="fp16", n=10_000, warm=100, budget=4_194_304):
+def run(config="cfg2", space="grid", precision="fp16", n=10_000, warm=100, budget=4_194_304, batch=0):
     exe = build_driver()
     decs = synth.cfg2_decisions(n + warm) if config == "cfg2" else synth.cfg3_decisions(n + warm)
     path = "/tmp/abacus_dec_%s_%s.bin" % (config, space)
     write_input(path, decs, PREC[precision], SPACE[space], budget, warm)
-    out = subprocess.check_output([exe, path]).decode()
+    out = subprocess.check_output([exe, path] + ([str(batch)] if batch else [])).decode()
     d = json.loads(out)
     d.update({"config": config, "space": space, "precision": precision,
               "budget": budget if space == "auto" else None, "ways": budget if space == "mway" else None,
-              "path": "C ABI (abacus_search), host steady clock around each call"})
+              "path": "C ABI (%s), host steady clock around each call" % (
+                  "abacus_search_batch" if batch else "abacus_search")})
     return d
 
 
@@ -63,5 +64,6 @@ if __name__ == "__main__":
     ap.add_argument("--precision", default="fp16")
     ap.add_argument("-n", type=int, default=10_000)
     ap.add_argument("--budget", type=int, default=4_194_304, help="AUTO budget, or the ways of mway")
+    ap.add_argument("--batch", type=int, default=0, help="decisions per abacus_search_batch call (0: single)")
     a = ap.parse_args()
-    print(json.dumps(run(a.config, a.space, a.precision, a.n, budget=a.budget)))
+    print(json.dumps(run(a.config, a.space, a.precision, a.n, budget=a.budget, batch=a.batch)))
