@@ -21,7 +21,6 @@ import json
 import os
 import sys
 import time
-from collections import deque
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
@@ -30,6 +29,7 @@ import torch  # noqa: E402
 
 import synth  # noqa: E402
 import paper_conf_sc_cui0czlzsmylg21_b200 as ab  # noqa: E402
+from paper_conf_sc_cui0czlzsmylg21_b200 import controller as ctl  # noqa: E402
 
 SPACE = {"grid": ab.ABACUS_SPACE_GRID, "chain": ab.ABACUS_SPACE_CHAIN, "auto": ab.ABACUS_SPACE_AUTO}
 
@@ -52,86 +52,24 @@ def simulate(ctx, qps, seconds, space, budget, seed=13):
     services = synth.cfg3_services()
     qos = {m: 2.0 * solo_latency(ctx, m) for m in services}
     arrivals = synth.cfg3_arrivals(qps, seconds * 1000.0, seed)
-    fifo = {m: deque() for m in services}
-    ai = 0
-    t = 0.0
-    done_lat, violations, drops, completed = [], 0, 0, 0
-    n_groups, search_us, group_ms, evaluated = 0, [], [], 0
-    active = {}  # service -> [arrival, bs, seqlen, next_op]
+    search_us = []
 
-    def admit(until):
-        nonlocal ai
-        while ai < len(arrivals) and arrivals[ai][0] <= until:
-            ta, m, bs, sl = arrivals[ai]
-            fifo[m].append((ta, bs, sl))
-            ai += 1
-
-    def refill():
-        for m in services:
-            if m not in active and fifo[m]:
-                ta, bs, sl = fifo[m].popleft()
-                active[m] = [ta, bs, sl, 1]
-
-    inflight = 0.0  # predicted latency of the group currently executing (Eq. 3)
-    horizon = seconds * 1000.0
-    while t < horizon or active or any(fifo.values()):
-        admit(t)
-        refill()
-        if not active:
-            if ai >= len(arrivals):
-                break
-            t = max(t, arrivals[ai][0])
-            continue
-        ms = list(active.keys())
-        qs = [synth.Query(m, active[m][3], active[m][1], active[m][2], qos[m], active[m][0]) for m in ms]
+    def search(qs, now, infl):
         w0 = time.perf_counter()
-        d = ab.abacus_search(ctx, qs, t, inflight, space, budget)
+        d = ab.abacus_search(ctx, qs, now, infl, space, budget)
         search_us.append((time.perf_counter() - w0) * 1e6)
-        evaluated += d.evaluated
-        if d.status == ab.ABACUS_DECIDE_DROP:
-            m = ms[d.critical]
-            del active[m]
-            drops += 1
-            violations += 1
-            continue
-        # issue the group: it runs for its predicted latency after the in-flight one
-        start = t + inflight
-        dur = float(d.pred_ms)
-        end = start + dur
-        n_groups += 1
-        group_ms.append(dur)
-        for i, m in enumerate(ms):
-            e = d.end_op[i]
-            if e == 0:
-                continue
-            if e >= synth.L(m):
-                lat = end - active[m][0]
-                done_lat.append(lat)
-                completed += 1
-                if lat > qos[m]:
-                    violations += 1
-                del active[m]
-            else:
-                active[m][3] = e + 1
-        # pipelining (Fig. 13): the next search happens now, while this group runs
-        t = start
-        inflight = dur
-    sim_ms = max(t + inflight, horizon)
-    lat = np.array(done_lat) if done_lat else np.zeros(1)
+        return d
+
+    r = ctl.simulate(search, arrivals, qos, {m: synth.L(m) for m in services})
+    out = {"qps_per_service": qps, "simulated_s": seconds, "space": space, "budget": budget, "qos_ms": qos}
+    out.update(ctl.summary(r, seconds))
     sa = np.array(search_us)
-    return {"qps_per_service": qps, "simulated_s": sim_ms / 1000.0, "space": space, "budget": budget,
-            "qos_ms": qos, "queries": len(arrivals), "completed": completed, "dropped": drops,
-            "qos_violation_rate": violations / max(1, len(arrivals)),
-            "throughput_qps": completed / (sim_ms / 1000.0), "latency_p50_ms": float(np.percentile(lat, 50)),
-            "latency_p99_ms": float(np.percentile(lat, 99)), "groups": n_groups,
-            "group_ms_mean": float(np.mean(group_ms)) if group_ms else 0.0,
-            "decisions": len(search_us), "candidates_evaluated": int(evaluated),
-            "search_us_p50": float(np.percentile(sa, 50)), "search_us_p99": float(np.percentile(sa, 99)),
-            "search_us_p999": float(np.percentile(sa, 99.9)),
-            "group_ms_min": float(np.min(group_ms)) if group_ms else 0.0,
-            "search_hidden": bool(group_ms) and float(np.max(sa)) / 1000.0 < float(np.min(group_ms)),
-            "note": "synthetic random-init predictor: its latency landscape is not a real model's, so QoS/throughput "
-                    "figures exercise the controller mechanics only"}
+    out.update({"search_us_p50": float(np.percentile(sa, 50)), "search_us_p99": float(np.percentile(sa, 99)),
+                "search_us_p999": float(np.percentile(sa, 99.9)),
+                "search_hidden": bool(r.group_ms) and float(np.max(sa)) / 1000.0 < float(np.min(r.group_ms)),
+                "note": "synthetic random-init predictor: its latency landscape is not a real model's, so "
+                        "QoS/throughput figures exercise the controller mechanics only"})
+    return out
 
 
 if __name__ == "__main__":
