@@ -325,6 +325,33 @@ def instance_samples(n: int, seed: int = 15, ks: Sequence[int] = (2, 3, 4),
     return out
 
 
+# ---------------------------------------------------------------------------
+# NEXT-3: a synthetic stand-in for the paper's profiled group latencies (the
+# 42 h of A100 runs behind Fig. 10 are out of scope).  This is the WORKLOAD's
+# ground truth, not the method: the predictor is trained to approximate it.
+#   solo_i  = base_m * (0.3 + 0.7 (bs/8)^0.85) * (seqlen/128)^0.9 [Bert only] * n_i / L_m
+#   latency = max_i solo_i + 0.35 * (sum_i solo_i - max_i solo_i) + 0.05 ms
+# times a seeded log-normal measurement noise (sigma 2 %).
+# ---------------------------------------------------------------------------
+LATENCY_BASE_MS = {1: 6.0, 2: 11.0, 3: 16.0, 4: 9.0, 5: 12.0, 6: 14.0, 7: 8.0, 8: 22.0}  # whole model, bs 8
+
+
+def group_latency_ms(groups: Sequence["Group"], seed: int = 16, noise: float = 0.02) -> np.ndarray:
+    rng = np.random.Generator(np.random.PCG64(seed))
+    y = np.zeros(len(groups), dtype=np.float64)
+    for i, g in enumerate(groups):
+        solo = []
+        for (m, ops, ope, bs, sl) in g.slots:
+            t = LATENCY_BASE_MS[m] * (0.3 + 0.7 * (bs / 8.0) ** 0.85)
+            if m in BERT_LIKE:
+                t *= (sl / 128.0) ** 0.9
+            solo.append(t * (ope - ops + 1) / L(m))
+        y[i] = max(solo) + 0.35 * (sum(solo) - max(solo)) + 0.05
+    if noise:
+        y *= np.exp(rng.normal(0.0, noise, len(groups)))
+    return y
+
+
 def tiny_grids(n: int, seed: int = 21, n_models: int = N_MODELS, kmax: int = K_MAX,
                max_len: int = 6) -> List[List[GridSlot]]:
     """Small random sweep grids for brute-force pins and ragged GPU parity:
