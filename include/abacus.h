@@ -50,6 +50,7 @@ extern "C" {
 #define ABACUS_HIDDEN 32
 #define ABACUS_ABI_VERSION 2
 #define ABACUS_BATCH_MAX (1 << 20) /* decisions per abacus_search_batch call */
+#define ABACUS_TRAIN_MAX_BATCH 65536 /* samples per training step */
 
 /* status codes */
 enum {
@@ -199,6 +200,43 @@ int abacus_predict_batch(abacus_ctx* ctx, const int16_t* d_features, uint64_t co
 int abacus_select_group(abacus_ctx* ctx, const abacus_grid_t* grid, uint64_t first, uint64_t count,
                         const float* d_latency_ms, float headroom_ms, unsigned long long* d_best_key,
                         void* stream);
+
+/* ------------------------------------------------------------------------ */
+/* Training the predictor                          */
+/* ------------------------------------------------------------------------ */
+/* The paper trains the MLP on instance-based samples (Fig. 9)
+ * and measures MAPE (Eq. 1) but states no training procedure.
+ * Readings (DESIGN.md t1-t3): loss = mean over the minibatch of
+ * (y_pred / y_true - 1)^2; Adam with bias correction; the learning rate is
+ * given per call.  All arithmetic is fp32 on the device. */
+typedef struct {
+    float beta1, beta2, eps; /* e.g. 0.9, 0.999, 1e-8 */
+} abacus_adam_t;
+
+/* Start (or restart) training from `params` (host, fp32, the
+ * abacus_load_predictor layout): copies them to the ctx's training state and
+ * zeroes the Adam moments and step counter.  Blocking.  Errors: E_INVALID
+ * (size, non-finite values, hyper-parameters), E_CUDA. */
+int abacus_train_begin(abacus_ctx* ctx, const float* params, size_t n_params, const abacus_adam_t* opt);
+
+/* One Adam step on a minibatch: d_features (device int16, count x D, Fig. 8
+ * rows as for abacus_predict_batch), d_latency_ms (device fp32, count, > 0).
+ * 1 <= count <= ABACUS_TRAIN_MAX_BATCH.  d_grad (device fp32, n_params, may
+ * be NULL) receives the minibatch gradient.  Async on `stream`.
+ * Errors: E_NOT_LOADED (no abacus_train_begin), E_INVALID, E_CUDA. */
+int abacus_train_step(abacus_ctx* ctx, const int16_t* d_features, const float* d_latency_ms, uint64_t count,
+                      float lr, float* d_grad, void* stream);
+
+/* Consecutive minibatches of `batch` rows (the last may be shorter), one
+ * Adam step each, learning rate lr.  d_losses (device fp32, one per step,
+ * may be NULL) receives each step's loss.  Async on `stream`. */
+int abacus_train_epoch(abacus_ctx* ctx, const int16_t* d_features, const float* d_latency_ms, uint64_t count,
+                       uint32_t batch, float lr, float* d_losses, void* stream);
+
+/* Blocking: copy the current parameters to params_out (host, n_params) and,
+ * if last_loss != NULL, the last step's loss.  Pass them to
+ * abacus_load_predictor to search with the trained predictor. */
+int abacus_train_params(abacus_ctx* ctx, float* params_out, float* last_loss);
 
 /* ------------------------------------------------------------------------ */
 /* Fused search (blocking)                                                   */

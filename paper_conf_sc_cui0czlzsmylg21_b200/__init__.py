@@ -12,6 +12,8 @@ import ctypes as C
 import os
 from typing import List, Optional, Sequence
 
+import numpy as np
+
 from . import _build
 
 HERE = os.path.dirname(os.path.abspath(__file__))
@@ -29,7 +31,12 @@ EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
             "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_nccl_unique_id",
             "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
-            "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version"]
+            "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version",
+            "abacus_train_begin", "abacus_train_step", "abacus_train_epoch", "abacus_train_params"]
+
+
+class abacus_adam_t(C.Structure):
+    _fields_ = [("beta1", C.c_float), ("beta2", C.c_float), ("eps", C.c_float)]
 
 
 class abacus_slot_t(C.Structure):
@@ -111,6 +118,10 @@ def lib():
         L.abacus_set_timing.argtypes = [vp, C.c_int]
         L.abacus_set_stream.argtypes = [vp, vp]
         L.abacus_abi_version.argtypes = []
+        L.abacus_train_begin.argtypes = [vp, P(C.c_float), C.c_size_t, P(abacus_adam_t)]
+        L.abacus_train_step.argtypes = [vp, vp, vp, C.c_uint64, C.c_float, vp, vp]
+        L.abacus_train_epoch.argtypes = [vp, vp, vp, C.c_uint64, C.c_uint32, C.c_float, vp, vp]
+        L.abacus_train_params.argtypes = [vp, P(C.c_float), P(C.c_float)]
         _lib = L
     return _lib
 
@@ -174,7 +185,6 @@ def abacus_last_error(ctx: int) -> str:
 
 
 def abacus_load_predictor(ctx: int, params, precision: int) -> None:
-    import numpy as np
     p = np.ascontiguousarray(params, dtype=np.float32)
     _check(ctx, lib().abacus_load_predictor(ctx, p.ctypes.data_as(C.POINTER(C.c_float)), p.size, precision))
 
@@ -279,6 +289,31 @@ def abacus_set_timing(ctx, on: bool) -> None:
 
 def abacus_set_stream(ctx, stream) -> None:
     _check(ctx, lib().abacus_set_stream(ctx, _stream(stream)))
+
+
+def abacus_train_begin(ctx, params, beta1: float = 0.9, beta2: float = 0.999, eps: float = 1e-8) -> None:
+    p = np.ascontiguousarray(params, dtype=np.float32)
+    opt = abacus_adam_t(beta1, beta2, eps)
+    _check(ctx, lib().abacus_train_begin(ctx, p.ctypes.data_as(C.POINTER(C.c_float)), p.size, C.byref(opt)))
+
+
+def abacus_train_step(ctx, d_features, d_latency_ms, count: int, lr: float, d_grad=None, stream=None) -> None:
+    _check(ctx, lib().abacus_train_step(ctx, _ptr(d_features), _ptr(d_latency_ms), count, lr, _ptr(d_grad),
+                                        _stream(stream)))
+
+
+def abacus_train_epoch(ctx, d_features, d_latency_ms, count: int, batch: int, lr: float, d_losses=None,
+                       stream=None) -> None:
+    _check(ctx, lib().abacus_train_epoch(ctx, _ptr(d_features), _ptr(d_latency_ms), count, batch, lr,
+                                         _ptr(d_losses), _stream(stream)))
+
+
+def abacus_train_params(ctx, n_params: int):
+    """Returns (params float32 array, last step's loss)."""
+    out = np.zeros(n_params, dtype=np.float32)
+    loss = C.c_float()
+    _check(ctx, lib().abacus_train_params(ctx, out.ctypes.data_as(C.POINTER(C.c_float)), C.byref(loss)))
+    return out, float(loss.value)
 
 
 def abacus_abi_version() -> int:

@@ -8,7 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libabacus.so")
 PROBE_LIB = os.path.join(HERE, "libabacus_probe.so")
-SOURCES = ["abacus.cu", "kernels_simt.cu", "kernels_tc.cu"]
+SOURCES = ["abacus.cu", "kernels_simt.cu", "kernels_tc.cu", "kernels_train.cu"]
 HEADERS = ["common.cuh", "device_common.cuh", "internal.h", "tc_ptx.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

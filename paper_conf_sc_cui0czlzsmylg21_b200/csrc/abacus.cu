@@ -63,6 +63,17 @@ struct abacus_ctx {
     Result* d_out = nullptr;
     std::vector<int32_t> b_order;  // [4 n] headroom order per decision
     std::vector<float> b_H;
+    // NEXT-3 training state (abacus_train_begin)
+    bool training = false;
+    abacus_adam_t adam{};
+    int64_t train_t = 0;          // Adam step counter
+    float* t_p = nullptr;         // parameters, m, v (device, n_params each)
+    float* t_m = nullptr;
+    float* t_v = nullptr;
+    float* t_partial = nullptr;   // [kTrainMaxBlocks][n_params]
+    float* t_loss_part = nullptr;
+    float* t_loss = nullptr;      // last step's loss (device scalar)
+    unsigned* t_ticket = nullptr;
 };
 
 namespace {
@@ -737,6 +748,13 @@ void abacus_destroy(abacus_ctx* c) {
     cudaFree(c->d_acc);
     cudaFree(c->d_y0);
     cudaFree(c->d_out);
+    cudaFree(c->t_p);
+    cudaFree(c->t_m);
+    cudaFree(c->t_v);
+    cudaFree(c->t_partial);
+    cudaFree(c->t_loss_part);
+    cudaFree(c->t_loss);
+    cudaFree(c->t_ticket);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->own_stream) cudaStreamDestroy(c->own_stream);
@@ -1063,6 +1081,118 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     d.total_ops = R.total_ops;
     for (int j = 0; j < grid->k; j++) d.end_op[j] = R.end_op[j];
     *out = d;
+    return ABACUS_OK;
+}
+
+// ---- NEXT-3: training (kernels_train.cu) ----------------------------------
+static constexpr uint64_t kTrainMaxBatch = ABACUS_TRAIN_MAX_BATCH;
+static constexpr unsigned kTrainMaxBlocks = (unsigned)(kTrainMaxBatch / 128);
+
+int abacus_train_begin(abacus_ctx* c, const float* params, size_t n_params, const abacus_adam_t* opt) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!params || !opt) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    const int np = train_n_params(c->D);
+    if (n_params != (size_t)np) return fail(c, ABACUS_E_INVALID, "n_params=%zu, expected %d", n_params, np);
+    for (size_t i = 0; i < n_params; i++)
+        if (!std::isfinite(params[i])) return fail(c, ABACUS_E_INVALID, "non-finite parameter %zu", i);
+    if (!(opt->beta1 >= 0.0f && opt->beta1 < 1.0f && opt->beta2 >= 0.0f && opt->beta2 < 1.0f && opt->eps > 0.0f))
+        return fail(c, ABACUS_E_INVALID, "bad Adam hyper-parameters");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    if (!c->t_p) {
+        CUDA_TRY(c, cudaMalloc(&c->t_p, np * sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_m, np * sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_v, np * sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_partial, (size_t)kTrainMaxBlocks * np * sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_loss_part, kTrainMaxBlocks * sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_loss, sizeof(float)));
+        CUDA_TRY(c, cudaMalloc(&c->t_ticket, sizeof(unsigned)));
+        CUDA_TRY(c, cudaMemset(c->t_ticket, 0, sizeof(unsigned)));
+    }
+    CUDA_TRY(c, cudaMemcpyAsync(c->t_p, params, np * sizeof(float), cudaMemcpyHostToDevice, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(c->t_m, 0, np * sizeof(float), c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(c->t_v, 0, np * sizeof(float), c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(c->t_loss, 0xFF, sizeof(float), c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    c->adam = *opt;
+    c->train_t = 0;
+    c->training = true;
+    return ABACUS_OK;
+}
+
+namespace {
+int train_one(abacus_ctx* c, const int16_t* d_x, const float* d_y, uint64_t count, float lr, float* d_grad,
+              float* d_loss, cudaStream_t st) {
+    c->train_t++;
+    TrainArgs A{};
+    A.p = c->t_p;
+    A.m = c->t_m;
+    A.v = c->t_v;
+    A.x = d_x;
+    A.t = d_y;
+    A.count = count;
+    A.D = c->D;
+    A.inv_count = (float)(1.0 / (double)count);
+    A.partial = c->t_partial;
+    A.loss_part = c->t_loss_part;
+    A.ticket = c->t_ticket;
+    A.loss_last = c->t_loss;
+    A.loss_out = d_loss;
+    A.grad_out = d_grad;
+    A.lr = lr;
+    A.beta1 = c->adam.beta1;
+    A.beta2 = c->adam.beta2;
+    A.eps = c->adam.eps;
+    A.bc1 = (float)(1.0 - std::pow((double)c->adam.beta1, (double)c->train_t));
+    A.bc2 = (float)(1.0 - std::pow((double)c->adam.beta2, (double)c->train_t));
+    const cudaError_t e = launch_train_step(A, st);
+    if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "train step launch: %s", cudaGetErrorString(e));
+    c->launches++;
+    return ABACUS_OK;
+}
+}  // namespace
+
+int abacus_train_step(abacus_ctx* c, const int16_t* d_features, const float* d_latency_ms, uint64_t count,
+                      float lr, float* d_grad, void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->training) return fail(c, ABACUS_E_NOT_LOADED, "abacus_train_begin not called");
+    if (!d_features || !d_latency_ms) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (count < 1 || count > kTrainMaxBatch) return fail(c, ABACUS_E_INVALID, "count=%llu", (unsigned long long)count);
+    if (!(lr >= 0.0f) || !std::isfinite(lr)) return fail(c, ABACUS_E_INVALID, "bad learning rate");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    return train_one(c, d_features, d_latency_ms, count, lr, d_grad, nullptr, pick_stream(c, stream));
+}
+
+int abacus_train_epoch(abacus_ctx* c, const int16_t* d_features, const float* d_latency_ms, uint64_t count,
+                       uint32_t batch, float lr, float* d_losses, void* stream) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->training) return fail(c, ABACUS_E_NOT_LOADED, "abacus_train_begin not called");
+    if (!d_features || !d_latency_ms) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (count < 1 || batch < 1 || batch > kTrainMaxBatch) return fail(c, ABACUS_E_INVALID, "count/batch");
+    if (!(lr >= 0.0f) || !std::isfinite(lr)) return fail(c, ABACUS_E_INVALID, "bad learning rate");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    cudaStream_t st = pick_stream(c, stream);
+    uint64_t step = 0;
+    for (uint64_t s = 0; s < count; s += batch, step++) {
+        const uint64_t n = count - s < batch ? count - s : batch;
+        const int rc = train_one(c, d_features + s * (uint64_t)c->D, d_latency_ms + s, n, lr, nullptr,
+                                 d_losses ? d_losses + step : nullptr, st);
+        if (rc) return rc;
+    }
+    return ABACUS_OK;
+}
+
+int abacus_train_params(abacus_ctx* c, float* params_out, float* last_loss) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->training) return fail(c, ABACUS_E_NOT_LOADED, "abacus_train_begin not called");
+    if (!params_out) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    CUDA_TRY(c, cudaDeviceSynchronize());
+    CUDA_TRY(c, cudaMemcpy(params_out, c->t_p, train_n_params(c->D) * sizeof(float), cudaMemcpyDeviceToHost));
+    if (last_loss) CUDA_TRY(c, cudaMemcpy(last_loss, c->t_loss, sizeof(float), cudaMemcpyDeviceToHost));
     return ABACUS_OK;
 }
 

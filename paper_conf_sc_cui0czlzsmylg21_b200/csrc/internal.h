@@ -46,6 +46,27 @@ cudaError_t launch_finalize_gather(Scratch* S, int nranks, Result* mapped, uint3
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out);
 // batched decisions: d_decs[n_dec] and d_segs on the device; acc/y0s zeroed / NaN-filled by the caller
+// NEXT-3: one Adam step on a minibatch (kernels_train.cu)
+struct TrainArgs {
+    float* p;                 // parameters (device, updated in place)
+    float* m;                 // Adam first moment
+    float* v;                 // Adam second moment
+    const int16_t* x;         // count x D features
+    const float* t;           // count target latencies (ms)
+    uint64_t count;
+    int32_t D;
+    float inv_count;
+    float* partial;           // [blocks][n_params] per-CTA gradient sums
+    float* loss_part;         // [blocks]
+    unsigned* ticket;         // zero between launches
+    float* loss_last;         // device scalar
+    float* loss_out;          // optional device scalar for this step
+    float* grad_out;          // optional device [n_params]
+    float lr, beta1, beta2, eps, bc1, bc2;  // bc = 1 - beta^t (bias corrections)
+};
+int train_n_params(int D);
+cudaError_t launch_train_step(const TrainArgs& A, cudaStream_t st);
+
 cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, uint64_t n_pairs,
                             uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1, BatchAcc* acc,
                             float* y0s, Result* out, int nsm, cudaStream_t st);
