@@ -92,12 +92,12 @@ __global__ void __launch_bounds__(kEncThreads) encode_grid_kernel(const __grid_c
 
 // ---------------------------------------------------------------------------
 // a2 + a3 fast path for D = 24 (N = 8): per block 1024 consecutive candidates,
-// thread t builds rows t, t + 128, ... in a shared-memory stage (3 x 16-byte
+// thread t builds rows t, t + 256, ... in a shared-memory stage (3 x 16-byte
 // stores for the bitmap and zeros, then 2 x 4-byte stores per present model at
 // its Fig.-8 position, read from a per-presence-pattern table), and one thread
 // writes the whole 48 KB stage to HBM with a TMA bulk store (double-buffered).
 // ---------------------------------------------------------------------------
-constexpr int kEnc24Threads = 128;
+constexpr int kEnc24Threads = 256;
 constexpr int kEnc24Rows = 1024;
 
 __global__ void __launch_bounds__(kEnc24Threads) encode_grid24_kernel(const __grid_constant__ Plan P, uint64_t first,
@@ -151,9 +151,21 @@ __global__ void __launch_bounds__(kEnc24Threads) encode_grid24_kernel(const __gr
             asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // stage reused two rounds later
         __syncthreads();
         const uint32_t nrows = (uint32_t)min((uint64_t)kEnc24Rows, count - base);
+        // digits of row threadIdx.x (fp64 split of the stage base + carry), then
+        // + kEnc24Threads per further row with a multiply-high carry chain
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, first + base, threadIdx.x, v);
         for (uint32_t r = threadIdx.x; r < nrows; r += kEnc24Threads) {
-            uint32_t v[kKMax];
-            decode_box<kKMax>(g, first + base, r, v);
+            if (r != threadIdx.x) {
+                uint32_t carry = kEnc24Threads;
+#pragma unroll
+                for (int d = kKMax - 1; d >= 0; d--) {
+                    const uint32_t x = v[d] + carry;
+                    const uint32_t q = fastdiv(x, g.fd[d]);
+                    v[d] = x - q * g.cnt[d];
+                    carry = q;
+                }
+            }
             uint32_t mask = 0;
 #pragma unroll
             for (int d = 0; d < kKMax; d++)
@@ -297,11 +309,13 @@ __global__ void __launch_bounds__(kPredThreads) predict_fp32_kernel(const __grid
 // ---------------------------------------------------------------------------
 constexpr int kSelThreads = 256;
 constexpr int kSelPer = 32;
+constexpr int kSelPad = kSelPer + 4;  // padded per-thread row of the load stage
 
 __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_constant__ Plan P, uint64_t first,
                                                              uint64_t count, const float* __restrict__ lat,
                                                              float H, unsigned long long* best) {
     __shared__ unsigned long long s_max[kSelThreads / 32];
+    __shared__ __align__(16) float s_y[kSelThreads * kSelPad];
     const SegP& g = P.seg[0];
     const int off = kKMax - P.k;  // digit of slot j = off + j
     // n of slot j at digit value d: 0 if absent (d == 0 and absent allowed), else nb_j + d
@@ -324,19 +338,41 @@ __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_consta
     const uint64_t chunk = (uint64_t)kSelThreads * kSelPer;
     for (uint64_t base = (uint64_t)blockIdx.x * chunk; base < count; base += (uint64_t)gridDim.x * chunk) {
         const uint64_t i0 = base + (uint64_t)threadIdx.x * kSelPer;
-        if (i0 >= count) continue;
+        const uint64_t w0 = base + (uint64_t)(threadIdx.x & ~31u) * kSelPer;  // the warp's 1024 candidates
+        const float* wsrc = lat + w0;
         float y[kSelPer];
-        const float* src = lat + i0;
-        if (i0 + kSelPer <= count && (reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+        if (w0 + 32 * kSelPer <= count && (reinterpret_cast<uintptr_t>(wsrc) & 15u) == 0) {
+            // coalesced: 8 x 512 B per warp into a padded shared stage, then each
+            // thread reads back its own 32 consecutive values (conflict-free)
+            float* sw = s_y + (threadIdx.x >> 5) * (32 * kSelPad);
+            const int lane = threadIdx.x & 31;
+            float4 a[kSelPer / 4];
 #pragma unroll
-            for (int q = 0; q < kSelPer / 4; q++) {
-                const float4 a = __ldcs(reinterpret_cast<const float4*>(src) + q);
-                y[4 * q] = a.x; y[4 * q + 1] = a.y; y[4 * q + 2] = a.z; y[4 * q + 3] = a.w;
+            for (int k = 0; k < kSelPer / 4; k++) a[k] = __ldcs(reinterpret_cast<const float4*>(wsrc) + k * 32 + lane);
+#pragma unroll
+            for (int k = 0; k < kSelPer / 4; k++) {
+                const int idx4 = k * 32 + lane;
+                *reinterpret_cast<float4*>(sw + (idx4 >> 3) * kSelPad + (idx4 & 7) * 4) = a[k];
             }
+            __syncwarp();
+#pragma unroll
+            for (int k = 0; k < kSelPer / 4; k++) {
+                const float4 b = *reinterpret_cast<const float4*>(sw + lane * kSelPad + 4 * k);
+                y[4 * k] = b.x; y[4 * k + 1] = b.y; y[4 * k + 2] = b.z; y[4 * k + 3] = b.w;
+            }
+            __syncwarp();
         } else {
+            if (i0 >= count) continue;
+            const float* src = lat + i0;
 #pragma unroll
             for (int q = 0; q < kSelPer; q++) y[q] = i0 + q < count ? src[q] : __int_as_float(0x7fc00000);
         }
+        if (i0 >= count) continue;
+        // feasibility bits of the thread's 32 consecutive candidates
+        uint32_t fm = 0;
+#pragma unroll
+        for (int q = 0; q < kSelPer; q++) fm |= (y[q] <= H ? 1u : 0u) << q;
+        if (!fm) continue;
         uint32_t v[kKMax];
         decode_box<kKMax>(g, first + base, threadIdx.x * kSelPer, v);
         auto nsum_rest = [&]() {
@@ -345,24 +381,34 @@ __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_consta
             for (int d = 0; d < kKMax - 1; d++) r += (ab[d] && v[d] == 0) ? 0 : nb[d] + (int32_t)v[d];
             return r;
         };
-        int32_t rest = nsum_rest();
+        // A run = consecutive candidates with no carry out of the last digit.
+        // Inside a run the index t and the last slot's n both grow with q, so
+        // the key ((sum_n + 1) << 40) | t is strictly increasing: only the last
+        // feasible candidate of each run can hold the run's maximum.
         const uint64_t t0 = first + i0;
-#pragma unroll
-        for (int q = 0; q < kSelPer; q++) {
-            if (y[q] <= H) {
-                const int32_t n3 = (ab[kKMax - 1] && v[kKMax - 1] == 0) ? 0 : nb[kKMax - 1] + (int32_t)v[kKMax - 1];
+        int32_t rest = nsum_rest();
+        uint32_t qa = 0;
+        while (true) {
+            const uint32_t left = (uint32_t)kSelPer - qa, room = cnt3 - v[kKMax - 1];
+            const uint32_t len = room < left ? room : left;
+            const uint32_t runm = (len >= 32u ? 0xffffffffu : ((1u << len) - 1u)) << qa;
+            const uint32_t m = fm & runm;
+            if (m) {
+                const uint32_t q = 31u - (uint32_t)__clz(m);
+                const uint32_t v3 = v[kKMax - 1] + (q - qa);
+                const int32_t n3 = (ab[kKMax - 1] && v3 == 0) ? 0 : nb[kKMax - 1] + (int32_t)v3;
                 mx = umax64(mx, ((unsigned long long)(rest + n3 + 1) << 40) | (t0 + q));
             }
-            // advance to t + 1
-            if (++v[kKMax - 1] == cnt3) {
-                v[kKMax - 1] = 0;
+            qa += len;
+            if (qa >= (uint32_t)kSelPer || !(fm >> qa)) break;
+            // carry: the last digit wraps to 0, the others count up
+            v[kKMax - 1] = 0;
 #pragma unroll
-                for (int d = kKMax - 2; d >= 0; d--) {
-                    if (++v[d] < g.cnt[d]) break;
-                    v[d] = 0;
-                }
-                rest = nsum_rest();
+            for (int d = kKMax - 2; d >= 0; d--) {
+                if (++v[d] < g.cnt[d]) break;
+                v[d] = 0;
             }
+            rest = nsum_rest();
         }
     }
     mx = warp_max_u64(mx);
