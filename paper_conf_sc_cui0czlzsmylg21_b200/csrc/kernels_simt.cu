@@ -14,6 +14,7 @@
 #include "common.cuh"
 #include "device_common.cuh"
 #include "internal.h"
+#include "tc_ptx.cuh"
 
 namespace abacus {
 
@@ -731,9 +732,111 @@ cudaError_t launch_encode_grid(const Plan& P, uint64_t first, uint64_t count, in
     return cudaGetLastError();
 }
 
+// a3 fast path for D = 24 (N = 8): persistent blocks stream tiles of 256
+// records (84 B each, 21.5 KB): the next tile's records are loaded into
+// registers (coalesced 16-byte loads) while the current tile is encoded from
+// shared memory; each thread zeroes its 48-byte row in a stage and stores the
+// bitmap entries and the (ops | ope << 16, bs | seqlen << 16) words of its
+// present models at their Fig.-8 positions; the stage is written back with
+// coalesced 16-byte streaming stores.
+constexpr int kEncG24Threads = 256;
+constexpr uint32_t kRecW = sizeof(GroupRec) / 4;                       // 21 words
+constexpr int kTileV = kEncG24Threads * (int)sizeof(GroupRec) / 16;    // 1,344 x 16 B
+constexpr int kPerV = (kTileV + kEncG24Threads - 1) / kEncG24Threads;  // 6
+
+__device__ __forceinline__ bool group_row24(const uint32_t* r, uint4* row) {
+    const int k = (int)r[0];
+    int32_t m[kKMax];
+    bool ok = k >= 0 && k <= kKMax;
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) {
+        m[j] = (int32_t)r[1 + 5 * j];
+        if (j < k) {
+            ok = ok && m[j] >= 1 && m[j] <= 8;
+#pragma unroll
+            for (int i = 0; i < j; i++) ok = ok && m[i] != m[j];
+        }
+    }
+    row[0] = make_uint4(0, 0, 0, 0);
+    row[1] = make_uint4(0, 0, 0, 0);
+    row[2] = make_uint4(0, 0, 0, 0);
+    if (ok) {
+        uint32_t* rw = reinterpret_cast<uint32_t*>(row);
+        uint16_t* rh = reinterpret_cast<uint16_t*>(row);
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) {
+            if (j >= k) continue;
+            int p = 0;
+#pragma unroll
+            for (int i = 0; i < kKMax; i++) p += (i < k && m[i] < m[j]) ? 1 : 0;
+            rh[m[j] - 1] = 1;  // bitmap x[m - 1] = 1
+            rw[4 + 2 * p] = (r[2 + 5 * j] & 0xFFFFu) | (r[3 + 5 * j] << 16);  // ops | ope
+            rw[5 + 2 * p] = (r[4 + 5 * j] & 0xFFFFu) | (r[5 + 5 * j] << 16);  // bs | seqlen
+        }
+    }
+    return ok;
+}
+
+__global__ void __launch_bounds__(kEncG24Threads) encode_groups24_kernel(const GroupRec* __restrict__ groups,
+                                                                         uint64_t count,
+                                                                         int16_t* __restrict__ out,
+                                                                         uint32_t* __restrict__ bad) {
+    __shared__ __align__(16) uint32_t s_rec[kEncG24Threads * kRecW];
+    __shared__ __align__(16) uint4 s_row[kEncG24Threads * 3];
+    __shared__ uint32_t s_bad;
+    const int tid = threadIdx.x;
+    if (tid == 0) s_bad = 0;
+    const uint64_t ntiles = (count + kEncG24Threads - 1) / kEncG24Threads;
+    uint4 a[kPerV];
+    auto load = [&](uint64_t t) {  // full tiles: into registers
+        const uint4* src = reinterpret_cast<const uint4*>(groups + t * kEncG24Threads);
+#pragma unroll
+        for (int u = 0; u < kPerV; u++) {
+            const int i = tid + u * kEncG24Threads;
+            if (i < kTileV) a[u] = __ldcs(src + i);
+        }
+    };
+    auto full = [&](uint64_t t) { return (t + 1) * kEncG24Threads <= count; };
+    uint32_t nbad = 0;
+    uint64_t t = blockIdx.x;
+    if (t < ntiles && full(t)) load(t);
+    for (; t < ntiles; t += gridDim.x) {
+        const uint32_t n = (uint32_t)min((uint64_t)kEncG24Threads, count - t * kEncG24Threads);
+        if (n == kEncG24Threads) {
+#pragma unroll
+            for (int u = 0; u < kPerV; u++) {
+                const int i = tid + u * kEncG24Threads;
+                if (i < kTileV) reinterpret_cast<uint4*>(s_rec)[i] = a[u];
+            }
+        } else {
+            const uint32_t* s32 = reinterpret_cast<const uint32_t*>(groups + t * kEncG24Threads);
+            for (uint32_t j = tid; j < n * kRecW; j += kEncG24Threads) s_rec[j] = __ldcs(s32 + j);
+        }
+        __syncthreads();
+        const uint64_t tn = t + gridDim.x;
+        if (tn < ntiles && full(tn)) load(tn);  // in flight while this tile is encoded
+        if ((uint32_t)tid < n) nbad += group_row24(s_rec + tid * kRecW, s_row + tid * 3) ? 0u : 1u;
+        __syncthreads();
+        uint4* dst = reinterpret_cast<uint4*>(out + t * kEncG24Threads * 24);
+        for (uint32_t j = tid; j < n * 3; j += kEncG24Threads) __stcs(dst + j, s_row[j]);
+        __syncthreads();
+    }
+    if (nbad) atomicAdd(&s_bad, nbad);
+    __syncthreads();
+    if (tid == 0 && bad && s_bad) atomicAdd(bad, s_bad);
+}
+
 cudaError_t launch_encode_groups(const void* groups, uint64_t count, int32_t n_models, int32_t D, int16_t* out,
                                  uint32_t* bad, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
+    if (D == 24 && n_models == 8 && (reinterpret_cast<uintptr_t>(out) & 15u) == 0 &&
+        (reinterpret_cast<uintptr_t>(groups) & 15u) == 0) {
+        const uint64_t blocks = (count + kEncG24Threads - 1) / kEncG24Threads;
+        const int grid = (int)(blocks < (uint64_t)nsm * 6 ? blocks : (uint64_t)nsm * 6);
+        encode_groups24_kernel<<<grid, kEncG24Threads, 0, st>>>(reinterpret_cast<const GroupRec*>(groups), count,
+                                                                 out, bad);
+        return cudaGetLastError();
+    }
     const uint64_t blocks = (count + kEncThreads - 1) / kEncThreads;
     const int grid = (int)(blocks < (uint64_t)nsm * 16 ? blocks : (uint64_t)nsm * 16);
     const size_t smem = (size_t)kEncThreads * D * sizeof(int16_t);

@@ -67,6 +67,18 @@ def test_encode_groups_bit_exact(ctx):
     assert bad == 0 and np.array_equal(x, x64)
     x, bad = ctx.encode_groups([[(3, 1, 2, 4, 0), (3, 2, 5, 4, 0)], [(2, 1, 9, 8, 0)]])
     assert bad == 1 and not x[0].any() and np.array_equal(x[1], oracle.encode(8, 4, [(2, 1, 9, 8, 0)]))
+    # invalid records scattered over full blocks and a ragged tail (1,000 = 3 x 256 + 232)
+    G = [g.slots for g in synth.instance_samples(1000, seed=16)]
+    invalid = {5: [(9, 1, 2, 4, 0)], 300: [(1, 1, 2, 4, 0), (1, 3, 4, 4, 0)], 999: [(0, 1, 2, 4, 0)]}
+    for i, g in invalid.items():
+        G[i] = g
+    x, bad = ctx.encode_groups(G)
+    assert bad == len(invalid)
+    for i in range(len(G)):
+        if i in invalid:
+            assert not x[i].any()
+        else:
+            assert np.array_equal(x[i], oracle.encode(8, 4, G[i])), i
 
 
 # ----------------------------------------------------------------- predict --
