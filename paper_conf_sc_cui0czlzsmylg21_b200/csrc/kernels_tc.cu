@@ -260,17 +260,24 @@ __device__ __forceinline__ void store_a1(uint32_t taddr, const uint32_t (&v)[kKM
 template <int FMT>
 struct TcPipe {
     TileIO X, Y;
-    uint32_t tC, lane_off, bar_id, ph;
+    uint32_t tCx, tCy, lane_off, bar_id, ph;  // bias constant chunk of X / Y (may be shared)
     uint64_t* bar;
     uint64_t db2, db3, db4;
     bool me[4];
 
+    // fused layout: 96 columns per group, one constant chunk at 480 for all
     __device__ __forceinline__ void init(uint32_t tbase, int g, int wq, uint64_t* mbar, uint64_t d2, uint64_t d3,
                                          uint64_t d4) {
         const uint32_t col = tbase + (uint32_t)g * 96u;
-        X = TileIO{col + 0, col + 64, col + 64};
-        Y = TileIO{col + 32, col + 80, col + 80};
-        tC = tbase + 480;
+        init_layout(TileIO{col + 0, col + 64, col + 64}, TileIO{col + 32, col + 80, col + 80}, tbase + 480,
+                    tbase + 480, g, wq, mbar, d2, d3, d4);
+    }
+    __device__ __forceinline__ void init_layout(const TileIO& x, const TileIO& y, uint32_t cx, uint32_t cy, int g,
+                                                int wq, uint64_t* mbar, uint64_t d2, uint64_t d3, uint64_t d4) {
+        X = x;
+        Y = y;
+        tCx = cx;
+        tCy = cy;
         lane_off = (uint32_t)(wq * 32) << 16;
         bar_id = 1 + (uint32_t)g;
         ph = 0;
@@ -310,20 +317,22 @@ struct TcPipe {
         constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 0 && TWO) {
-            issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tC, db, bar);
+            issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
         } else if (!TWO) {
-            issue_layer_asm<FMT, ID, CH>(X.d, X.a, tC, db, bar);
+            issue_layer_asm<FMT, ID, CH>(X.d, X.a, tCx, db, bar);
         } else {
             uint64_t d[5];
 #pragma unroll
             for (int i = 0; i < 5; i++) d[i] = db + (uint64_t)(i * (CH >> 4));
-            issue_layer_e<FMT>(X.d, X.a, tC, d, ID);
-            issue_layer_e<FMT>(Y.d, Y.a, tC, d, ID);
+            issue_layer_e<FMT>(X.d, X.a, tCx, d, ID);
+            issue_layer_e<FMT>(Y.d, Y.a, tCy, d, ID);
             mma_commit_elect(bar);
         }
     }
     // wait for the previous layer's MMAs, ReLU + pack into A, hand off, issue layer LAYER
-    template <int LAYER, bool TWO>
+    // CONST: also (re)write the per-tile constant chunks (layouts where the
+    // chunk shares the columns of the consumed layer-1 operand)
+    template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage() {
         wait();
         if (TWO) {
@@ -335,16 +344,25 @@ struct TcPipe {
 #pragma unroll
             for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(b[2 * c], b[2 * c + 1]);
             tmem_st16(Y.a + lane_off, h);
-            tmem_wait_st();
         } else {
-            hidden_epilogue<FMT>(X.d + lane_off, X.a + lane_off);
+            uint32_t a[32], h[16];
+            tmem_ld32(X.d + lane_off, a);
+#pragma unroll
+            for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(a[2 * c], a[2 * c + 1]);
+            tmem_st16(X.a + lane_off, h);
         }
+        if (CONST) {
+            uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
+            tmem_st8(tCx + lane_off, c8);
+            if (TWO) tmem_st8(tCy + lane_off, c8);
+        }
+        tmem_wait_st();
         if (handoff(me[LAYER])) issue_next<LAYER, TWO>();
     }
     // the three hidden stages, then wait for the output MMA and read y (column 0 of D)
-    template <bool TWO>
+    template <bool TWO, bool CONST = false>
     __device__ __forceinline__ void run_layers(uint32_t& yx, uint32_t& yy) {
-        stage<0, TWO>();
+        stage<0, TWO, CONST>();
         stage<1, TWO>();
         stage<2, TWO>();
         wait();
@@ -873,84 +891,37 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
     fence_after();
     const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
 
+    // per group 128 columns: X = D [0,32) U [32,64), Y = D [64,96) U [96,128);
+    // U holds the layer-1 operand, then A = U[0,16) and the constant chunk U[16,24)
     const uint32_t col = tbase + (uint32_t)g * 128u;
-    const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
     const TileIO X{col + 0, col + 32, col + 32}, Y{col + 64, col + 96, col + 96};
     const uint32_t r = (uint32_t)(tid & 127);
     const uint32_t sbase = smem_u32(smem);
-    constexpr uint32_t id32 = idesc_f16(FMT, 32), id16 = idesc_f16(FMT, 16);
-    uint64_t* barX = &bars[2 * g];
-    uint64_t* barY = &bars[2 * g + 1];
+    constexpr uint32_t id32 = idesc_f16(FMT, 32);
+    TcPipe<FMT> pp;
+    pp.init_layout(X, Y, col + 48, col + 112, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3),
+                   smem_desc(sbase + L.w4));
+    const uint32_t lane_off = pp.lane_off;
     uint64_t* tbX = &tbars[2 * g];
     uint64_t* tbY = &tbars[2 * g + 1];
-    uint32_t phX = 0, phY = 0, tphX = 0, tphY = 0;
+    uint32_t tphX = 0, tphY = 0;
     uint8_t* stX = smem + L.stage + (uint32_t)(2 * g) * stage_bytes;
     uint8_t* stY = stX + stage_bytes;
-    uint64_t d2[C::kNchHid], d3[C::kNchHid], d4[C::kNchOut];
-#pragma unroll
-    for (int i = 0; i < C::kNchHid; i++) {
-        d2[i] = smem_desc(sbase + L.w2 + i * kChunkBytesN32);
-        d3[i] = smem_desc(sbase + L.w3 + i * kChunkBytesN32);
-    }
-#pragma unroll
-    for (int i = 0; i < C::kNchOut; i++) d4[i] = smem_desc(sbase + L.w4 + i * kChunkBytesN16);
     const uint64_t d1base = smem_desc(sbase + L.b1);
-    const uint32_t idX = 1 + 2 * g, idY = 2 + 2 * g;
-    bool meX[4], meY[4];
-#pragma unroll
-    for (int p = 0; p < 4; p++) {
-        meX[p] = ((g + p) & 3) == wq;
-        meY[p] = ((g + 2 + p) & 3) == wq;
-    }
     const bool tma_ok = (row_bytes % 16u) == 0 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0;
 
-    auto handoff = [&](uint32_t bar_id, bool me) -> bool {
-        fence_before();
-        if (me) {
-            named_bar_sync(bar_id, 128);
-            fence_after();
-        } else {
-            named_bar_arrive(bar_id, 128);
-        }
-        return me;
-    };
-    auto issue_l1 = [&](const TileIO& T, uint64_t* bar) {
+    auto issue_l1 = [&](const TileIO& T) {
         for (int cb = 0; cb < nch; cb++)
             mma_ts_elect(T.d, T.a1 + 8 * cb, d1base + (uint64_t)(cb * (kChunkBytesN32 >> 4)), id32,
                          cb > 0 ? 1u : 0u);
         if (FMT == 1)
             for (int cb = 0; cb < nch; cb++)
                 mma_ts_elect(T.d, T.a1 + 8 * cb, d1base + (uint64_t)((nch + cb) * (kChunkBytesN32 >> 4)), id32, 1u);
-        mma_commit_elect(bar);
     };
-    // epilogue: ReLU + pack into A (= U[0,16)); the first hidden layer also
-    // (re)writes the constant chunk U[16,24) over the consumed layer-1 operand
-    auto stage = [&](const TileIO& T, uint64_t* bar, uint32_t& ph, const uint64_t* dl, uint32_t bar_id, bool me,
-                     uint32_t idesc, bool write_const) {
-        mbar_wait(bar, ph);
-        ph ^= 1u;
-        fence_after();
-        {
-            uint32_t rr[32];
-            tmem_ld32(T.d + lane_off, rr);
-            uint32_t h[16];
-#pragma unroll
-            for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(rr[2 * c], rr[2 * c + 1]);
-            tmem_st16(T.a + lane_off, h);
-            if (write_const) {
-                uint32_t c8[8] = {C::kOne2, 0, 0, 0, 0, 0, 0, 0};
-                tmem_st8(T.a + 16 + lane_off, c8);
-            }
-            tmem_wait_st();
-        }
-        if (handoff(bar_id, me)) {
-            issue_layer_e<FMT>(T.d, T.a, T.a + 16, dl, idesc);
-            mma_commit_elect(bar);
-        }
-    };
-    // feature rows of tile w: TMA bulk copy into the slot's stage (one elected thread)
+    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    // feature rows of tile w: TMA bulk copy into a slot's stage (lane 0 of the issuing warp)
     auto fetch = [&](uint64_t w, uint8_t* st, uint64_t* tb) {
-        if (!tma_ok || w >= (count + kTileM - 1) / kTileM) return;
+        if (!tma_ok || w >= n_tiles) return;
         if (lane == 0) {
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of `st`
             const uint64_t row0 = w * kTileM;
@@ -959,7 +930,7 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
             bulk_g2s(st, x + row0 * (uint64_t)D, nrows * row_bytes, tb);
         }
     };
-    // layer-1 operand row from the staged features: [x_hi (D), x_lo (D), 1, 1, 0...]
+    // layer-1 operand row from the staged features (no tcgen05.st wait)
     auto encode = [&](const TileIO& T, uint64_t w, uint8_t* st, uint64_t* tb, uint32_t& tph) {
         const uint64_t row0 = w * kTileM;
         const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
@@ -994,7 +965,6 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
                 for (int i = 0; i < 8; i++) a8[i] = av[8 * cb + i];
                 tmem_st8(T.a1 + lane_off + 8 * cb, a8);
             }
-            tmem_wait_st();
             return;
         }
         for (int cb = 0; cb < nch; cb++) {
@@ -1015,75 +985,37 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
             }
             tmem_st8(T.a1 + lane_off + 8 * cb, a);
         }
-        tmem_wait_st();
     };
-
-    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    // tiles w (and w + 1) enter the slots: encode, hand off, issue layer 1, refill the stages
+    auto enter = [&](uint64_t w, bool two) {
+        encode(X, w, stX, tbX, tphX);
+        if (two) encode(Y, w + 1, stY, tbY, tphY);
+        tmem_wait_st();
+        if (pp.handoff(pp.me[3])) {
+            issue_l1(X);
+            if (two) issue_l1(Y);
+            pp.commit();
+            fetch(w + 2, stX, tbX);  // every thread has consumed the stages (hand-off)
+            if (two) fetch(w + 3, stY, tbY);
+        }
+    };
     uint64_t wb, we;
     work_range(n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
     if (wb < we) {
-        bool xLive = true, yLive = wb + 1 < we;
         if (r == 0) {
             fetch(wb, stX, tbX);
-            if (yLive) fetch(wb + 1, stY, tbY);
+            if (wb + 1 < we) fetch(wb + 1, stY, tbY);
         }
-        // the issuing warp waits for all 128 threads (rows of the stage consumed),
-        // then refills the stage with the slot's next tile
-        encode(X, wb, stX, tbX, tphX);
-        if (handoff(idX, meX[3])) {
-            issue_l1(X, barX);
-            fetch(wb + 2 < we ? wb + 2 : ~0ull, stX, tbX);
-        }
-        if (yLive) {
-            encode(Y, wb + 1, stY, tbY, tphY);
-            if (handoff(idY, meY[3])) {
-                issue_l1(Y, barY);
-                fetch(wb + 3 < we ? wb + 3 : ~0ull, stY, tbY);
-            }
-        }
-        for (uint64_t w = wb; xLive; w += 2) {
-            stage(X, barX, phX, d2, idX, meX[0], id32, true);
-            if (yLive) stage(Y, barY, phY, d2, idY, meY[0], id32, true);
-            stage(X, barX, phX, d3, idX, meX[1], id32, false);
-            if (yLive) stage(Y, barY, phY, d3, idY, meY[1], id32, false);
-            stage(X, barX, phX, d4, idX, meX[2], id16, false);
-            if (yLive) stage(Y, barY, phY, d4, idY, meY[2], id16, false);
-            mbar_wait(barX, phX);
-            phX ^= 1u;
-            fence_after();
-            {
-                uint32_t yb;
-                tmem_ld1(X.d + lane_off, yb);
-                const uint64_t row = w * kTileM + r;
-                if (row < count) y[row] = __uint_as_float(yb);
-            }
-            xLive = w + 2 < we;
-            if (xLive) {
-                encode(X, w + 2, stX, tbX, tphX);
-                if (handoff(idX, meX[3])) {
-                    issue_l1(X, barX);
-                    fetch(w + 4 < we ? w + 4 : ~0ull, stX, tbX);
-                }
-            }
-            if (yLive) {
-                mbar_wait(barY, phY);
-                phY ^= 1u;
-                fence_after();
-                {
-                    uint32_t yb;
-                    tmem_ld1(Y.d + lane_off, yb);
-                    const uint64_t row = (w + 1) * kTileM + r;
-                    if (row < count) y[row] = __uint_as_float(yb);
-                }
-                yLive = w + 3 < we;
-                if (yLive) {
-                    encode(Y, w + 3, stY, tbY, tphY);
-                    if (handoff(idY, meY[3])) {
-                        issue_l1(Y, barY);
-                        fetch(w + 5 < we ? w + 5 : ~0ull, stY, tbY);
-                    }
-                }
-            }
+        enter(wb, wb + 1 < we);
+        for (uint64_t w = wb; w < we; w += 2) {
+            uint32_t yx, yy = 0;
+            const bool two = w + 1 < we;
+            if (two) pp.template run_layers<true, true>(yx, yy);
+            else pp.template run_layers<false, true>(yx, yy);
+            const uint64_t row = w * kTileM + r;
+            if (row < count) y[row] = __uint_as_float(yx);
+            if (two && row + kTileM < count) y[row + kTileM] = __uint_as_float(yy);
+            if (w + 2 < we) enter(w + 2, w + 3 < we);
         }
     }
     fence_before();

@@ -207,7 +207,7 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
 // the MMAs of one layer for TWO tiles (same B operand) and ONE commit
 template <int FMT, uint32_t IDESC, uint32_t CHUNK>
 __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
-                                                 uint32_t tC, uint64_t dbase, uint64_t* bar) {
+                                                 uint32_t tCx, uint32_t tCy, uint64_t dbase, uint64_t* bar) {
     static_assert(FMT == 0, "lock-step pair issue: fp16 layout");
     constexpr uint32_t U = CHUNK >> 4;
     asm volatile(
@@ -227,11 +227,11 @@ __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uin
         "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%4], d2, %9, pt;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %5, %9, pf;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %9, pt;\n\t"
-        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%4], d2, %9, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%10], d2, %9, pt;\n\t"
         "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t"
         "}" ::"r"(tDx),
-        "r"(tAx), "r"(tDy), "r"(tAy), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
-        "n"((uint64_t)(2 * U)), "n"(IDESC)
+        "r"(tAx), "r"(tDy), "r"(tAy), "r"(tCx), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
+        "n"((uint64_t)(2 * U)), "n"(IDESC), "r"(tCy)
         : "memory");
 }
 
