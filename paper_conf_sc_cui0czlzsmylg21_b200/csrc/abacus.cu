@@ -28,6 +28,14 @@
 
 using namespace abacus;
 
+// one decision of a batch after a1 (host): its grid, threshold, size and space
+struct BatchIn {
+    abacus_grid_t g;
+    float H;
+    uint32_t chain;
+    uint64_t T;
+};
+
 struct abacus_ctx {
     int device = 0;
     int nsm = 0;
@@ -53,8 +61,6 @@ struct abacus_ctx {
     TcWeights tw[2]{};
     // batched decisions: staging and device buffers, grown on demand (first call of a larger batch)
     int32_t batch_cap = 0;
-    BatchDec* h_decs = nullptr;  // pinned
-    SegP* h_segs = nullptr;      // pinned, kMaxSegBatch per decision
     Result* h_out = nullptr;     // pinned
     BatchDec* d_decs = nullptr;
     SegP* d_segs = nullptr;
@@ -63,6 +69,9 @@ struct abacus_ctx {
     Result* d_out = nullptr;
     std::vector<int32_t> b_order;  // [4 n] headroom order per decision
     std::vector<float> b_H;
+    BatchIn* h_in = nullptr;       // pinned: a1 results (grid, H, T, space) per decision
+    BatchIn* d_in = nullptr;
+    uint64_t* d_pairs = nullptr;   // [n] tile pairs per decision, then [n] = total
     // NEXT-3 training state (abacus_train_begin)
     bool training = false;
     abacus_adam_t adam{};
@@ -129,7 +138,7 @@ const NcclApi& nccl() {
         if (e__ != cudaSuccess) return fail(ctx, ABACUS_E_CUDA, "%s: %s", #call, cudaGetErrorString(e__)); \
     } while (0)
 
-FastDiv make_fastdiv(uint32_t d) {
+__host__ __device__ FastDiv make_fastdiv(uint32_t d) {
     FastDiv f{};
     f.d = d;
     uint32_t p = 0;
@@ -170,7 +179,7 @@ int validate_grid(abacus_ctx* c, const abacus_grid_t* g, uint64_t* T_out) {
 }
 
 // ---- plans ------------------------------------------------------------------
-void fill_strides(Plan& P) {
+__host__ __device__ void fill_strides(Plan& P) {
     uint64_t b = 1;
     for (int j = kKMax - 1; j >= 0; j--) {
         P.slot[j].tstride = b;
@@ -179,7 +188,7 @@ void fill_strides(Plan& P) {
     }
 }
 
-void fill_slots(Plan& P, const abacus_grid_t* g) {
+__host__ __device__ void fill_slots(Plan& P, const abacus_grid_t* g) {
     for (int j = 0; j < kKMax; j++) {
         SlotP& s = P.slot[j];
         if (j < g->k) {
@@ -195,7 +204,7 @@ void fill_slots(Plan& P, const abacus_grid_t* g) {
     fill_strides(P);
 }
 
-void finish_box(SegP& s) {
+__host__ __device__ void finish_box(SegP& s) {
     uint64_t b = 1;
     for (int j = kKMax - 1; j >= 0; j--) {
         s.bstride[j] = b;
@@ -205,18 +214,18 @@ void finish_box(SegP& s) {
     }
 }
 
-uint64_t box_size(const SegP& s) {
+__host__ __device__ uint64_t box_size(const SegP& s) {
     uint64_t b = 1;
     for (int j = 0; j < kKMax; j++) b *= s.cnt[j];
     return b;
 }
 
 // whole grid as one box: digits = grid digits (encode / select kernels)
-Plan plan_whole_grid(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T) {
+__host__ __device__ Plan plan_whole_grid(int32_t n_models, int32_t D, const abacus_grid_t* g, uint64_t T) {
     Plan P{};
     P.k = g->k;
-    P.n_models = c->n_models;
-    P.D = c->D;
+    P.n_models = n_models;
+    P.D = D;
     P.mode = kModeGrid;
     P.T = T;
     fill_slots(P, g);
@@ -236,7 +245,7 @@ Plan plan_whole_grid(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T) {
 // number of elements of segment box `s` with index < a.  Per SLOT j the box
 // digit set is: present -> [dlo_j, dlo_j + cnt_j), absent -> {0}; elements
 // are ordered lexicographically by slot (index order).
-uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const uint32_t* scnt, uint64_t a) {
+__host__ __device__ uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const uint32_t* scnt, uint64_t a) {
     if (a >= P.T) return box_size(s);
     uint32_t dig[kKMax] = {0, 0, 0, 0};
     uint64_t rem = a;
@@ -254,7 +263,7 @@ uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const u
         bool inside;
         if (present) {
             const int64_t b = (int64_t)dig[j] - (int64_t)dlo[j];
-            below = (uint64_t)std::min<int64_t>(std::max<int64_t>(b, 0), (int64_t)scnt[j]);
+            below = (uint64_t)(b < 0 ? 0 : (b > (int64_t)scnt[j] ? (int64_t)scnt[j] : b));
             inside = dig[j] >= dlo[j] && dig[j] < dlo[j] + scnt[j];
         } else {
             below = dig[j] > 0 ? 1 : 0;
@@ -268,7 +277,7 @@ uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const u
 
 // Lay the per-slot box (scnt, sistride) out in digit order: slots with
 // cnt == 1 first, then the varying ones in slot order (common.cuh).
-void order_digits(SegP& s, int k, const uint32_t* scnt, const uint64_t* sistride) {
+__host__ __device__ void order_digits(SegP& s, int k, const uint32_t* scnt, const uint64_t* sistride) {
     int d = 0;
     for (int pass = 0; pass < 2; pass++)
         for (int j = 0; j < kKMax; j++) {
@@ -283,7 +292,7 @@ void order_digits(SegP& s, int k, const uint32_t* scnt, const uint64_t* sistride
     s.fast_carry = s.cnt[kKMax - 1] >= (uint32_t)kTileM ? 1u : 0u;
 }
 
-void set_positions(const Plan& P, SegP& s) {
+__host__ __device__ void set_positions(const Plan& P, SegP& s) {
     for (int j = 0; j < kKMax; j++) {
         s.pos[j] = -1;
         if (j >= P.k || !((s.mask >> j) & 1u)) continue;
@@ -295,12 +304,12 @@ void set_positions(const Plan& P, SegP& s) {
 }
 
 // GRID / sweep: one segment per presence pattern, restricted to [first, last)
-Plan plan_grid_segments(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T, uint64_t first, uint64_t last,
-                        float H) {
+__host__ __device__ Plan plan_grid_segments(int32_t n_models, int32_t D, const abacus_grid_t* g, uint64_t T,
+                                            uint64_t first, uint64_t last, float H) {
     Plan P{};
     P.k = g->k;
-    P.n_models = c->n_models;
-    P.D = c->D;
+    P.n_models = n_models;
+    P.D = D;
     P.mode = kModeGrid;
     P.T = T;
     P.H = H;
@@ -357,11 +366,11 @@ Plan plan_grid_segments(const abacus_ctx* c, const abacus_grid_t* g, uint64_t T,
 
 // CHAIN (decision mode): u = 0 critical only; block j: slots < j full, slot j
 // grows op by op, later slots absent
-Plan plan_chain(const abacus_ctx* c, const abacus_grid_t* g, float H, uint64_t* n_out) {
+__host__ __device__ Plan plan_chain(int32_t n_models, int32_t D, const abacus_grid_t* g, float H, uint64_t* n_out) {
     Plan P{};
     P.k = g->k;
-    P.n_models = c->n_models;
-    P.D = c->D;
+    P.n_models = n_models;
+    P.D = D;
     P.mode = kModeChain;
     P.H = H;
     P.want_y0 = 1;
@@ -628,21 +637,72 @@ unsigned long long* trace_ptr() { return g_trace_ptr; }
 // ============================================================================
 // C ABI
 // ============================================================================
+// ---- batched decisions: planning on the device -----------------------------
+// One thread per decision runs the same planner as the single-round path
+// (plan_grid_segments / plan_chain, __host__ __device__) and writes the
+// decision's header and segments (fixed slots of kMaxSegBatch) in place.
+__global__ void batch_plan_kernel(const BatchIn* __restrict__ in, int32_t n, int32_t n_models, int32_t D,
+                                  BatchDec* __restrict__ decs, SegP* __restrict__ segs, uint64_t* __restrict__ pairs) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const BatchIn b = in[i];
+    uint64_t n_eval = 0;
+    Plan P = b.chain ? plan_chain(n_models, D, &b.g, b.H, &n_eval) : plan_grid_segments(n_models, D, &b.g, b.T, 0, b.T, b.H);
+    if (!b.chain) n_eval = P.n_eval;
+    BatchDec& bd = decs[i];
+    bd.h = static_cast<const PlanHdr&>(P);
+    bd.h.want_y0 = 1;
+    bd.h.n_eval = n_eval;
+    bd.h.mapped = nullptr;
+    bd.h.trace = nullptr;
+    bd.seg0 = (uint32_t)(kMaxSegBatch * i);
+    for (int sg = 0; sg < P.n_seg && sg < kMaxSegBatch; sg++) segs[(size_t)kMaxSegBatch * i + sg] = P.seg[sg];
+    pairs[i] = (P.n_tiles + 1) / 2;  // tiles padded to pairs (lock-step slots never straddle decisions)
+}
+
+// exclusive prefix sum of the tile pairs -> decs[i].pair0, pairs[n] = total (one block)
+constexpr int kScanThreads = 1024;
+__global__ void __launch_bounds__(kScanThreads) batch_scan_kernel(BatchDec* __restrict__ decs,
+                                                                  uint64_t* __restrict__ pairs, int32_t n) {
+    __shared__ uint64_t s[kScanThreads];
+    const int t = threadIdx.x;
+    const int per = (n + kScanThreads - 1) / kScanThreads;
+    const int i0 = t * per, i1 = min(n, i0 + per);
+    uint64_t sum = 0;
+    for (int i = i0; i < i1; i++) sum += pairs[i];
+    s[t] = sum;
+    __syncthreads();
+    for (int off = 1; off < kScanThreads; off <<= 1) {  // inclusive Hillis-Steele scan
+        const uint64_t v = t >= off ? s[t - off] : 0;
+        __syncthreads();
+        s[t] += v;
+        __syncthreads();
+    }
+    uint64_t run = s[t] - sum;
+    for (int i = i0; i < i1; i++) {
+        decs[i].pair0 = run;
+        run += pairs[i];
+    }
+    if (t == kScanThreads - 1) pairs[n] = s[t];
+}
+
 namespace {
 int grow_batch(abacus_ctx* c, int32_t n) {
     if (n <= c->batch_cap) return ABACUS_OK;
     int32_t cap = c->batch_cap ? c->batch_cap : 256;
     while (cap < n) cap *= 2;
-    if (c->h_decs) cudaFreeHost(c->h_decs);
-    if (c->h_segs) cudaFreeHost(c->h_segs);
     if (c->h_out) cudaFreeHost(c->h_out);
     cudaFree(c->d_decs);
     cudaFree(c->d_segs);
     cudaFree(c->d_acc);
     cudaFree(c->d_y0);
     cudaFree(c->d_out);
-    c->h_decs = nullptr;
-    c->h_segs = nullptr;
+    if (c->h_in) cudaFreeHost(c->h_in);
+    cudaFree(c->d_in);
+    cudaFree(c->d_pairs);
+    c->h_in = nullptr;
+    c->d_in = nullptr;
+    c->d_pairs = nullptr;
     c->h_out = nullptr;
     c->d_decs = nullptr;
     c->d_segs = nullptr;
@@ -651,16 +711,18 @@ int grow_batch(abacus_ctx* c, int32_t n) {
     c->d_out = nullptr;
     c->batch_cap = 0;
     const size_t nd = (size_t)cap, ns = (size_t)cap * kMaxSegBatch;
-    CUDA_TRY(c, cudaHostAlloc(&c->h_decs, nd * sizeof(BatchDec), cudaHostAllocDefault));
-    CUDA_TRY(c, cudaHostAlloc(&c->h_segs, ns * sizeof(SegP), cudaHostAllocDefault));
     CUDA_TRY(c, cudaHostAlloc(&c->h_out, nd * sizeof(Result), cudaHostAllocDefault));
     CUDA_TRY(c, cudaMalloc(&c->d_decs, nd * sizeof(BatchDec)));
     CUDA_TRY(c, cudaMalloc(&c->d_segs, ns * sizeof(SegP)));
     CUDA_TRY(c, cudaMalloc(&c->d_acc, nd * sizeof(BatchAcc)));
     CUDA_TRY(c, cudaMalloc(&c->d_y0, nd * sizeof(float)));
     CUDA_TRY(c, cudaMalloc(&c->d_out, nd * sizeof(Result)));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_in, nd * sizeof(BatchIn), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaMalloc(&c->d_in, nd * sizeof(BatchIn)));
+    CUDA_TRY(c, cudaMalloc(&c->d_pairs, (nd + 1) * sizeof(uint64_t)));
     c->b_order.resize(4 * nd);
     c->b_H.resize(nd);
+
     c->batch_cap = cap;
     return ABACUS_OK;
 }
@@ -740,14 +802,15 @@ void abacus_destroy(abacus_ctx* c) {
     cudaFree(c->d_blob[0]);
     cudaFree(c->d_blob[1]);
     if (c->host_result) cudaFreeHost(c->host_result);
-    if (c->h_decs) cudaFreeHost(c->h_decs);
-    if (c->h_segs) cudaFreeHost(c->h_segs);
     if (c->h_out) cudaFreeHost(c->h_out);
     cudaFree(c->d_decs);
     cudaFree(c->d_segs);
     cudaFree(c->d_acc);
     cudaFree(c->d_y0);
     cudaFree(c->d_out);
+    if (c->h_in) cudaFreeHost(c->h_in);
+    cudaFree(c->d_in);
+    cudaFree(c->d_pairs);
     cudaFree(c->t_p);
     cudaFree(c->t_m);
     cudaFree(c->t_v);
@@ -831,7 +894,7 @@ int abacus_encode_candidates(abacus_ctx* c, const abacus_grid_t* grid, uint64_t 
     if (first > T || count > T - first) return fail(c, ABACUS_E_INVALID, "range beyond T=%llu", (unsigned long long)T);
     if (count && !d_features) return fail(c, ABACUS_E_INVALID, "d_features is NULL");
     CUDA_TRY(c, cudaSetDevice(c->device));
-    const Plan P = plan_whole_grid(c, grid, T);
+    const Plan P = plan_whole_grid(c->n_models, c->D, grid, T);
     CUDA_TRY(c, launch_encode_grid(P, first, count, d_features, c->nsm, pick_stream(c, stream)));
     if (count) c->launches++;
     return ABACUS_OK;
@@ -881,7 +944,7 @@ int abacus_select_group(abacus_ctx* c, const abacus_grid_t* grid, uint64_t first
     if (!d_best_key || (count && !d_latency_ms)) return fail(c, ABACUS_E_INVALID, "NULL device buffer");
     if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
     CUDA_TRY(c, cudaSetDevice(c->device));
-    const Plan P = plan_whole_grid(c, grid, T);
+    const Plan P = plan_whole_grid(c->n_models, c->D, grid, T);
     CUDA_TRY(c, launch_select(P, first, count, d_latency_ms, headroom_ms, d_best_key, c->nsm,
                               pick_stream(c, stream)));
     if (count) c->launches++;
@@ -906,9 +969,9 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
     Plan P;
     uint64_t n_eval = 0;
     if (chain) {
-        P = plan_chain(c, &g, H, &n_eval);
+        P = plan_chain(c->n_models, c->D, &g, H, &n_eval);
     } else {
-        P = plan_grid_segments(c, &g, T, 0, T, H);
+        P = plan_grid_segments(c->n_models, c->D, &g, T, 0, T, H);
         n_eval = P.n_eval;
     }
     P.want_y0 = 1;
@@ -945,55 +1008,55 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     CUDA_TRY(c, cudaSetDevice(c->device));
     int rc = grow_batch(c, n);
     if (rc) return rc;
-    uint64_t pair = 0;
-    uint32_t seg = 0, maxcnt = 0;
+    // a1 and validation on the host, in order (the first failing decision is
+    // reported and nothing is launched); everything after runs on the device
+    uint64_t pairs_ub = 0;
+    uint32_t maxcnt = 0;
     for (int32_t i = 0; i < n; i++) {
-        int32_t* order = &c->b_order[4 * (size_t)i];
-        abacus_grid_t g{};
-        rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], order, &c->b_H[i], &g);
+        BatchIn& b = c->h_in[i];
+        rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], &c->b_order[4 * (size_t)i],
+                            &c->b_H[i], &b.g);
         if (rc) {
             c->err = "decision " + std::to_string(i) + ": " + c->err;
             return rc;
         }
-        uint64_t T = 0;
-        validate_grid(c, &g, &T);
-        const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
-        uint64_t n_eval = 0;
-        Plan P = chain ? plan_chain(c, &g, c->b_H[i], &n_eval) : plan_grid_segments(c, &g, T, 0, T, c->b_H[i]);
-        if (!chain) n_eval = P.n_eval;
-        if (P.n_seg > kMaxSegBatch) return fail(c, ABACUS_E_INVALID, "decision %d: %d segments", i, P.n_seg);
-        BatchDec& bd = c->h_decs[i];
-        bd.h = static_cast<const PlanHdr&>(P);
-        bd.h.want_y0 = 1;
-        bd.h.n_eval = n_eval;
-        bd.h.mapped = nullptr;
-        bd.h.trace = nullptr;
-        bd.pair0 = pair;
-        bd.seg0 = seg;
-        for (int s = 0; s < P.n_seg; s++) {
-            c->h_segs[seg + s] = P.seg[s];
-            for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
+        validate_grid(c, &b.g, &b.T);
+        b.H = c->b_H[i];
+        b.chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && b.T > grid_budget);
+        // bounds the device plan cannot exceed: the widest segment digit (selects the
+        // split layer-1 layout) and the tile pairs (<= one partial tile per segment)
+        uint64_t n_cand = b.T;
+        if (b.chain) {
+            n_cand = 1;
+            for (int j = 1; j < b.g.k; j++) n_cand += (uint64_t)(b.g.slot[j].end_hi - b.g.slot[j].start_op + 1);
         }
-        seg += (uint32_t)P.n_seg;
-        pair += (P.n_tiles + 1) / 2;
+        for (int j = b.chain ? 1 : 0; j < b.g.k; j++) {  // CHAIN: the critical slot's digit is fixed
+            const abacus_slot_t& sl = b.g.slot[j];
+            const uint32_t w = (uint32_t)(sl.end_hi - (b.chain ? sl.start_op : sl.end_lo) + 1);
+            maxcnt = w > maxcnt ? w : maxcnt;
+        }
+        pairs_ub += (n_cand / kTileM + kMaxSegBatch + 1) / 2 + 1;
     }
     cudaStream_t st = c->stream;
-    CUDA_TRY(c, cudaMemcpyAsync(c->d_decs, c->h_decs, (size_t)n * sizeof(BatchDec), cudaMemcpyHostToDevice, st));
-    CUDA_TRY(c, cudaMemcpyAsync(c->d_segs, c->h_segs, (size_t)seg * sizeof(SegP), cudaMemcpyHostToDevice, st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->d_in, c->h_in, (size_t)n * sizeof(BatchIn), cudaMemcpyHostToDevice, st));
+    batch_plan_kernel<<<(n + 127) / 128, 128, 0, st>>>(c->d_in, n, c->n_models, c->D, c->d_decs, c->d_segs,
+                                                       c->d_pairs);
+    batch_scan_kernel<<<1, kScanThreads, 0, st>>>(c->d_decs, c->d_pairs, n);
+    CUDA_TRY(c, cudaGetLastError());
+    c->launches += 2;
     CUDA_TRY(c, cudaMemsetAsync(c->d_acc, 0, (size_t)n * sizeof(BatchAcc), st));
     CUDA_TRY(c, cudaMemsetAsync(c->d_y0, 0xFF, (size_t)n * sizeof(float), st));  // NaN
     if (c->timed) cudaEventRecord(c->ev0, st);
     const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
-    cudaError_t e = launch_batch_tc(c->d_decs, c->d_segs, n, pair, maxcnt, c->D, c->tw[fmt], c->d_w1b1, c->d_acc,
-                                    c->d_y0, c->d_out, c->nsm, st);
+    cudaError_t e = launch_batch_tc(c->d_decs, c->d_segs, n, c->d_pairs + n, pairs_ub, maxcnt, c->D, c->tw[fmt],
+                                    c->d_w1b1, c->d_acc, c->d_y0, c->d_out, c->nsm, st);
     if (c->timed) cudaEventRecord(c->ev1, st);
     if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "batched search launch: %s", cudaGetErrorString(e));
     c->launches += 2;
     CUDA_TRY(c, cudaMemcpyAsync(c->h_out, c->d_out, (size_t)n * sizeof(Result), cudaMemcpyDeviceToHost, st));
     CUDA_TRY(c, cudaStreamSynchronize(st));
     for (int32_t i = 0; i < n; i++)
-        out[i] = assemble_decision(c->h_out[i], &c->b_order[4 * (size_t)i], k[i], c->b_H[i],
-                                   c->h_decs[i].h.n_eval);
+        out[i] = assemble_decision(c->h_out[i], &c->b_order[4 * (size_t)i], k[i], c->b_H[i], c->h_out[i].evaluated);
     return ABACUS_OK;
 }
 
@@ -1009,7 +1072,7 @@ int abacus_search_mway(abacus_ctx* c, const abacus_query_t* q, int32_t k, double
     int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g);
     if (rc) return rc;
     uint64_t n_chain = 0;
-    Plan P = plan_chain(c, &g, H, &n_chain);
+    Plan P = plan_chain(c->n_models, c->D, &g, H, &n_chain);
     P.mapped = c->dev_result;
     P.seq = next_seq(c);
     CUDA_TRY(c, cudaSetDevice(c->device));
@@ -1048,7 +1111,7 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     if (first > T || count > T - first) return fail(c, ABACUS_E_INVALID, "range beyond T");
     if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
     CUDA_TRY(c, cudaSetDevice(c->device));
-    Plan P = plan_grid_segments(c, grid, T, first, first + count, headroom_ms);
+    Plan P = plan_grid_segments(c->n_models, c->D, grid, T, first, first + count, headroom_ms);
     const uint32_t seq = next_seq(c);
     P.mapped = nccl_comm ? nullptr : c->dev_result;  // with a combine, the finalize kernel publishes
     P.seq = seq;

@@ -45,7 +45,8 @@ cudaError_t launch_finalize_gather(Scratch* S, int nranks, Result* mapped, uint3
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out);
-// batched decisions: d_decs[n_dec] and d_segs on the device; acc/y0s zeroed / NaN-filled by the caller
+// batched decisions: d_decs[n_dec] and d_segs planned on the device, *d_n_pairs their tile-pair total
+// (pairs_ub >= it sizes the grid); acc/y0s zeroed / NaN-filled by the caller
 // NEXT-3: one Adam step on a minibatch (kernels_train.cu)
 struct TrainArgs {
     float* p;                 // parameters (device, updated in place)
@@ -67,9 +68,9 @@ struct TrainArgs {
 int train_n_params(int D);
 cudaError_t launch_train_step(const TrainArgs& A, cudaStream_t st);
 
-cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, uint64_t n_pairs,
-                            uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1, BatchAcc* acc,
-                            float* y0s, Result* out, int nsm, cudaStream_t st);
+cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, const uint64_t* d_n_pairs,
+                            uint64_t pairs_ub, uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1,
+                            BatchAcc* acc, float* y0s, Result* out, int nsm, cudaStream_t st);
 cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
                               float* y, int nsm, cudaStream_t st);
 

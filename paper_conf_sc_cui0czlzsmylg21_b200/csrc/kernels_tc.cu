@@ -567,7 +567,7 @@ __host__ __device__ inline TcSmem batch_smem_layout(int D, int ng, uint32_t* pla
 template <int FMT, bool SPLIT, int NG>
 __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const BatchDec* __restrict__ decs,
                                                                      const SegP* __restrict__ segs, int32_t n_dec,
-                                                                     uint64_t n_pairs, int32_t D,
+                                                                     const uint64_t* __restrict__ n_pairs_dev, int32_t D,
                                                                      const __grid_constant__ TcParams TP,
                                                                      const float* __restrict__ w1b1, BatchAcc* acc,
                                                                      float* y0s) {
@@ -605,6 +605,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
         pp.issue_l1(T, d1base + (uint64_t)((uint32_t)su * kSegStep));
     };
 
+    const uint64_t n_pairs = *n_pairs_dev;  // written by the planning kernels
     uint64_t pb, pe;
     work_range(n_pairs, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, pb, pe);
     if (pb < pe) {
@@ -1067,33 +1068,33 @@ cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b
 }
 
 template <int FMT, bool SPLIT>
-static cudaError_t launch_batch_fmt(const BatchDec* decs, const SegP* segs, int32_t n_dec, uint64_t n_pairs,
-                                    int32_t D, const TcParams& tp, const float* w1b1, BatchAcc* acc, float* y0s,
-                                    int nsm, cudaStream_t st) {
+static cudaError_t launch_batch_fmt(const BatchDec* decs, const SegP* segs, int32_t n_dec, const uint64_t* n_pairs,
+                                    uint64_t pairs_ub, int32_t D, const TcParams& tp, const float* w1b1,
+                                    BatchAcc* acc, float* y0s, int nsm, cudaStream_t st) {
     uint32_t plans_off;
     const TcSmem L = batch_smem_layout<FMT>(D, kFusedNG, &plans_off);
     auto kern = fused_batch_tc_kernel<FMT, SPLIT, kFusedNG>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
-    uint64_t g = (n_pairs + kFusedNG - 1) / kFusedNG;
+    uint64_t g = (pairs_ub + kFusedNG - 1) / kFusedNG;  // the exact count is only known on the device
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     kern<<<(int)g, kFusedNG * 128, L.total, st>>>(decs, segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s);
     return cudaGetLastError();
 }
 
-cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, uint64_t n_pairs,
-                            uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1, BatchAcc* acc,
-                            float* y0s, Result* out, int nsm, cudaStream_t st) {
+cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, const uint64_t* d_n_pairs,
+                            uint64_t pairs_ub, uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1,
+                            BatchAcc* acc, float* y0s, Result* out, int nsm, cudaStream_t st) {
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
     const bool split = need_split(TW.fmt, maxcnt);
     cudaError_t e;
+#define ABACUS_BATCH_ARGS d_decs, d_segs, n_dec, d_n_pairs, pairs_ub, D, tp, w1b1, acc, y0s, nsm, st
     if (TW.fmt == 0)
-        e = split ? launch_batch_fmt<0, true>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st)
-                  : launch_batch_fmt<0, false>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st);
+        e = split ? launch_batch_fmt<0, true>(ABACUS_BATCH_ARGS) : launch_batch_fmt<0, false>(ABACUS_BATCH_ARGS);
     else
-        e = split ? launch_batch_fmt<1, true>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st)
-                  : launch_batch_fmt<1, false>(d_decs, d_segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s, nsm, st);
+        e = split ? launch_batch_fmt<1, true>(ABACUS_BATCH_ARGS) : launch_batch_fmt<1, false>(ABACUS_BATCH_ARGS);
+#undef ABACUS_BATCH_ARGS
     if (e != cudaSuccess) return e;
     const int threads = 256;
     const int blocks = (int)(((int64_t)n_dec * 32 + threads - 1) / threads);
