@@ -108,6 +108,9 @@ def lib():
         L.orc_sweep.argtypes = [C.c_int32, C.c_int32, P(C.c_float), C.c_int32, P(GSlot), C.c_double,
                                 C.c_uint64, C.c_uint64, C.c_double, C.c_int32, P(C.c_double),
                                 P(C.c_int16), P(C.c_int32), P(SweepResult)]
+        L.orc_sweep_shell.restype = C.c_int32
+        L.orc_sweep_shell.argtypes = [C.c_int32, C.c_int32, P(C.c_float), C.c_int32, P(GSlot), C.c_double,
+                                      C.c_int32, C.c_double, C.c_int32, P(SweepResult)]
         L.orc_search.restype = C.c_int32
         L.orc_search.argtypes = [C.c_int32, C.c_int32, P(C.c_int32), P(C.c_float), P(QueryC),
                                  C.c_int32, C.c_double, C.c_double, C.c_int32, C.c_uint64,
@@ -236,6 +239,17 @@ def sweep(params, grid, H, first=0, count=None, eps=1e-4, n_models=8, kmax=4, em
     if rc != 0:
         raise ValueError("orc_sweep rejected the grid")
     return r, y, x, o
+
+
+def sweep_shell(params, grid, H, nsum_min, eps=1e-4, n_models=8, kmax=4, emu_flags=0):
+    """The whole grid restricted to candidates with sum_n >= nsum_min (orc_sweep_shell)."""
+    p, pp = _f32(params)
+    r = SweepResult()
+    rc = lib().orc_sweep_shell(n_models, kmax, pp, len(grid), _gslots(grid), float(H), int(nsum_min), eps,
+                               emu_flags, C.byref(r))
+    if rc != 0:
+        raise ValueError("orc_sweep_shell rejected the grid")
+    return r
 
 
 def search(params, queries, now, inflight, space=0, budget=2**40, eps=1e-4, n_models=8, kmax=4,

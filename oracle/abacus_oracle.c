@@ -293,6 +293,8 @@ typedef struct {
     int16_t* x_out;
     int32_t* ope_out;
     orc_sweep_result_t* r;
+    int32_t nsum_min;             /* orc_sweep_shell: visit only sum_n >= nsum_min */
+    int32_t rest_max[ORC_KMAX + 1];
 } orc_sweep_state_t;
 
 static void orc_visit(orc_sweep_state_t* st) {
@@ -354,6 +356,67 @@ static void orc_rec(orc_sweep_state_t* st, int32_t j) {
         else st->ope[j] = s->end_lo + dgt;
         orc_rec(st, j + 1);
     }
+}
+
+/* The same enumeration restricted to the candidates with sum_n >= nsum_min:
+ * a subtree whose largest reachable sum_n (the ops taken so far plus every
+ * later slot at its largest end op) is below the bound is skipped whole, its
+ * indices counted.  Used to check a huge sweep's answer: every key above it
+ * has a sum_n at least the answer's (reading c12), so the check needs only
+ * this shell (SURVEY.md §8(c) "Large sweeps"). */
+static void orc_rec_shell(orc_sweep_state_t* st, int32_t j, int32_t psum) {
+    if (j == st->k) {
+        orc_visit(st);
+        st->counter++;
+        return;
+    }
+    const orc_gslot_t* s = &st->g[j];
+    int32_t radix = s->allow_absent + (s->end_hi - s->end_lo + 1);
+    for (int32_t dgt = 0; dgt < radix; dgt++) {
+        int32_t ope;
+        if (s->allow_absent) ope = dgt == 0 ? 0 : s->end_lo + dgt - 1;
+        else ope = s->end_lo + dgt;
+        int32_t n_j = ope == 0 ? 0 : ope - s->start_op + 1;
+        if (psum + n_j + st->rest_max[j + 1] < st->nsum_min) {
+            st->counter += st->sub[j];
+            continue;
+        }
+        st->ope[j] = ope;
+        orc_rec_shell(st, j + 1, psum + n_j);
+    }
+}
+
+int32_t orc_sweep_shell(int32_t n_models, int32_t kmax, const float* prm, int32_t k, const orc_gslot_t* g,
+                        double H, int32_t nsum_min, double eps, int32_t emu_flags, orc_sweep_result_t* r) {
+    orc_sweep_state_t st;
+    if (k < 1 || k > kmax || k > ORC_KMAX) return -1;
+    memset(&st, 0, sizeof(st));
+    memset(r, 0, sizeof(*r));
+    r->y0 = NAN;
+    r->best_y = NAN;
+    st.n_models = n_models;
+    st.kmax = kmax;
+    st.d = n_models + 4 * kmax;
+    st.k = k;
+    st.flags = emu_flags;
+    st.prm = prm;
+    st.g = g;
+    st.H = H;
+    st.eps = eps;
+    st.first = 0;
+    st.last = UINT64_MAX;
+    st.r = r;
+    st.nsum_min = nsum_min;
+    st.rest_max[k] = 0;
+    for (int32_t j = k - 1; j >= 0; j--) st.rest_max[j] = st.rest_max[j + 1] + (g[j].end_hi - g[j].start_op + 1);
+    for (int32_t j = 0; j < k; j++) {
+        uint64_t sz = 1;
+        for (int32_t i = j + 1; i < k; i++)
+            sz *= (uint64_t)(g[i].allow_absent + g[i].end_hi - g[i].end_lo + 1);
+        st.sub[j] = sz;
+    }
+    orc_rec_shell(&st, 0, 0);
+    return 0;
 }
 
 /* grid size T = prod radix; 0 if invalid */

@@ -254,6 +254,40 @@ def test_search_grid_cfg4_fullsize_linear_closed_form(prec):
         c.close()
 
 
+_SHELL = {}
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_search_grid_cfg4_fullsize_shaped_shell_verified(prec):
+    """The bench's exact workload (config 4, 9.19e9 candidates, shaped weights,
+    the stored headroom) in the launch configuration it times.  Every key
+    above the GPU's answer has sum_n >= the answer's, so the oracle's shell
+    sweep over those ~2.9e6 candidates fixes the acceptance window (c18)
+    exactly; y(t*) is checked against the oracle one by one."""
+    params = synth.weights(1)
+    slots = synth.cfg4_grid()
+    H = synth.cfg4_headroom()
+    T = oracle.grid_size(slots)
+    eps = EPS[prec]
+    c = Ctx(params=params, precision=prec)
+    try:
+        d = ab.abacus_search_grid(c.h, ab.make_grid(slots), H, 0, T)
+    finally:
+        c.close()
+    assert d.evaluated == T and d.status == ab.ABACUS_DECIDE_OK
+    smin = int(d.key >> 40) - 1
+    key = (eps, smin)
+    if key not in _SHELL:
+        _SHELL[key] = oracle.sweep_shell(params, slots, H, smin, eps=eps)
+    sh = _SHELL[key]
+    assert accept_key(d.key, sh.maxkey_strict, sh.maxkey_loose), (d.key, sh.maxkey_strict, sh.maxkey_loose)
+    _, yt, _, ope = oracle.sweep(params, slots, H, first=d.index, count=1, want_y=True, want_ope=True)
+    assert abs(d.pred_ms - yt[0]) <= eps * abs(yt[0])
+    assert yt[0] <= H + eps * abs(H)
+    assert list(d.end_op)[:4] == [int(v) for v in ope[0]]
+    assert d.total_ops == smin
+
+
 # --------------------------------------------------------------- decisions --
 @pytest.mark.parametrize("prec", PRECS)
 @pytest.mark.parametrize("space", [ab.ABACUS_SPACE_GRID, ab.ABACUS_SPACE_CHAIN, ab.ABACUS_SPACE_AUTO])

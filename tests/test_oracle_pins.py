@@ -252,6 +252,27 @@ def test_range_shards_combine_to_full_sweep():
         assert sum(q.hash for q in parts) % 2**64 == full.hash
 
 
+def test_shell_sweep_matches_full_sweep_and_counts():
+    """orc_sweep_shell (only sum_n >= s_min) against the full sweep: it
+    evaluates exactly the sum-n polynomial's tail, and its max keys are the
+    full sweep's whenever those lie in the shell, else 0 (nothing above them
+    is in the shell)."""
+    p = synth.raw_weights(5)
+    rng = np.random.default_rng(11)
+    for grid in synth.tiny_grids(30, seed=12, kmax=4, max_len=7):
+        _, y, _, _ = oracle.sweep(p, grid, 0.0, want_y=True)
+        H = float(np.quantile(y, rng.uniform(0.1, 0.9)))
+        full, _, _, _ = oracle.sweep(p, grid, H, eps=1e-2)
+        poly = sum_n_polynomial(grid)
+        for s_min in sorted({0, 1, len(poly) // 2, len(poly) - 1, int(rng.integers(0, len(poly)))}):
+            sh = oracle.sweep_shell(p, grid, H, s_min, eps=1e-2)
+            assert sh.evaluated == sum(poly[s_min:])
+            for name in ("best_key", "maxkey_strict", "maxkey_loose"):
+                kf = getattr(full, name)
+                want = kf if kf and (kf >> 40) - 1 >= s_min else 0
+                assert getattr(sh, name) == want, (name, s_min)
+
+
 def test_linear_predictor_knapsack_closed_form():
     """Linear ReLU-transparent predictor: the max-Sigma-n feasible group is a
     unit-value knapsack (cheapest slot positions first) and t* the greedy
