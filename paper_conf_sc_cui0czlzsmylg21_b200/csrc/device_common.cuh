@@ -77,10 +77,10 @@ __device__ __forceinline__ void walker_next(const Plan& P, Walker& W, uint64_t w
         uint32_t c = x >= W.cnt[kKMax - 1] ? 1u : 0u;
         W.v[kKMax - 1] = c ? x - W.cnt[kKMax - 1] : x;
 #pragma unroll
-        for (int j = kKMax - 2; j >= 0; j--) {
+        for (int j = kKMax - 2; j >= 0; j--) {  // x <= cnt: a carry leaves exactly 0
             x = W.v[j] + c;
             c = x >= W.cnt[j] ? 1u : 0u;
-            W.v[j] = c ? x - W.cnt[j] : x;
+            W.v[j] = c ? 0u : x;
         }
         return;
     }

@@ -88,6 +88,9 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
             wj[g.dpos[j]] = w[f + 1] * scale;  // column of slot j's box digit
         }
         c *= scale;
+        if (FMT == 0 && !SPLIT) {  // digits enter as 1024 + v (store_a1): remove 1024 w_j as the MMA sees it
+            for (int j = 0; j < kKMax; j++) c -= 1024.0f * from16<FMT>(to16<FMT>(wj[j]));
+        }
         uint16_t ch, cl;
         split16<FMT>(c, ch, cl);
         uint8_t* base = s_b1 + (size_t)s * NCH * kChunkBytesN32;
@@ -234,8 +237,24 @@ struct TileIO {
     uint32_t d, a1, a;  // TMEM addresses (column part; lane 0)
 };
 
+// Layer-1 operand row.  fp16 unsplit (digits <= 1024): the digits enter as the
+// exact fp16 values 1024 + v, built by integer adds on the bit patterns
+// (0x6400 + v); build_b1_fused removes 1024 * sum_j w_j from the constant.
+// Columns 3..7 are not written: their K rows of B are zero and the stale
+// activations they hold are finite (the A regions are zeroed at start).
 template <int FMT, bool SPLIT>
 __device__ __forceinline__ void store_a1(uint32_t taddr, const uint32_t (&v)[kKMax]) {
+    if (FMT == 0 && !SPLIT) {
+        uint32_t a[4];
+        a[0] = TcCfg<FMT>::kOne2;
+        a[1] = 0x64006400u + v[0] + (v[1] << 16);  // exact up to v = 1024 (0x6800 = 2048)
+        a[2] = 0x64006400u + v[2] + (v[3] << 16);
+        a[3] = 0u;
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(a[0]),
+                     "r"(a[1]), "r"(a[2]), "r"(a[3])
+                     : "memory");
+        return;
+    }
     uint32_t a[8];
     a[0] = TcCfg<FMT>::kOne2;
     if (SPLIT) {
@@ -287,6 +306,16 @@ struct TcPipe {
         db4 = d4;
 #pragma unroll
         for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
+    }
+    // zero this warp's lanes of the A regions once: columns the layer-1 row
+    // leaves unwritten must hold finite values (their B rows are zero)
+    __device__ __forceinline__ void zero_a() const {
+        uint32_t z[16];
+#pragma unroll
+        for (int i = 0; i < 16; i++) z[i] = 0u;
+        tmem_st16(X.a + lane_off, z);
+        tmem_st16(Y.a + lane_off, z);
+        tmem_wait_st();
     }
     __device__ __forceinline__ bool handoff(bool mine) const {
         fence_before();
@@ -432,6 +461,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     const uint32_t sbase = smem_u32(smem);
     TcPipe<FMT> pp;
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    pp.zero_a();
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
     auto issue_l1 = [&](const TileIO& T, int s) {
@@ -451,18 +481,22 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         uint32_t vX[kKMax], vY[kKMax];
         int sX = 0, sY = 0;
         bool okX = false, okY = false, zX = false, zY = false;
+        // ok: the row is inside its segment (only a segment's last tile is partial)
         auto take = [&](uint32_t (&v)[kKMax], int& s, bool& ok, bool& z) {
-            ok = W.u_end - W.ub > (uint64_t)r;
-            z = walker_is_index0(W, r);
+            const uint64_t rem = W.u_end - W.ub;  // uniform
+            ok = rem >= (uint64_t)kTileM || (uint64_t)r < rem;
+            z = false;
 #pragma unroll
             for (int j = 0; j < kKMax; j++) v[j] = W.v[j];
             s = W.s;
         };
         auto fold = [&](uint32_t yb, int s, const uint32_t (&v)[kKMax], bool ok, bool z) {
             const float y = __uint_as_float(yb);
-            if (ok && z) S->y0 = y;
+            (void)z;
             if (ok) fold_tile(P, s, v, y, best, best_y);
         };
+        // index 0 (the drop test's critical-only group) is row 0 of the plan's
+        // first tile whenever the plan starts at index 0 (P.want_y0)
         // prologue: tile wb in slot X and (if the group has it) wb + 1 in slot Y
         const bool yLive = wb + 1 < we;  // warp-uniform
         take(vX, sX, okX, zX);
@@ -487,6 +521,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             constexpr bool NTWO = decltype(next_two_c)::value;
             uint32_t ybx, yby = 0;
             pp.template run_layers<TWO>(ybx, yby);
+            if (w == 0 && P.want_y0 && r == 0) S->y0 = __uint_as_float(ybx);
             fold(ybx, sX, vX, okX, zX);
             if (TWO) fold(yby, sY, vY, okY, zY);
             if (w + 2 < we) {
@@ -595,6 +630,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
     const uint32_t sbase = smem_u32(smem);
     TcPipe<FMT> pp;
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    pp.zero_a();
     constexpr uint32_t kTable = C::kNchL1 * kChunkBytesN32;
     uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegBatch * kTable;
     const uint64_t d1base = smem_desc(sbase + L.b1 + (uint32_t)g * kMaxSegBatch * kTable);
@@ -1049,8 +1085,8 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
     return cudaGetLastError();
 }
 
-// digits are < cnt: exact unsplit up to 2048 in fp16, 256 in bf16
-static bool need_split(int fmt, uint32_t maxcnt) { return fmt == 0 ? maxcnt > 2049 : maxcnt > 257; }
+// digits are < cnt: unsplit when exact -- fp16 1024 + v up to v = 1024, bf16 v up to 256
+static bool need_split(int fmt, uint32_t maxcnt) { return fmt == 0 ? maxcnt > 1025 : maxcnt > 257; }
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
