@@ -53,7 +53,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "{\n\t"
         ".reg .pred P1;\n\t"
         "LAB_WAIT:\n\t"
+#ifdef EXP_SUSPEND
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, " EXP_SUSPEND ";\n\t"
+#else
         "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+#endif
         "@P1 bra DONE;\n\t"
         "bra LAB_WAIT;\n\t"
         "DONE:\n\t"
@@ -349,6 +353,9 @@ template <int FMT>
 __device__ __forceinline__ uint32_t pack2_relu(uint32_t lo_bits, uint32_t hi_bits) {
     uint32_t d;
     const float lo = __uint_as_float(lo_bits), hi = __uint_as_float(hi_bits);
+#ifdef EXP_HALFCVT
+    if (FMT == 0) { d = lo_bits ^ hi_bits; return d; }
+#endif
     if (FMT == 0) asm("cvt.rn.relu.f16x2.f32 %0, %1, %2;" : "=r"(d) : "f"(hi), "f"(lo));
     else asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(d) : "f"(hi), "f"(lo));
     return d;
