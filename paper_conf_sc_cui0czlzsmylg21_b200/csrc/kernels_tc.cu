@@ -40,6 +40,7 @@ struct TcParams {
     const uint8_t* blob;  // device weight blob (layer 2, layer 3, output chunks)
     uint32_t bytes;
     float l1_scale;
+    float b4;             // output bias (fp32)
 };
 
 template <int FMT>
@@ -283,6 +284,30 @@ struct TcPipe {
     uint64_t* bar;
     uint64_t db2, db3, db4;
     bool me[4];
+    // fp16: the output layer runs without its bias K chunk and b4 is added to y
+    // in fp32 when y is read (one MMA fewer per tile)
+    bool outbias = false;
+    float b4 = 0.0f;
+    __device__ __forceinline__ void set_outbias(float bias) {
+        outbias = FMT == 0;
+        b4 = bias;
+    }
+    __device__ __forceinline__ uint32_t add_b4(uint32_t ybits) const {
+        return outbias ? __float_as_uint(__uint_as_float(ybits) + b4) : ybits;
+    }
+#ifdef EXP_STAGETRACE
+    unsigned long long* tr = nullptr;  // CTA 0, group 0, lane 0 of each warp
+    uint32_t it = 0, wqq = 0;
+    __device__ __forceinline__ void stamp(int st, int k) {
+        if (tr && it >= 64 && it < 80 && (threadIdx.x & 31) == 0) {
+            long long c;
+            asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
+            tr[16 + (((it - 64) * 4 + wqq) * 4 + st) * 3 + k] = (unsigned long long)c;
+        }
+    }
+#else
+    __device__ __forceinline__ void stamp(int, int) {}
+#endif
 
     // fused layout: 96 columns per group, one constant chunk at 480 for all
     __device__ __forceinline__ void init(uint32_t tbase, int g, int wq, uint64_t* mbar, uint64_t d2, uint64_t d3,
@@ -346,8 +371,16 @@ struct TcPipe {
         constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 0 && TWO) {
+            if (LAYER == 2 && outbias) {
+                issue_layer2_asm<0, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+                return;
+            }
             issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
         } else if (!TWO) {
+            if (FMT == 0 && LAYER == 2 && outbias) {
+                issue_layer_asm<FMT, ID, CH, false>(X.d, X.a, tCx, db, bar);
+                return;
+            }
             issue_layer_asm<FMT, ID, CH>(X.d, X.a, tCx, db, bar);
         } else {
             uint64_t d[5];
@@ -364,6 +397,7 @@ struct TcPipe {
     template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage() {
         wait();
+        stamp(LAYER, 0);
         if (TWO) {
             uint32_t a[32], b[32], h[16];
             tmem_ld32x2(X.d + lane_off, Y.d + lane_off, a, b);
@@ -386,7 +420,11 @@ struct TcPipe {
             if (TWO) tmem_st8(tCy + lane_off, c8);
         }
         tmem_wait_st();
-        if (handoff(me[LAYER])) issue_next<LAYER, TWO>();
+        stamp(LAYER, 1);
+        if (handoff(me[LAYER])) {
+            stamp(LAYER, 2);
+            issue_next<LAYER, TWO>();
+        }
     }
     // the three hidden stages, then wait for the output MMA and read y (column 0 of D)
     template <bool TWO, bool CONST = false>
@@ -395,8 +433,11 @@ struct TcPipe {
         stage<1, TWO>();
         stage<2, TWO>();
         wait();
+        stamp(3, 0);
         if (TWO) tmem_ld1x2(X.d + lane_off, Y.d + lane_off, yx, yy);
         else tmem_ld1(X.d + lane_off, yx);
+        yx = add_b4(yx);
+        if (TWO) yy = add_b4(yy);
     }
 };
 
@@ -515,12 +556,16 @@ struct PackedWalker {
         }
         if (tl == 1 && last_rows < (uint32_t)kTileM && r >= last_rows) sn = 0u;
     }
-    __device__ __forceinline__ void store(uint32_t taddr) const {
-        asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(0x3C003C00u),
-                     "r"(a1), "r"(a2), "r"(0u)
-                     : "memory");
-    }
+    __device__ __forceinline__ void store(uint32_t taddr) const;
 };
+
+// layer-1 operand row (1, 1, 1024 + v0 .. 1024 + v3, 0, 0) of a packed tile row
+__device__ __forceinline__ void store_a1_packed(uint32_t taddr, uint32_t a1, uint32_t a2) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(0x3C003C00u),
+                 "r"(a1), "r"(a2), "r"(0u)
+                 : "memory");
+}
+__device__ __forceinline__ void PackedWalker::store(uint32_t taddr) const { store_a1_packed(taddr, a1, a2); }
 
 // fold one row of a packed tile: the key is built only when the row fits the
 // headroom and its sum_n can reach the running best
@@ -574,6 +619,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     const uint32_t sbase = smem_u32(smem);
     TcPipe<FMT> pp;
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    pp.set_outbias(TP.b4);
     pp.zero_a();
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
@@ -590,6 +636,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     work_range(P.n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
     if constexpr (FMT == 0 && !SPLIT) {
         if (wb < we) {
+#ifdef EXP_STAGETRACE
+            if (blockIdx.x == 0 && g == 0) pp.tr = P.trace;
+            pp.wqq = wq;
+#endif
             PackedWalker W;
             W.begin(P, wb, r);
             uint32_t x1, x2, xs, y1 = 0, y2 = 0, ys = 0;  // X / Y rows: a1, a2, sn
@@ -613,25 +663,50 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             auto iteration = [&](auto two_c, auto next_two_c) {
                 constexpr bool TWO = decltype(two_c)::value;
                 constexpr bool NTWO = decltype(next_two_c)::value;
+                pp.template stage<0, TWO>();
+                pp.template stage<1, TWO>();
+                pp.template stage<2, TWO>();
+                // the next tiles' operand rows are computed while the output MMA runs
+                const bool more = w + 2 < we;  // warp-uniform
+                uint32_t n1 = 0, n2 = 0, ns = 0;
+                int nsX = 0;
+                if (more) {
+                    W.next(P, r);
+                    n1 = W.a1;
+                    n2 = W.a2;
+                    ns = W.sn;
+                    nsX = W.s;
+                    if (NTWO) W.next(P, r);
+                }
+                pp.wait();
+                pp.stamp(3, 0);
                 uint32_t ybx, yby = 0;
-                pp.template run_layers<TWO>(ybx, yby);
+                if (TWO) tmem_ld1x2(pp.X.d + pp.lane_off, pp.Y.d + pp.lane_off, ybx, yby);
+                else tmem_ld1(pp.X.d + pp.lane_off, ybx);
+                ybx = pp.add_b4(ybx);
+                if (TWO) yby = pp.add_b4(yby);
                 if (w == 0 && P.want_y0 && r == 0) S->y0 = __uint_as_float(ybx);
                 fold_packed(P, sX, x1, x2, xs, __uint_as_float(ybx), best, best_y, bsn);
                 if (TWO) fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
-                if (w + 2 < we) {
-                    W.next(P, r);
-                    takeX();
-                    if (NTWO) {
-                        W.next(P, r);
-                        takeY();
-                    }
+                if (more) {
+                    x1 = n1;
+                    x2 = n2;
+                    xs = ns;
+                    sX = nsX;
+                    store_a1_packed(pp.X.a1 + pp.lane_off, x1, x2);
+                    if (NTWO) takeY();
                     tmem_wait_st();
+                    pp.stamp(3, 1);
                     if (pp.handoff(pp.me[3])) {
+                        pp.stamp(3, 2);
                         issue_l1(pp.X, sX);
                         if (NTWO) issue_l1(pp.Y, sY);
                         pp.commit();
                     }
                 }
+#ifdef EXP_STAGETRACE
+                pp.it++;
+#endif
                 w += 2;
             };
             while (w + 3 < we) iteration(T2{}, T2{});
@@ -685,23 +760,15 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             uint32_t ybx, yby = 0;
             pp.template run_layers<TWO>(ybx, yby);
             if (w == 0 && P.want_y0 && r == 0) S->y0 = __uint_as_float(ybx);
-#ifndef EXP_NOFOLD
             fold(ybx, sX, vX, okX, zX);
             if (TWO) fold(yby, sY, vY, okY, zY);
-#else
-            if (ybx == 0x7f800001u && yby == 0x7f800001u) best = ybx;
-#endif
             if (w + 2 < we) {
-#ifndef EXP_NOWALK
                 walker_next(P, W, w + 2, r);
                 take(vX, sX, okX, zX);
-#endif
                 store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
                 if (NTWO) {
-#ifndef EXP_NOWALK
                     walker_next(P, W, w + 3, r);
                     take(vY, sY, okY, zY);
-#endif
                     store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
                 }
                 tmem_wait_st();
@@ -801,6 +868,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
     const uint32_t sbase = smem_u32(smem);
     TcPipe<FMT> pp;
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    pp.set_outbias(TP.b4);
     pp.zero_a();
     constexpr uint32_t kTable = C::kNchL1 * kChunkBytesN32;
     uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegBatch * kTable;
@@ -1109,6 +1177,7 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
     TcPipe<FMT> pp;
     pp.init_layout(X, Y, col + 48, col + 112, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3),
                    smem_desc(sbase + L.w4));
+    pp.set_outbias(TP.b4);
     const uint32_t lane_off = pp.lane_off;
     uint64_t* tbX = &tbars[2 * g];
     uint64_t* tbY = &tbars[2 * g + 1];
@@ -1261,7 +1330,7 @@ static bool need_split(int fmt, uint32_t maxcnt) { return fmt == 0 ? maxcnt > 10
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
-    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
     uint32_t maxcnt = 0;
     for (int s = 0; s < P.n_seg; s++)
         for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
@@ -1293,7 +1362,7 @@ static cudaError_t launch_batch_fmt(const BatchDec* decs, const SegP* segs, int3
 cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, const uint64_t* d_n_pairs,
                             uint64_t pairs_ub, uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1,
                             BatchAcc* acc, float* y0s, Result* out, int nsm, cudaStream_t st) {
-    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
     const bool split = need_split(TW.fmt, maxcnt);
     cudaError_t e;
 #define ABACUS_BATCH_ARGS d_decs, d_segs, n_dec, d_n_pairs, pairs_ub, D, tp, w1b1, acc, y0s, nsm, st
@@ -1331,7 +1400,7 @@ cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D,
                               float* y, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
     if (D > 31) return cudaErrorInvalidValue;  // layer-1 operand: 4 K-chunks = the 32-column U region
-    TcParams tp{TW.blob, TW.bytes, TW.l1_scale};
+    TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
     if (TW.fmt == 0) return launch_predict_fmt<0>(tp, w1b1, D, x, count, y, nsm, st);
     return launch_predict_fmt<1>(tp, w1b1, D, x, count, y, nsm, st);
 }

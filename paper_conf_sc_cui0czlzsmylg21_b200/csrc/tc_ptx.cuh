@@ -53,11 +53,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "{\n\t"
         ".reg .pred P1;\n\t"
         "LAB_WAIT:\n\t"
-#ifdef EXP_SUSPEND
-        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, " EXP_SUSPEND ";\n\t"
-#else
         "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
-#endif
         "@P1 bra DONE;\n\t"
         "bra LAB_WAIT;\n\t"
         "DONE:\n\t"
@@ -157,10 +153,29 @@ __device__ __forceinline__ void mma_commit_elect(uint64_t* bar) {
 // immediate, one elected lane issues the MMAs and the commit.
 //   FMT 0 (fp16):  D  = A[0:8) W_c0 + A[8:16) W_c1 + C bias
 //   FMT 1 (bf16):  D  = A[0:8) Whi_c0 + A[8:16) Whi_c1 + A[0:8) Wlo_c0 + A[8:16) Wlo_c1 + C bias
-template <int FMT, uint32_t IDESC, uint32_t CHUNK>
+template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
 __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32_t tC, uint64_t dbase,
                                                 uint64_t* bar) {
     constexpr uint32_t U = CHUNK >> 4;
+    if (FMT == 0 && !BIAS) {  // the two data chunks only (the bias is added outside)
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1;\n\t"
+            ".reg .b32 a8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %2, %4;\n\t"
+            "add.u32 a8, %1, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %5, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d1, %5, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%3];\n\t"
+            "}" ::"r"(tD),
+            "r"(tA), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"(IDESC)
+            : "memory");
+        return;
+    }
     if (FMT == 0) {
         asm volatile(
             "{\n\t"
@@ -209,11 +224,33 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
 }
 
 // the MMAs of one layer for TWO tiles (same B operand) and ONE commit
-template <int FMT, uint32_t IDESC, uint32_t CHUNK>
+template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
 __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
                                                  uint32_t tCx, uint32_t tCy, uint64_t dbase, uint64_t* bar) {
     static_assert(FMT == 0, "lock-step pair issue: fp16 layout");
     constexpr uint32_t U = CHUNK >> 4;
+    if (!BIAS) {  // the two data chunks only (the bias is added outside)
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1;\n\t"
+            ".reg .b32 ax8, ay8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %4, %6;\n\t"
+            "add.u32 ax8, %1, 8;\n\t"
+            "add.u32 ay8, %3, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %4, %7, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d1, %7, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %4, %7, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %7, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%5];\n\t"
+            "}" ::"r"(tDx),
+            "r"(tAx), "r"(tDy), "r"(tAy), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"(IDESC)
+            : "memory");
+        return;
+    }
     asm volatile(
         "{\n\t"
         ".reg .pred e, pf, pt;\n\t"
@@ -353,9 +390,6 @@ template <int FMT>
 __device__ __forceinline__ uint32_t pack2_relu(uint32_t lo_bits, uint32_t hi_bits) {
     uint32_t d;
     const float lo = __uint_as_float(lo_bits), hi = __uint_as_float(hi_bits);
-#ifdef EXP_HALFCVT
-    if (FMT == 0) { d = lo_bits ^ hi_bits; return d; }
-#endif
     if (FMT == 0) asm("cvt.rn.relu.f16x2.f32 %0, %1, %2;" : "=r"(d) : "f"(hi), "f"(lo));
     else asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(d) : "f"(hi), "f"(lo));
     return d;
