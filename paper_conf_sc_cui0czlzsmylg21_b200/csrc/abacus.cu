@@ -926,7 +926,7 @@ int abacus_predict_batch(abacus_ctx* c, const int16_t* d_features, uint64_t coun
     } else {
         if (c->D > 31) return fail(c, ABACUS_E_INVALID, "tensor predict supports D <= 31 (N <= 15 models)");
         const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
-        CUDA_TRY(c, launch_predict_tc(c->tw[fmt], c->d_w1b1, c->D, d_features, count, d_latency_ms, c->nsm, st));
+        CUDA_TRY(c, launch_predict_tc(c->tw[fmt], c->w234, c->d_w1b1, c->D, d_features, count, d_latency_ms, c->nsm, st));
     }
     if (count) c->launches++;
     return ABACUS_OK;

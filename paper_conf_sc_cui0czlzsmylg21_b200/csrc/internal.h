@@ -71,7 +71,8 @@ cudaError_t launch_train_step(const TrainArgs& A, cudaStream_t st);
 cudaError_t launch_batch_tc(const BatchDec* d_decs, const SegP* d_segs, int32_t n_dec, const uint64_t* d_n_pairs,
                             uint64_t pairs_ub, uint32_t maxcnt, int32_t D, const TcWeights& TW, const float* w1b1,
                             BatchAcc* acc, float* y0s, Result* out, int nsm, cudaStream_t st);
-cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
+cudaError_t launch_predict_tc(const TcWeights& TW, const W234& W, const float* w1b1, int32_t D, const int16_t* x,
+                              uint64_t count,
                               float* y, int nsm, cudaStream_t st);
 
 }  // namespace abacus

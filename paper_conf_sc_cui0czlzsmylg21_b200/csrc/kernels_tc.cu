@@ -1302,6 +1302,221 @@ __global__ void __launch_bounds__(NG * 128, 1) predict_tc_kernel(const __grid_co
 }
 
 // ---------------------------------------------------------------------------
+// predict, fp16, D = 24 (N = 8, K_MAX = 4: the canonical width) -- the
+// fused kernel's pipeline (5 groups x 2 lock-step tiles, 96 TMEM columns per
+// group) fed from HBM instead of the walker.  A row's 24 features enter the
+// layer-1 operand as the exact fp16 values 1024 + v (bit pattern
+// 0x6400 | v, valid for 0 <= v < 1024: every Fig.-8 feature of the registry),
+// so layer 1 is 2 K chunks (24 features + the (1, 1) bias pair) and the
+// operand is exactly the 16-column A region.  Rows with a feature outside
+// [0, 1024) are flagged (one OR over the 12 packed words) and recomputed on
+// the CUDA cores in fp32 after the tile; their tensor result is discarded.
+// The 128 rows (6 KB) of a tile come in by a 1-D TMA bulk copy into one of
+// two stages per slot, issued two iterations ahead.
+// ---------------------------------------------------------------------------
+constexpr int kPred24NG = 5;
+constexpr uint32_t kRow24 = 48;
+constexpr uint32_t kStage24 = kTileM * kRow24;  // 6 KB
+
+// layer-1 B operand (2 chunks): k < 24: w_nk s1; k = 24, 25: (b1_n s1 - 1024 sum_k w_nk s1) as (hi, lo)
+__device__ void build_b1_predict24(const float* __restrict__ w1b1, float scale, uint8_t* s_b1) {
+    constexpr int FMT = 0, D = 24;
+    const float* b1 = w1b1 + kHidden * D;
+    for (int e = threadIdx.x; e < kHidden * 32; e += blockDim.x) {
+        const int n = e >> 5, k = e & 31;
+        uint16_t v = 0;
+        if (k < D) {
+            v = to16<FMT>(w1b1[n * D + k] * scale);
+        } else if (k < D + 2) {
+            double off = 0.0;
+            for (int j = 0; j < D; j++) off += (double)from16<FMT>(to16<FMT>(w1b1[n * D + j] * scale)) * 1024.0;
+            const float bb = (float)((double)b1[n] * (double)scale - off);
+            uint16_t h, l;
+            split16<FMT>(bb, h, l);
+            v = k == D ? h : l;
+        }
+        *reinterpret_cast<uint16_t*>(s_b1 + (size_t)(k >> 4) * kChunkBytesN32 + b_offset(n, k & 15)) = v;
+    }
+}
+
+// fp32 SIMT forward of one row (the rare rows outside the tensor path's range)
+__device__ __forceinline__ float predict_row_fp32(const W234& W, const float* __restrict__ w1b1,
+                                               const int16_t* __restrict__ row) {
+    constexpr int D = 24;
+    float h1[kHidden], h2[kHidden];
+#pragma unroll 1
+    for (int i = 0; i < kHidden; i++) {
+        float s = w1b1[kHidden * D + i];
+        for (int k = 0; k < D; k++) s = fmaf(w1b1[i * D + k], (float)row[k], s);
+        h1[i] = fmaxf(s, 0.0f);
+    }
+#pragma unroll 1
+    for (int i = 0; i < kHidden; i++) {
+        float s = W.b2[i];
+        for (int j = 0; j < kHidden; j++) s = fmaf(W.W2[i][j], h1[j], s);
+        h2[i] = fmaxf(s, 0.0f);
+    }
+    float acc = W.b4;
+#pragma unroll 1
+    for (int i = 0; i < kHidden; i++) {
+        float s = W.b3[i];
+        for (int j = 0; j < kHidden; j++) s = fmaf(W.W3[i][j], h2[j], s);
+        acc = fmaf(W.w4[i], fmaxf(s, 0.0f), acc);
+    }
+    return acc;
+}
+
+template <int NG>
+__global__ void __launch_bounds__(NG * 128, 1) predict24_tc_kernel(const __grid_constant__ TcParams TP,
+                                                                   const __grid_constant__ W234 W,
+                                                                   const float* __restrict__ w1b1,
+                                                                   const int16_t* __restrict__ x, uint64_t count,
+                                                                   float* __restrict__ y) {
+    constexpr int FMT = 0;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    // stages: per group X0 X1 Y0 Y1 (4 x 6 KB); TMA mbarriers after the TMEM slot
+    const TcSmem L = tc_smem_layout<FMT>(2, kChunkBytesN32, NG, 4 * kStage24);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
+    uint64_t* tbars = reinterpret_cast<uint64_t*>(smem + L.total);  // per group: X0 X1 Y0 Y1
+    const int tid = threadIdx.x;
+    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+    const int g = warp >> 2, wq = warp & 3;
+    {
+        const int4* src = reinterpret_cast<const int4*>(TP.blob);
+        int4* dst = reinterpret_cast<int4*>(smem);
+        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
+    }
+    build_b1_predict24(w1b1, TP.l1_scale, smem + L.b1);
+    if (tid == 0)
+        for (int i = 0; i < 4 * NG; i++) mbar_init(&tbars[i], 1);
+    const uint32_t tbase = fused_prologue_tmem<FMT, NG>(bars, tmem_slot, warp, g, wq);
+
+    const uint32_t r = (uint32_t)(tid & 127);
+    const uint32_t sbase = smem_u32(smem);
+    TcPipe<FMT> pp;
+    pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
+    pp.set_outbias(TP.b4);
+    const uint64_t d1 = smem_desc(sbase + L.b1);
+    uint8_t* stg = smem + L.stage + (uint32_t)g * 4u * kStage24;  // X0 X1 Y0 Y1
+    uint64_t* tb = &tbars[4 * g];
+    uint32_t tph = 0;  // phase bit per stage (bit i: stage i)
+    const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+    uint64_t wb, we;
+    work_range(n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
+    // stage index of tile w: slot (w - wb) & 1, buffer ((w - wb) >> 1) & 1
+    auto sidx = [&](uint64_t w) -> int { return (int)(((w - wb) & 1u) * 2u + (((w - wb) >> 1) & 1u)); };
+    auto fetch = [&](uint64_t w) {  // one thread of the group
+        if (w >= we) return;
+        const int si = sidx(w);
+        const uint64_t row0 = w * kTileM;
+        const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_arrive_expect_tx(&tb[si], nrows * kRow24);
+        bulk_g2s(stg + (uint32_t)si * kStage24, x + row0 * 24u, nrows * kRow24, &tb[si]);
+    };
+    // operand words of this thread's row of tile w (after its stage landed)
+    auto load = [&](uint64_t w, uint32_t (&a)[16], uint32_t& bad) {
+        const int si = sidx(w);
+        mbar_wait(&tb[si], (tph >> si) & 1u);
+        tph ^= 1u << si;
+        const uint64_t row0 = w * kTileM;
+        const uint32_t nrows = (uint32_t)min((uint64_t)kTileM, count - row0);
+        const uint4* rp = reinterpret_cast<const uint4*>(stg + (uint32_t)si * kStage24 + min(r, nrows - 1) * kRow24);
+        const uint4 q0 = rp[0], q1 = rp[1], q2 = rp[2];
+        a[0] = q0.x; a[1] = q0.y; a[2] = q0.z; a[3] = q0.w;
+        a[4] = q1.x; a[5] = q1.y; a[6] = q1.z; a[7] = q1.w;
+        a[8] = q2.x; a[9] = q2.y; a[10] = q2.z; a[11] = q2.w;
+        const uint32_t o = (a[0] | a[1] | a[2] | a[3]) | (a[4] | a[5] | a[6] | a[7]) | (a[8] | a[9] | a[10] | a[11]);
+        bad = (o & 0xFC00FC00u) != 0u ? 1u : 0u;  // a feature < 0 or >= 1024: recomputed in fp32
+#pragma unroll
+        for (int i = 0; i < 12; i++) a[i] |= 0x64006400u;
+        a[12] = TcCfg<FMT>::kOne2;
+        a[13] = a[14] = a[15] = 0u;
+    };
+    auto issue_l1 = [&](const TileIO& T) {
+        constexpr uint32_t id32 = idesc_f16(FMT, 32);
+        mma_ts_elect(T.d, T.a1, d1, id32, 0u);
+        mma_ts_elect(T.d, T.a1 + 8, d1 + (kChunkBytesN32 >> 4), id32, 1u);
+    };
+    auto put_y = [&](uint64_t w, uint32_t yb, uint32_t bad) {
+        const uint64_t row = w * kTileM + r;
+        if (row >= count) return;
+        float v = __uint_as_float(yb);
+        if (bad) v = predict_row_fp32(W, w1b1, x + row * 24u);
+        y[row] = v;
+    };
+    using T1 = std::integral_constant<bool, false>;
+    using T2 = std::integral_constant<bool, true>;
+    if (wb < we) {
+        if (r == 0)
+            for (uint64_t w = wb; w < wb + 4; w++) fetch(w);
+        uint32_t ax[16], ay[16];
+        uint32_t badX = 0, badY = 0;
+        const bool yLive = wb + 1 < we;
+        load(wb, ax, badX);
+        tmem_st16(pp.X.a + pp.lane_off, ax);
+        if (yLive) {
+            load(wb + 1, ay, badY);
+            tmem_st16(pp.Y.a + pp.lane_off, ay);
+        }
+        tmem_wait_st();
+        if (pp.handoff(pp.me[3])) {
+            issue_l1(pp.X);
+            if (yLive) issue_l1(pp.Y);
+            pp.commit();
+        }
+        uint64_t w = wb;
+        auto iteration = [&](auto two_c, auto next_two_c) {
+            constexpr bool TWO = decltype(two_c)::value;
+            constexpr bool NTWO = decltype(next_two_c)::value;
+            pp.template stage<0, TWO>();
+            pp.template stage<1, TWO>();
+            pp.template stage<2, TWO>();
+            // the next tiles' operand rows are read while the output MMA runs
+            const bool more = w + 2 < we;
+            uint32_t nbx = 0, nby = 0;
+            if (more) load(w + 2, ax, nbx);
+            pp.wait();
+            uint32_t yx, yy = 0;
+            if (TWO) tmem_ld1x2(pp.X.d + pp.lane_off, pp.Y.d + pp.lane_off, yx, yy);
+            else tmem_ld1(pp.X.d + pp.lane_off, yx);
+            yx = pp.add_b4(yx);
+            if (TWO) yy = pp.add_b4(yy);
+            if (more) {
+                tmem_st16(pp.X.a + pp.lane_off, ax);
+                if (NTWO) {
+                    load(w + 3, ay, nby);
+                    tmem_st16(pp.Y.a + pp.lane_off, ay);
+                }
+                tmem_wait_st();
+                if (pp.handoff(pp.me[3])) {
+                    issue_l1(pp.X);
+                    if (NTWO) issue_l1(pp.Y);
+                    pp.commit();
+                    if ((tid & 31) == 0) {  // every thread has read these stages (hand-off barrier)
+                        fetch(w + 4);
+                        if (NTWO) fetch(w + 5);
+                    }
+                }
+            }
+            put_y(w, yx, badX);
+            if (TWO) put_y(w + 1, yy, badY);
+            badX = nbx;
+            badY = nby;
+            w += 2;
+        };
+        while (w + 3 < we) iteration(T2{}, T2{});
+        if (w + 1 < we) iteration(T2{}, T1{});
+        if (w < we) iteration(T1{}, T1{});
+    }
+    fence_before();
+    __syncthreads();
+    fence_after();
+    if (warp == 0) tmem_dealloc(tbase, 512);
+}
+
+// ---------------------------------------------------------------------------
 // launchers
 // ---------------------------------------------------------------------------
 constexpr int kFusedNG = 5;
@@ -1396,11 +1611,25 @@ static cudaError_t launch_predict_fmt(const TcParams& tp, const float* w1b1, int
     return cudaGetLastError();
 }
 
-cudaError_t launch_predict_tc(const TcWeights& TW, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
-                              float* y, int nsm, cudaStream_t st) {
+cudaError_t launch_predict_tc(const TcWeights& TW, const W234& W, const float* w1b1, int32_t D, const int16_t* x,
+                              uint64_t count, float* y, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
     if (D > 31) return cudaErrorInvalidValue;  // layer-1 operand: 4 K-chunks = the 32-column U region
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
+    if (TW.fmt == 0 && D == 24 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0) {
+        constexpr int NG = kPred24NG;
+        const TcSmem L = tc_smem_layout<0>(2, kChunkBytesN32, NG, 4 * kStage24);
+        const uint32_t total = L.total + 8u * 4u * NG;  // + TMA mbarriers
+        auto kern = predict24_tc_kernel<NG>;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)total);
+        if (e != cudaSuccess) return e;
+        const uint64_t n_tiles = (count + kTileM - 1) / kTileM;
+        uint64_t g = (n_tiles + NG - 1) / NG;
+        if (g > (uint64_t)nsm) g = (uint64_t)nsm;
+        if (g < 1) g = 1;
+        kern<<<(int)g, NG * 128, total, st>>>(tp, W, w1b1, x, count, y);
+        return cudaGetLastError();
+    }
     if (TW.fmt == 0) return launch_predict_fmt<0>(tp, w1b1, D, x, count, y, nsm, st);
     return launch_predict_fmt<1>(tp, w1b1, D, x, count, y, nsm, st);
 }

@@ -133,6 +133,36 @@ def test_predict_cfg5_tolerance(prec, variant):
         c.close()
 
 
+@pytest.mark.parametrize("prec", PRECS)
+def test_predict_any_int16_features(prec):
+    """The ABI takes any int16 feature value.  The fp16 D = 24 kernel enters
+    features as 1024 + v (exact for 0 <= v < 1024) and recomputes rows with a
+    feature outside that range in fp32; rows of every kind are mixed inside
+    the same tiles (in-range, negative, >= 1024, int16 extremes) with a ragged
+    last tile, and each must be within its bar of the fp64 oracle."""
+    params = synth.weights(1)
+    c = Ctx(params=params, precision=prec)
+    try:
+        groups = synth.instance_samples(20_000, seed=16)
+        X = oracle.encode_groups(8, 4, [g.slots for g in groups])[:12_345].copy()
+        rng = np.random.default_rng(17)
+        kind = rng.integers(0, 4, size=len(X))
+        col = rng.integers(0, 24, size=len(X))
+        rows = np.arange(len(X))
+        X[rows[kind == 1], col[kind == 1]] = -rng.integers(1, 40, size=(kind == 1).sum())
+        X[rows[kind == 2], col[kind == 2]] = rng.integers(1024, 4000, size=(kind == 2).sum())
+        X[rows[kind == 3], col[kind == 3]] = rng.choice(np.array([-32768, 32767, 1024, -1], dtype=np.int16),
+                                                        size=(kind == 3).sum())
+        y64 = oracle.mlp64_batch(params, X)
+        y = c.predict(X)
+        err = rel_err(y, y64, output_term_magnitude(params, X))
+        print(NAMES[prec], "max rel err %.3e (in range %.3e)" % (err.max(), err[kind == 0].max()))
+        assert np.all(np.isfinite(y))
+        assert err.max() <= EPS[prec]
+    finally:
+        c.close()
+
+
 def output_term_magnitude(params, X):
     """|b4| + sum_j |w4_j h3_j(x)| in fp64 (normalisation only, not a reference)."""
     W1, b1, W2, b2, W3, b3, w4, b4 = [a.astype(np.float64) for a in synth.split_params(params)]
