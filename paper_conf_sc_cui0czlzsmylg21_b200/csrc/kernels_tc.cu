@@ -926,6 +926,55 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             if ((tid & 31) == 0 && best) acc_fold(&acc[d], best, best_y);
             best = 0;
         };
+        if constexpr (FMT == 0 && !SPLIT) {
+            // packed walker + three-instruction fold (as fused_tc_kernel)
+            PackedWalker W{};
+            uint32_t x1 = 0, x2 = 0, xs = 0, y1 = 0, y2 = 0, ys = 0, bsn = 1u;
+            int sX = 0, sY = 0;
+            uint64_t ltX = 0;
+            // move the walker to local tile lt (the next one); a decision's pad tile has no rows
+            auto adv = [&](uint64_t lt) {
+                if (lt >= P.n_tiles) W.sn = 0u;
+                else W.next(P, r);
+            };
+            auto enter_pair = [&](uint64_t p, bool fresh) {
+                const uint64_t lt = 2 * (p - dec_pair0);
+                if (fresh) W.begin(P, lt, r);
+                else adv(lt);
+                x1 = W.a1; x2 = W.a2; xs = W.sn; sX = W.s; ltX = lt;
+                W.store(pp.X.a1 + pp.lane_off);
+                adv(lt + 1);
+                y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s;
+                W.store(pp.Y.a1 + pp.lane_off);
+                tmem_wait_st();
+                if (pp.handoff(pp.me[3])) {
+                    issue_l1(pp.X, sX);
+                    issue_l1(pp.Y, sY);
+                    pp.commit();
+                }
+            };
+            load_decision();
+            enter_pair(pb, true);
+            for (uint64_t p = pb; p < pe; p++) {
+                uint32_t ybx, yby;
+                pp.template run_layers<true>(ybx, yby);
+                if (ltX == 0 && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
+                fold_packed(P, sX, x1, x2, xs, __uint_as_float(ybx), best, best_y, bsn);
+                fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
+                if (p + 1 == dec_pair_end) {  // leaving decision d
+                    flush();
+                    bsn = 1u;
+                    if (p + 1 < pe) {
+                        d++;
+                        load_decision();
+                        enter_pair(p + 1, true);
+                    }
+                } else if (p + 1 < pe) {
+                    enter_pair(p + 1, false);
+                }
+            }
+            flush();
+        } else {
         Walker W{};
         uint32_t vX[kKMax], vY[kKMax];
         int sX = 0, sY = 0;
@@ -978,6 +1027,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             }
         }
         flush();  // the last decision of the range (a no-op if it was flushed at its end)
+        }
     }
     fence_before();
     __syncthreads();
