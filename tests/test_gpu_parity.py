@@ -246,6 +246,44 @@ def test_search_grid_ragged_shards(prec):
         c.close()
 
 
+@pytest.mark.parametrize("prec", PRECS)
+def test_search_grid_long_fast_digit_shards(prec):
+    """Grids whose fastest digit has >= 128 values (the packed walker's
+    one-carry tile advance) mixed with short ones, absent options (several
+    segments, some with a short last digit), shards that start and end inside
+    segments and inside tiles, and single-tile / single-row windows."""
+    c = Ctx(params=synth.weights(1), precision=prec)
+    rng = np.random.default_rng(23)
+    try:
+        for it in range(8):
+            k = int(rng.integers(2, 4))
+            models = [int(m) for m in rng.choice(np.arange(1, 9), size=k, replace=False)]
+            slots = []
+            for j, m in enumerate(models):
+                Lm = synth.L(m)
+                if j == k - 1 and Lm >= 140:   # the fastest digit: long range
+                    lo = int(rng.integers(1, Lm - 130))
+                    hi = int(rng.integers(lo + 128, min(Lm, lo + 600) + 1))
+                else:                          # the others: short ranges keep T small
+                    lo = int(rng.integers(1, Lm + 1))
+                    hi = int(min(Lm, lo + rng.integers(0, 6)))
+                slots.append(synth.GridSlot(m, int(rng.integers(1, lo + 1)), int(rng.choice([1, 8, 32])),
+                                            synth.seqlen_for(m, int(rng.integers(8, 513))), lo, hi,
+                                            int(rng.integers(0, 2))))
+            T = oracle.grid_size(slots)
+            _, y64, _, _ = oracle.sweep(c.params, slots, 0.0, want_y=True)
+            H = float(np.float32(np.quantile(y64, rng.uniform(0.05, 0.95))))
+            full = _check_sweep(c, slots, H)
+            G = int(rng.integers(2, 8))
+            keys = [_check_sweep(c, slots, H, *ab.shard_range(T, r, G)).key for r in range(G)]
+            assert max(keys) == full.key
+            for first, count in [(int(rng.integers(0, T)), 1), (int(rng.integers(0, max(1, T - 128))), 128),
+                                 (int(rng.integers(0, max(1, T - 300))), 300)]:
+                _check_sweep(c, slots, H, first, min(count, T - first))
+    finally:
+        c.close()
+
+
 def test_search_grid_deterministic(ctx):
     slots = synth.cfg1_grids()[2][1]
     T = oracle.grid_size(slots)
