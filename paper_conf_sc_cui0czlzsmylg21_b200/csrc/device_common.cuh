@@ -142,6 +142,114 @@ __device__ __forceinline__ bool walker_is_index0(const Walker& W, uint32_t r) {
 }
 
 // ---------------------------------------------------------------------------
+// Packed tile walker (fp16 with unsplit digits, i.e. every box digit < 1024:
+// the headline path).  A row keeps its layer-1 operand words directly,
+//     a1 = (0x6400 + v0) | (0x6400 + v1) << 16,  a2 = (0x6400 + v2) | (0x6400 + v3) << 16
+// (the exact fp16 values 1024 + v_j, store_a1's layout), and sn = sum_n + 1
+// (reading c12, the key's high part).  A tile advance adds 128 to v3 and
+// carries on the packed words with predicated adds; sn follows the carries.
+// Segment changes are a uniform countdown of the segment's tiles, and the
+// rows past the end of a segment's last tile get sn = 0, which no fold
+// accepts (every candidate has sn >= 1).  The digits themselves are unpacked
+// only when a fold has to build a key.
+// ---------------------------------------------------------------------------
+struct PackedWalker {
+    uint32_t a1, a2, sn;  // per row: the most recently taken tile
+    int32_t s;            // segment (uniform)
+    uint32_t tl;          // tiles of the segment left, the current one included (uniform)
+    uint32_t last_rows;   // valid rows of the segment's last tile (uniform)
+    uint32_t fast;        // cnt3 >= 128: one carry at most per tile advance
+    uint32_t lim3, dec3, dsn3, lim2, cnt2, dsn2, lim1, dec1, dsn1;  // carry constants (uniform)
+    uint64_t ub;          // box ordinal of the current tile's row 0 (general advance only)
+
+    __device__ __forceinline__ void pack(const SegP& g, const uint32_t (&v)[kKMax], uint32_t r) {
+        a1 = 0x64006400u + v[0] + (v[1] << 16);
+        a2 = 0x64006400u + v[2] + (v[3] << 16);
+        sn = (uint32_t)(g.n_base + 1) + v[0] + v[1] + v[2] + v[3];
+        if (tl == 1 && r >= last_rows) sn = 0u;
+    }
+    __device__ __forceinline__ void enter(const Plan& P, int seg, uint64_t w, uint32_t r) {
+        const SegP& g = P.seg[seg];
+        s = seg;
+        const uint64_t o = w - g.tile0;
+        const uint64_t n = g.u_end - g.u_begin;
+        const uint64_t nt = (n + kTileM - 1) / kTileM;
+        tl = (uint32_t)(nt - o);
+        last_rows = (uint32_t)(n - (nt - 1) * kTileM);
+        ub = g.u_begin + o * kTileM;
+        fast = g.fast_carry;
+        lim3 = (0x6400u + g.cnt[3]) << 16;
+        dec3 = (g.cnt[3] << 16) - 1u;
+        dsn3 = g.cnt[3] - 1u;
+        lim2 = 0x6400u + g.cnt[2];
+        cnt2 = g.cnt[2];
+        dsn2 = g.cnt[2] - 1u;
+        lim1 = (0x6400u + g.cnt[1]) << 16;
+        dec1 = (g.cnt[1] << 16) - 1u;
+        dsn1 = g.cnt[1] - 1u;
+        uint32_t v[kKMax];
+        decode_box<kKMax>(g, ub, r, v);
+        pack(g, v, r);
+    }
+    __device__ __forceinline__ void begin(const Plan& P, uint64_t w, uint32_t r) { enter(P, find_segment(P, w), w, r); }
+    // move to the next tile (w + 1 of the plan)
+    __device__ __forceinline__ void next(const Plan& P, uint32_t r) {
+        if (tl == 1) {
+            const int ns = s + 1;
+            enter(P, ns, P.seg[ns].tile0, r);
+            return;
+        }
+        tl--;
+        ub += kTileM;
+        if (fast) {
+            a2 += (uint32_t)kTileM << 16;
+            sn += kTileM;
+            const bool c3 = a2 >= lim3;  // the low half (0x6400 + v2) never reaches bit 16
+            if (c3) { a2 -= dec3; sn -= dsn3; }  // v3 -= cnt3, v2 += 1
+            const bool c2 = (a2 & 0xFFFFu) >= lim2;
+            if (c2) { a2 -= cnt2; a1 += 0x10000u; sn -= dsn2; }  // v2 -= cnt2, v1 += 1
+            const bool c1 = a1 >= lim1;
+            if (c1) { a1 -= dec1; sn -= dsn1; }  // v1 -= cnt1, v0 += 1 (v0 stays in the box)
+        } else {
+            const SegP& g = P.seg[s];
+            uint32_t v[kKMax] = {(a1 & 0xFFFFu) - 0x6400u, (a1 >> 16) - 0x6400u, (a2 & 0xFFFFu) - 0x6400u,
+                                 (a2 >> 16) - 0x6400u};
+            uint32_t carry = kTileM;
+#pragma unroll
+            for (int j = kKMax - 1; j >= 0; j--) {
+                const uint32_t x = v[j] + carry;
+                const uint32_t q = fastdiv(x, g.fd[j]);
+                v[j] = x - q * g.cnt[j];
+                carry = q;
+            }
+            a1 = 0x64006400u + v[0] + (v[1] << 16);
+            a2 = 0x64006400u + v[2] + (v[3] << 16);
+            sn = (uint32_t)(g.n_base + 1) + v[0] + v[1] + v[2] + v[3];
+        }
+        if (tl == 1 && last_rows < (uint32_t)kTileM && r >= last_rows) sn = 0u;
+    }
+};
+
+// fold one row of a packed tile: the key is built only when the row fits the
+// headroom and its sum_n can reach the running best
+__device__ __forceinline__ void fold_packed(const Plan& P, int s, uint32_t a1, uint32_t a2, uint32_t sn, float y,
+                                            unsigned long long& best, float& best_y, uint32_t& bsn) {
+    if (y <= P.H && sn >= bsn) {
+        const SegP& g = P.seg[s];
+        const uint64_t idx = g.t_base + (uint64_t)((a1 & 0xFFFFu) - 0x6400u) * g.istride[0] +
+                             (uint64_t)((a1 >> 16) - 0x6400u) * g.istride[1] +
+                             (uint64_t)((a2 & 0xFFFFu) - 0x6400u) * g.istride[2] +
+                             (uint64_t)((a2 >> 16) - 0x6400u) * g.istride[3];
+        const unsigned long long key = ((unsigned long long)sn << 40) | idx;
+        if (key > best) {
+            best = key;
+            best_y = y;
+            bsn = sn;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
 // Last-CTA epilogue shared by the fused kernels (a5 cross-CTA + a7 decode).
 // Each CTA publishes its best (key, y); the last CTA to arrive reduces them,
 // decodes the winning index into end ops per slot and resets the ticket.

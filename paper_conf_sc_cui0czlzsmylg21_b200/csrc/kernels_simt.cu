@@ -496,6 +496,128 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedBlocksPerSM) fused_fp32_k
     cta_publish_and_finish(P, S, best, best_y);
 }
 
+// Two candidates per thread (rows r of tiles w and w + 1): each weight of
+// layers 2-4 is read once from shared memory (LDS.128 broadcast, four weights)
+// and feeds two FFMAs, so the kernel is bound by the FMA pipe instead of the
+// constant cache that the one-candidate kernel reads every weight from.  The
+// per-candidate arithmetic (FMA order) is the one-candidate kernel's.
+constexpr int kFused2Threads = 128;
+constexpr int kFused2BlocksPerSM = 2;
+
+struct W234s {  // layers 2..4 in shared memory, rows 16-byte aligned
+    float4 W2[kHidden][kHidden / 4];
+    float4 W3[kHidden][kHidden / 4];
+    float b2[kHidden], b3[kHidden], w4[kHidden];
+    float b4;
+};
+
+__device__ __forceinline__ void mlp_tail_fp32_x2(const W234s& W, const float (&hx)[kHidden],
+                                                 const float (&hy)[kHidden], float& yx, float& yy) {
+    float gx[kHidden], gy[kHidden];
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) {
+        float sx = W.b2[i], sy = sx;
+#pragma unroll
+        for (int q = 0; q < kHidden / 4; q++) {
+            const float4 w = W.W2[i][q];
+            sx = fmaf(w.x, hx[4 * q + 0], sx); sy = fmaf(w.x, hy[4 * q + 0], sy);
+            sx = fmaf(w.y, hx[4 * q + 1], sx); sy = fmaf(w.y, hy[4 * q + 1], sy);
+            sx = fmaf(w.z, hx[4 * q + 2], sx); sy = fmaf(w.z, hy[4 * q + 2], sy);
+            sx = fmaf(w.w, hx[4 * q + 3], sx); sy = fmaf(w.w, hy[4 * q + 3], sy);
+        }
+        gx[i] = fmaxf(sx, 0.0f);
+        gy[i] = fmaxf(sy, 0.0f);
+    }
+    float ax = W.b4, ay = W.b4;
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) {
+        float sx = W.b3[i], sy = sx;
+#pragma unroll
+        for (int q = 0; q < kHidden / 4; q++) {
+            const float4 w = W.W3[i][q];
+            sx = fmaf(w.x, gx[4 * q + 0], sx); sy = fmaf(w.x, gy[4 * q + 0], sy);
+            sx = fmaf(w.y, gx[4 * q + 1], sx); sy = fmaf(w.y, gy[4 * q + 1], sy);
+            sx = fmaf(w.z, gx[4 * q + 2], sx); sy = fmaf(w.z, gy[4 * q + 2], sy);
+            sx = fmaf(w.w, gx[4 * q + 3], sx); sy = fmaf(w.w, gy[4 * q + 3], sy);
+        }
+        ax = fmaf(W.w4[i], fmaxf(sx, 0.0f), ax);
+        ay = fmaf(W.w4[i], fmaxf(sy, 0.0f), ay);
+    }
+    yx = ax;
+    yy = ay;
+}
+
+__device__ __forceinline__ void layer1_fp32(const float* c, const float* wc, const uint32_t (&v)[kKMax],
+                                            float (&h)[kHidden]) {
+#pragma unroll
+    for (int i = 0; i < kHidden; i++) {
+        float z = c[i];
+#pragma unroll
+        for (int j = 0; j < kKMax; j++) z = fmaf(wc[j * kHidden + i], (float)v[j], z);
+        h[i] = fmaxf(z, 0.0f);
+    }
+}
+
+__global__ void __launch_bounds__(kFused2Threads, kFused2BlocksPerSM) fused_fp32x2_kernel(
+    const __grid_constant__ Plan P, const __grid_constant__ W234 Wt, const float* __restrict__ w1b1, Scratch* S) {
+    __shared__ float s_c[kMaxSeg * kHidden];
+    __shared__ float s_w[kMaxSeg * kKMax * kHidden];
+    __shared__ W234s s_W;
+    build_l1_tables(P, w1b1, s_c, s_w);
+    for (int e = threadIdx.x; e < kHidden * kHidden; e += blockDim.x) {
+        const int i = e / kHidden, j = e % kHidden;
+        reinterpret_cast<float*>(&s_W.W2[i][0])[j] = Wt.W2[i][j];
+        reinterpret_cast<float*>(&s_W.W3[i][0])[j] = Wt.W3[i][j];
+    }
+    if (threadIdx.x < kHidden) {
+        s_W.b2[threadIdx.x] = Wt.b2[threadIdx.x];
+        s_W.b3[threadIdx.x] = Wt.b3[threadIdx.x];
+        s_W.w4[threadIdx.x] = Wt.w4[threadIdx.x];
+    }
+    if (threadIdx.x == 0) s_W.b4 = Wt.b4;
+    __syncthreads();
+
+    const uint32_t r = threadIdx.x;
+    unsigned long long best = 0;
+    float best_y = __int_as_float(0x7fc00000);
+    uint32_t bsn = 1u;
+    // work items are tile pairs (w, w + 1); the last pair may have only w.
+    // The packed walker (device_common.cuh) carries each row's digits and sum_n;
+    // rows past a segment's end have sn = 0, which no fold accepts.
+    auto unpack = [](uint32_t a1, uint32_t a2, uint32_t (&v)[kKMax]) {
+        v[0] = (a1 & 0xFFFFu) - 0x6400u;
+        v[1] = (a1 >> 16) - 0x6400u;
+        v[2] = (a2 & 0xFFFFu) - 0x6400u;
+        v[3] = (a2 >> 16) - 0x6400u;
+    };
+    const uint64_t n_pairs = (P.n_tiles + 1) / 2;
+    uint64_t pb, pe;
+    work_range(n_pairs, (uint64_t)blockIdx.x, (uint64_t)gridDim.x, pb, pe);
+    PackedWalker W;
+    if (pb < pe) W.begin(P, 2 * pb, r);
+    for (uint64_t p = pb; p < pe; p++) {
+        const uint64_t w = 2 * p;
+        if (p != pb) W.next(P, r);
+        const uint32_t x1 = W.a1, x2 = W.a2, xs = W.sn;
+        const int sX = W.s;
+        uint32_t v[kKMax];
+        unpack(x1, x2, v);
+        float hx[kHidden], hy[kHidden];
+        layer1_fp32(s_c + sX * kHidden, s_w + sX * kKMax * kHidden, v, hx);
+        const bool hasY = w + 1 < P.n_tiles;
+        if (hasY) W.next(P, r);
+        const uint32_t ys = hasY ? W.sn : 0u;
+        unpack(W.a1, W.a2, v);
+        layer1_fp32(s_c + W.s * kHidden, s_w + W.s * kKMax * kHidden, v, hy);
+        float yx, yy;
+        mlp_tail_fp32_x2(s_W, hx, hy, yx, yy);
+        if (w == 0 && P.want_y0 && r == 0) S->y0 = yx;
+        fold_packed(P, sX, x1, x2, xs, yx, best, best_y, bsn);
+        fold_packed(P, W.s, W.a1, W.a2, ys, yy, best, best_y, bsn);
+    }
+    cta_publish_and_finish(P, S, best, best_y);
+}
+
 // ---------------------------------------------------------------------------
 // a6 tail: after the NCCL all-gather of the per-rank Result records, every
 // rank reduces the same records to the same global decision.
@@ -866,6 +988,21 @@ cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const f
 
 cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,
                               cudaStream_t st, int* grid_out) {
+    uint32_t maxcnt = 0;
+    for (int s = 0; s < P.n_seg; s++)
+        for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
+#ifndef EXP_FP32X1
+    if (maxcnt < 32768u) {  // the packed walker holds a digit as 0x6400 + v in 16 bits
+
+        const uint64_t n_pairs = (P.n_tiles + 1) / 2;
+        uint64_t g = (uint64_t)nsm * kFused2BlocksPerSM;
+        if (n_pairs < g) g = n_pairs;
+        if (g < 1) g = 1;
+        *grid_out = (int)g;
+        fused_fp32x2_kernel<<<(int)g, kFused2Threads, 0, st>>>(P, W, w1b1, S);
+        return cudaGetLastError();
+    }
+#endif
     uint64_t g = (uint64_t)nsm * kFusedBlocksPerSM;
     if (P.n_tiles < g) g = P.n_tiles;
     if (g < 1) g = 1;
