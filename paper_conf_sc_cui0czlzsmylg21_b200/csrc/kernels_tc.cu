@@ -43,6 +43,7 @@ struct TcParams {
     float b4;             // output bias (fp32)
 };
 
+
 template <int FMT>
 struct TcCfg {
     static constexpr int kNchL1 = FMT == 0 ? 1 : 2;      // layer-1 B chunks per segment (fused)
@@ -166,18 +167,6 @@ __device__ __forceinline__ void issue_layer_p(uint32_t pred, uint32_t tD, uint32
         mma_ts_p(pred, tD, tA + 8, d[3], idesc, 1u);
         mma_ts_p(pred, tD, tC, d[4], idesc, 1u);
     }
-}
-
-// epilogue of a hidden layer: D (fp32, 32 columns) -> ReLU -> 16-bit pairs -> A
-template <int FMT>
-__device__ __forceinline__ void hidden_epilogue(uint32_t tD_lane, uint32_t tA_lane) {
-    uint32_t r[32];
-    tmem_ld32(tD_lane, r);
-    uint32_t h[16];
-#pragma unroll
-    for (int c = 0; c < 16; c++) h[c] = pack2_relu<FMT>(r[2 * c], r[2 * c + 1]);
-    tmem_st16(tA_lane, h);
-    tmem_wait_st();
 }
 
 // shared-memory carve-up common to both kernels
@@ -368,7 +357,10 @@ struct TcPipe {
     template <int LAYER, bool TWO>
     __device__ __forceinline__ void issue_next() const {
         constexpr uint32_t CH = LAYER == 2 ? kChunkBytesN16 : kChunkBytesN32;
-        constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32);
+        // fp16: hidden layers 2 and 3 accumulate in f16 (their epilogues then read
+        // half the TMEM bytes); layer 1 (the 1024 + v digits cancel there) and
+        // the output layer accumulate in fp32
+        constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32, FMT != 0 || LAYER == 2);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 0 && TWO) {
             if (LAYER == 2 && outbias) {
@@ -398,7 +390,19 @@ struct TcPipe {
     __device__ __forceinline__ void stage() {
         wait();
         stamp(LAYER, 0);
-        if (TWO) {
+        if (FMT == 0 && LAYER >= 1) {  // f16 accumulators of layer 2 / 3: ReLU on packed pairs
+            uint32_t a[16], b[16];
+            if (TWO) tmem_ld16p_x2(X.d + lane_off, Y.d + lane_off, a, b);
+            else tmem_ld16p_x2(X.d + lane_off, X.d + lane_off, a, b);
+#pragma unroll
+            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(a[c]) : "r"(0u));
+            tmem_st16(X.a + lane_off, a);
+            if (TWO) {
+#pragma unroll
+                for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(b[c]) : "r"(0u));
+                tmem_st16(Y.a + lane_off, b);
+            }
+        } else if (TWO) {
             uint32_t a[32], b[32], h[16];
             tmem_ld32x2(X.d + lane_off, Y.d + lane_off, a, b);
 #pragma unroll

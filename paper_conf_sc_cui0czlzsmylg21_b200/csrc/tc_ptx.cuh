@@ -19,10 +19,10 @@ __host__ __device__ constexpr uint32_t b_offset(int n, int k) {
 constexpr uint32_t kChunkBytesN32 = 32 * 16 * 2;  // 1 KB
 constexpr uint32_t kChunkBytesN16 = 16 * 16 * 2;  // 512 B
 
-// instruction descriptor, kind::f16: D fp32, A/B fp16 (fmt 0) or bf16 (fmt 1),
+// instruction descriptor, kind::f16: D fp32 (or f16: f32_accum false), A/B fp16 (fmt 0) or bf16 (fmt 1),
 // both K-major, M = 128.
-__host__ __device__ constexpr uint32_t idesc_f16(int fmt, int N) {
-    return (1u << 4) | ((uint32_t)fmt << 7) | ((uint32_t)fmt << 10) | ((uint32_t)(N >> 3) << 17) |
+__host__ __device__ constexpr uint32_t idesc_f16(int fmt, int N, bool f32_accum = true) {
+    return ((uint32_t)f32_accum << 4) | ((uint32_t)fmt << 7) | ((uint32_t)fmt << 10) | ((uint32_t)(N >> 3) << 17) |
            ((uint32_t)(128 >> 4) << 24);
 }
 
@@ -341,6 +341,22 @@ __device__ __forceinline__ void tmem_ld32x2(uint32_t ta, uint32_t tb, uint32_t (
           "=r"(b[14]), "=r"(b[15]), "=r"(b[16]), "=r"(b[17]), "=r"(b[18]), "=r"(b[19]), "=r"(b[20]),
           "=r"(b[21]), "=r"(b[22]), "=r"(b[23]), "=r"(b[24]), "=r"(b[25]), "=r"(b[26]), "=r"(b[27]),
           "=r"(b[28]), "=r"(b[29]), "=r"(b[30]), "=r"(b[31])
+        : "r"(ta), "r"(tb)
+        : "memory");
+}
+// two 32-column loads of f16 accumulators (value in the low half of each
+// column), adjacent columns packed into one register (.pack::16b)
+__device__ __forceinline__ void tmem_ld16p_x2(uint32_t ta, uint32_t tb, uint32_t (&a)[16], uint32_t (&b)[16]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.pack::16b.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%32];\n\t"
+        "tcgen05.ld.sync.aligned.32x32b.x16.pack::16b.b32 "
+        "{%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%33];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(a[0]), "=r"(a[1]), "=r"(a[2]), "=r"(a[3]), "=r"(a[4]), "=r"(a[5]), "=r"(a[6]), "=r"(a[7]),
+          "=r"(a[8]), "=r"(a[9]), "=r"(a[10]), "=r"(a[11]), "=r"(a[12]), "=r"(a[13]), "=r"(a[14]), "=r"(a[15]),
+          "=r"(b[0]), "=r"(b[1]), "=r"(b[2]), "=r"(b[3]), "=r"(b[4]), "=r"(b[5]), "=r"(b[6]), "=r"(b[7]),
+          "=r"(b[8]), "=r"(b[9]), "=r"(b[10]), "=r"(b[11]), "=r"(b[12]), "=r"(b[13]), "=r"(b[14]), "=r"(b[15])
         : "r"(ta), "r"(tb)
         : "memory");
 }
