@@ -509,8 +509,14 @@ std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, f
             const float bb = (float)((double)b[n] * sout);
             const uint16_t bh = conv(bb);
             const size_t cb = base + (size_t)(nch - 1) * tc::kChunkBytesN32;
-            put(cb, n, 0, bh);
-            put(cb, n, 1, conv(bb - back(bh)));
+            if (fmt == 0) {
+                // fp16: no bias MMA; the chunk holds the f16 biases as 16 pairs (unit 2i
+                // low, 2i + 1 high) that the epilogue adds with HFMA2.RELU
+                memcpy(blob.data() + cb + 2 * (size_t)n, &bh, 2);
+            } else {
+                put(cb, n, 0, bh);
+                put(cb, n, 1, conv(bb - back(bh)));
+            }
         }
     };
     hidden(0, W2, b2, s1, s2);

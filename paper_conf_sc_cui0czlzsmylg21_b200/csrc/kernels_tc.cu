@@ -272,6 +272,7 @@ struct TcPipe {
     uint32_t tCx, tCy, lane_off, bar_id, ph;  // bias constant chunk of X / Y (may be shared)
     uint64_t* bar;
     uint64_t db2, db3, db4;
+    uint32_t hb_smem, hb_step;  // fp16: shared address of layer 2's bias words, layer 3's offset
     bool me[4];
     // fp16: the output layer runs without its bias K chunk and b4 is added to y
     // in fp32 when y is read (one MMA fewer per tile)
@@ -318,6 +319,9 @@ struct TcPipe {
         db2 = d2;
         db3 = d3;
         db4 = d4;
+        // fp16: the bias chunk of each hidden layer holds its 16 f16 bias pairs instead
+        hb_smem = ((uint32_t)(d2 & 0x3FFFu) << 4) + 2u * kChunkBytesN32;
+        hb_step = (((uint32_t)(d3 & 0x3FFFu) - (uint32_t)(d2 & 0x3FFFu)) << 4);
 #pragma unroll
         for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
     }
@@ -363,13 +367,13 @@ struct TcPipe {
         constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32, FMT != 0 || LAYER == 2);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 0 && TWO) {
-            if (LAYER == 2 && outbias) {
+            if (LAYER < 2 || outbias) {
                 issue_layer2_asm<0, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
                 return;
             }
             issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
         } else if (!TWO) {
-            if (FMT == 0 && LAYER == 2 && outbias) {
+            if (FMT == 0 && (LAYER < 2 || outbias)) {
                 issue_layer_asm<FMT, ID, CH, false>(X.d, X.a, tCx, db, bar);
                 return;
             }
@@ -388,18 +392,25 @@ struct TcPipe {
     // chunk shares the columns of the consumed layer-1 operand)
     template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage() {
+        uint32_t hbw[16];
+        if (FMT == 0 && LAYER >= 1) lds_words16(hb_smem + (LAYER == 1 ? 0u : hb_step), hbw);
         wait();
         stamp(LAYER, 0);
-        if (FMT == 0 && LAYER >= 1) {  // f16 accumulators of layer 2 / 3: ReLU on packed pairs
+        if (FMT == 0 && LAYER >= 1) {
+            // f16 accumulators of layer 2 / 3 (no bias MMA): bias + ReLU on packed
+            // pairs, one HFMA2.RELU per pair; the 16 bias words were loaded from
+            // shared memory before the mbarrier wait
             uint32_t a[16], b[16];
             if (TWO) tmem_ld16p_x2(X.d + lane_off, Y.d + lane_off, a, b);
             else tmem_ld16p_x2(X.d + lane_off, X.d + lane_off, a, b);
+            const uint32_t one = 0x3C003C00u;
 #pragma unroll
-            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(a[c]) : "r"(0u));
+            for (int c = 0; c < 16; c++) asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(a[c]) : "r"(one), "r"(hbw[c]));
             tmem_st16(X.a + lane_off, a);
             if (TWO) {
 #pragma unroll
-                for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(b[c]) : "r"(0u));
+                for (int c = 0; c < 16; c++)
+                    asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(b[c]) : "r"(one), "r"(hbw[c]));
                 tmem_st16(Y.a + lane_off, b);
             }
         } else if (TWO) {

@@ -344,6 +344,19 @@ __device__ __forceinline__ void tmem_ld32x2(uint32_t ta, uint32_t tb, uint32_t (
         : "r"(ta), "r"(tb)
         : "memory");
 }
+// 16 consecutive 32-bit words from shared memory (four 16-byte loads); volatile
+// so it stays ahead of a following mbarrier wait
+__device__ __forceinline__ void lds_words16(uint32_t saddr, uint32_t (&w)[16]) {
+    asm volatile(
+        "ld.shared.v4.b32 {%0,%1,%2,%3}, [%16];\n\t"
+        "ld.shared.v4.b32 {%4,%5,%6,%7}, [%16+16];\n\t"
+        "ld.shared.v4.b32 {%8,%9,%10,%11}, [%16+32];\n\t"
+        "ld.shared.v4.b32 {%12,%13,%14,%15}, [%16+48];"
+        : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7]),
+          "=r"(w[8]), "=r"(w[9]), "=r"(w[10]), "=r"(w[11]), "=r"(w[12]), "=r"(w[13]), "=r"(w[14]), "=r"(w[15])
+        : "r"(saddr)
+        : "memory");
+}
 // two 32-column loads of f16 accumulators (value in the low half of each
 // column), adjacent columns packed into one register (.pack::16b)
 __device__ __forceinline__ void tmem_ld16p_x2(uint32_t ta, uint32_t tb, uint32_t (&a)[16], uint32_t (&b)[16]) {
