@@ -392,6 +392,12 @@ struct TcPipe {
     // chunk shares the columns of the consumed layer-1 operand)
     template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage() {
+        stage_as<LAYER, TWO, CONST>(me[LAYER]);
+    }
+    // the same with the issuer role given by the caller (a compile-time
+    // constant in the fused kernel's role-specialised loop)
+    template <int LAYER, bool TWO, bool CONST = false>
+    __device__ __forceinline__ void stage_as(bool mine) {
         uint32_t hbw[16];
         if (FMT == 0 && LAYER >= 1) lds_words16(hb_smem + (LAYER == 1 ? 0u : hb_step), hbw);
         wait();
@@ -436,7 +442,7 @@ struct TcPipe {
         }
         tmem_wait_st();
         stamp(LAYER, 1);
-        if (handoff(me[LAYER])) {
+        if (handoff(mine)) {
             stamp(LAYER, 2);
             issue_next<LAYER, TWO>();
         }
@@ -546,6 +552,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             if (blockIdx.x == 0 && g == 0) pp.tr = P.trace;
             pp.wqq = wq;
 #endif
+            // issuer roles fixed per warp: stage p (0..2 = layers 2, 3, out; 3 =
+            // the next layer 1) is issued by the group's warp wq == p, so every
+            // SMSP issues one stage of every group; the role test is one
+            // compare of the warp-uniform wq with an immediate
             PackedWalker W;
             W.begin(P, wb, r);
             uint32_t x1, x2, xs, y1 = 0, y2 = 0, ys = 0;  // X / Y rows: a1, a2, sn
@@ -560,20 +570,24 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                 takeY();
             }
             tmem_wait_st();
-            if (pp.handoff(pp.me[3])) {
+            if (pp.handoff(wq == 3)) {
                 issue_l1(pp.X, sX);
                 if (yLive) issue_l1(pp.Y, sY);
                 pp.commit();
             }
-            uint64_t w = wb;
+            // 32-bit iteration state (a group's range is < 2^32 tiles); y(0) is owed
+            // only by the row that holds index 0 (the plan's first tile)
+            const uint32_t nw = (uint32_t)(we - wb);
+            uint32_t w = 0;
+            bool owe_y0 = wb == 0 && P.want_y0 && r == 0;
             auto iteration = [&](auto two_c, auto next_two_c) {
                 constexpr bool TWO = decltype(two_c)::value;
                 constexpr bool NTWO = decltype(next_two_c)::value;
-                pp.template stage<0, TWO>();
-                pp.template stage<1, TWO>();
-                pp.template stage<2, TWO>();
+                pp.template stage_as<0, TWO>(wq == 0);
+                pp.template stage_as<1, TWO>(wq == 1);
+                pp.template stage_as<2, TWO>(wq == 2);
                 // the next tiles' operand rows are computed while the output MMA runs
-                const bool more = w + 2 < we;  // warp-uniform
+                const bool more = w + 2 < nw;  // warp-uniform
                 uint32_t n1 = 0, n2 = 0, ns = 0;
                 int nsX = 0;
                 if (more) {
@@ -591,7 +605,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                 else tmem_ld1(pp.X.d + pp.lane_off, ybx);
                 ybx = pp.add_b4(ybx);
                 if (TWO) yby = pp.add_b4(yby);
-                if (w == 0 && P.want_y0 && r == 0) S->y0 = __uint_as_float(ybx);
+                if (owe_y0) {
+                    S->y0 = __uint_as_float(ybx);
+                    owe_y0 = false;
+                }
                 fold_packed(P, sX, x1, x2, xs, __uint_as_float(ybx), best, best_y, bsn);
                 if (TWO) fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
                 if (more) {
@@ -603,7 +620,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                     if (NTWO) takeY();
                     tmem_wait_st();
                     pp.stamp(3, 1);
-                    if (pp.handoff(pp.me[3])) {
+                    if (pp.handoff(wq == 3)) {
                         pp.stamp(3, 2);
                         issue_l1(pp.X, sX);
                         if (NTWO) issue_l1(pp.Y, sY);
@@ -615,9 +632,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
 #endif
                 w += 2;
             };
-            while (w + 3 < we) iteration(T2{}, T2{});
-            if (w + 1 < we) iteration(T2{}, T1{});
-            if (w < we) iteration(T1{}, T1{});
+            while (w + 3 < nw) iteration(T2{}, T2{});
+            if (w + 1 < nw) iteration(T2{}, T1{});
+            if (w < nw) iteration(T1{}, T1{});
+
         }
     } else if (wb < we) {
         Walker W;
