@@ -558,20 +558,27 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             // compare of the warp-uniform wq with an immediate
             PackedWalker W;
             W.begin(P, wb, r);
-            uint32_t x1, x2, xs, y1 = 0, y2 = 0, ys = 0;  // X / Y rows: a1, a2, sn
-            int sX, sY = 0;
+            // X rows alternate between two register sets (the loop is unrolled by
+            // two with the roles swapped), so the next X row needs no copy
+            struct Row {
+                uint32_t a1, a2, sn;
+                int s;
+            };
+            Row RA, RB{0u, 0u, 0u, 0};
+            uint32_t y1 = 0, y2 = 0, ys = 0;  // Y row: a1, a2, sn
+            int sY = 0;
             uint32_t bsn = 1u;
-            auto takeX = [&]() { x1 = W.a1; x2 = W.a2; xs = W.sn; sX = W.s; store_a1_packed(pp.X.a1 + pp.lane_off, W.a1, W.a2); };
             auto takeY = [&]() { y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s; store_a1_packed(pp.Y.a1 + pp.lane_off, W.a1, W.a2); };
             const bool yLive = wb + 1 < we;  // warp-uniform
-            takeX();
+            RA = Row{W.a1, W.a2, W.sn, W.s};
+            store_a1_packed(pp.X.a1 + pp.lane_off, RA.a1, RA.a2);
             if (yLive) {
                 W.next(P, r);
                 takeY();
             }
             tmem_wait_st();
             if (pp.handoff(wq == 3)) {
-                issue_l1(pp.X, sX);
+                issue_l1(pp.X, RA.s);
                 if (yLive) issue_l1(pp.Y, sY);
                 pp.commit();
             }
@@ -580,7 +587,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             const uint32_t nw = (uint32_t)(we - wb);
             uint32_t w = 0;
             bool owe_y0 = wb == 0 && P.want_y0 && r == 0;
-            auto iteration = [&](auto two_c, auto next_two_c) {
+            auto iteration = [&](auto two_c, auto next_two_c, Row& cx, Row& nx) {
                 constexpr bool TWO = decltype(two_c)::value;
                 constexpr bool NTWO = decltype(next_two_c)::value;
                 pp.template stage_as<0, TWO>(wq == 0);
@@ -588,14 +595,9 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                 pp.template stage_as<2, TWO>(wq == 2);
                 // the next tiles' operand rows are computed while the output MMA runs
                 const bool more = w + 2 < nw;  // warp-uniform
-                uint32_t n1 = 0, n2 = 0, ns = 0;
-                int nsX = 0;
                 if (more) {
                     W.next(P, r);
-                    n1 = W.a1;
-                    n2 = W.a2;
-                    ns = W.sn;
-                    nsX = W.s;
+                    nx = Row{W.a1, W.a2, W.sn, W.s};
                     if (NTWO) W.next(P, r);
                 }
                 pp.wait();
@@ -609,20 +611,16 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                     S->y0 = __uint_as_float(ybx);
                     owe_y0 = false;
                 }
-                fold_packed(P, sX, x1, x2, xs, __uint_as_float(ybx), best, best_y, bsn);
+                fold_packed(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y, bsn);
                 if (TWO) fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
                 if (more) {
-                    x1 = n1;
-                    x2 = n2;
-                    xs = ns;
-                    sX = nsX;
-                    store_a1_packed(pp.X.a1 + pp.lane_off, x1, x2);
+                    store_a1_packed(pp.X.a1 + pp.lane_off, nx.a1, nx.a2);
                     if (NTWO) takeY();
                     tmem_wait_st();
                     pp.stamp(3, 1);
                     if (pp.handoff(wq == 3)) {
                         pp.stamp(3, 2);
-                        issue_l1(pp.X, sX);
+                        issue_l1(pp.X, nx.s);
                         if (NTWO) issue_l1(pp.Y, sY);
                         pp.commit();
                     }
@@ -632,9 +630,27 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
 #endif
                 w += 2;
             };
-            while (w + 3 < nw) iteration(T2{}, T2{});
-            if (w + 1 < nw) iteration(T2{}, T1{});
-            if (w < nw) iteration(T1{}, T1{});
+            // the tail: at most one pair with a lone successor, then a lone X
+            auto tail = [&](Row& cx, Row& nx) {
+                if (w + 1 < nw) {
+                    iteration(T2{}, T1{}, cx, nx);
+                    if (w < nw) iteration(T1{}, T1{}, nx, cx);
+                } else if (w < nw) {
+                    iteration(T1{}, T1{}, cx, nx);
+                }
+            };
+            for (;;) {
+                if (!(w + 3 < nw)) {
+                    tail(RA, RB);
+                    break;
+                }
+                iteration(T2{}, T2{}, RA, RB);
+                if (!(w + 3 < nw)) {
+                    tail(RB, RA);
+                    break;
+                }
+                iteration(T2{}, T2{}, RB, RA);
+            }
 
         }
     } else if (wb < we) {
