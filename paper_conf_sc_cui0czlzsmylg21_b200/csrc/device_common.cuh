@@ -249,6 +249,21 @@ __device__ __forceinline__ void fold_packed(const Plan& P, int s, uint32_t a1, u
     }
 }
 
+// fold the two lock-step rows of a thread with one divergent branch: the cheap
+// tests of both rows first, the key construction only for a row that passes
+// (the key comparison inside is authoritative, so testing Y against the bsn
+// from before X's fold is safe)
+__device__ __forceinline__ void fold_packed2(const Plan& P, int sx, uint32_t x1, uint32_t x2, uint32_t xs, float yx,
+                                             int sy, uint32_t y1, uint32_t y2, uint32_t ys, float yy,
+                                             unsigned long long& best, float& best_y, uint32_t& bsn) {
+    const bool cx = yx <= P.H && xs >= bsn;
+    const bool cy = yy <= P.H && ys >= bsn;
+    if (cx || cy) {
+        if (cx) fold_packed(P, sx, x1, x2, xs, yx, best, best_y, bsn);
+        if (cy) fold_packed(P, sy, y1, y2, ys, yy, best, best_y, bsn);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // Last-CTA epilogue shared by the fused kernels (a5 cross-CTA + a7 decode).
 // Each CTA publishes its best (key, y); the last CTA to arrive reduces them,

@@ -611,8 +611,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                     S->y0 = __uint_as_float(ybx);
                     owe_y0 = false;
                 }
-                fold_packed(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y, bsn);
-                if (TWO) fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
+                if (TWO)
+                    fold_packed2(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), sY, y1, y2, ys,
+                                 __uint_as_float(yby), best, best_y, bsn);
+                else
+                    fold_packed(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y, bsn);
                 if (more) {
                     store_a1_packed(pp.X.a1 + pp.lane_off, nx.a1, nx.a2);
                     if (NTWO) takeY();
