@@ -1522,8 +1522,17 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
     const TcSmem L =
         tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, kFusedNG, w1_stage_bytes(P.D, kFusedNG));
     auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    // the shared-memory opt-in is a host API call on the decision path: raise it
+    // only when a launch needs more than this device has been given so far
+    static int s_granted[64] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= 64 || s_granted[dev] < (int)L.total) {
+        e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+        if (e != cudaSuccess) return e;
+        if (dev >= 0 && dev < 64) s_granted[dev] = (int)L.total;
+    }
     // spread the tiles over as many SMs as possible (one tile per group first)
     uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;

@@ -23,10 +23,11 @@ raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_outpu
 rr = list(csv.reader(io.StringIO(raw)))
 if len(rr) > 2:
     hh = rr[0]
+    units = dict(zip(hh, rr[1]))
     vals = dict(zip(hh, rr[2]))
     for k in hh:
         if re.search(r"pipe_tensor.*active|dram__bytes_(read|write)\.sum$|sm__inst_executed_pipe_(alu|fma|fp16|uniform|xu).*sum$", k):
-            print("%-70s %s" % (k, vals[k]))
+            print("%-70s %s %s" % (k, vals[k], units.get(k, "")))
 src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=sass"], capture_output=True,
                      text=True).stdout
 srows = list(csv.reader(io.StringIO(src)))
