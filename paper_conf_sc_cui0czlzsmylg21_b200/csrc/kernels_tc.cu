@@ -272,7 +272,7 @@ struct TcPipe {
     uint32_t tCx, tCy, lane_off, bar_id, ph;  // bias constant chunk of X / Y (may be shared)
     uint64_t* bar;
     uint64_t db2, db3, db4;
-    uint32_t hb_smem, hb_step;  // fp16: shared address of layer 2's bias words, layer 3's offset
+    uint32_t hb_smem;  // fp16: shared address of layer 2's bias words (layer 3's follow one blob later)
     bool me[4];
     // fp16: the output layer runs without its bias K chunk and b4 is added to y
     // in fp32 when y is read (one MMA fewer per tile)
@@ -321,7 +321,6 @@ struct TcPipe {
         db4 = d4;
         // fp16: the bias chunk of each hidden layer holds its 16 f16 bias pairs instead
         hb_smem = ((uint32_t)(d2 & 0x3FFFu) << 4) + 2u * kChunkBytesN32;
-        hb_step = (((uint32_t)(d3 & 0x3FFFu) - (uint32_t)(d2 & 0x3FFFu)) << 4);
 #pragma unroll
         for (int p = 0; p < 4; p++) me[p] = ((g + p) & 3) == wq;
     }
@@ -399,7 +398,9 @@ struct TcPipe {
     template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage_as(bool mine) {
         uint32_t hbw[16];
-        if (FMT == 0 && LAYER >= 1) lds_words16(hb_smem + (LAYER == 1 ? 0u : hb_step), hbw);
+        // layer 3's bias words sit one hidden-layer blob (kNchHid chunks) after layer 2's
+        if (FMT == 0 && LAYER >= 1)
+            lds_words16(hb_smem + (LAYER == 1 ? 0u : (uint32_t)TcCfg<FMT>::kNchHid * kChunkBytesN32), hbw);
         wait();
         stamp(LAYER, 0);
         if (FMT == 0 && LAYER >= 1) {
