@@ -10,6 +10,9 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:fused_tc -s 1 -c 1 -o gpurun_out/${TAG}_fused_fp16 python tools/profile_run.py --precision fp16 --frac 32 --reps 1 > gpurun_out/${TAG}_ncu_fused.log 2>&1
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:predict -s 1 -c 1 -o gpurun_out/${TAG}_predict_fp16 python tools/profile_run.py --precision fp16 --frac 100000 --reps 0 --predict > gpurun_out/${TAG}_ncu_predict.log 2>&1
 timeout 600 python tools/bench_kernels.py --out gpurun_out/${TAG}_kernels.json > gpurun_out/${TAG}_kernels.log 2>&1
+for k in encode_grid24 select_kernel encode_groups24; do
+  timeout 600 ncu --set full --clock-control none -k regex:$k -c 1 -o gpurun_out/${TAG}_$k python tools/bench_kernels.py --rows 16777216 --reps 1 > gpurun_out/${TAG}_ncu_$k.log 2>&1
+done
 timeout 600 python tools/accuracy_replay.py --out gpurun_out/${TAG}_acc.json > gpurun_out/${TAG}_acc.log 2>&1
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err
 for p in bf16 fp32; do
