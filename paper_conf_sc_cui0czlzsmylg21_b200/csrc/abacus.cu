@@ -448,7 +448,7 @@ int scale_exp(double bound) {
 }
 
 // blob: [W2 chunks][W3 chunks][out chunks]; chunk = N rows x 16 K, b_offset layout
-std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, float* w4s, float* b4_out) {
+std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, float* b4_out) {
     const int D = c->D;
     const float* p = c->params.data();
     const float* W1 = p;
@@ -484,7 +484,6 @@ std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, f
         s3 = std::ldexp(1.0, -scale_exp(B3));
     }
     *l1_scale = (float)s1;
-    for (int j = 0; j < kHidden; j++) w4s[j] = (float)((double)w4[j] / s3);  // exact: s3 is a power of two
     *b4_out = b4;
     const int nch = fmt == 0 ? 3 : 5;
     const size_t hid_bytes = (size_t)nch * tc::kChunkBytesN32;
@@ -873,7 +872,7 @@ int abacus_load_predictor(abacus_ctx* c, const float* params, size_t n_params, i
     for (int fmt = 0; fmt < 2; fmt++) {
         float l1s = 1.0f;
         TcWeights tw{};
-        std::vector<uint8_t> blob = build_blob(c, fmt, &l1s, tw.w4s, &tw.b4);
+        std::vector<uint8_t> blob = build_blob(c, fmt, &l1s, &tw.b4);
         if (c->d_blob[fmt]) cudaFree(c->d_blob[fmt]);
         CUDA_TRY(c, cudaMalloc(&c->d_blob[fmt], blob.size()));
         CUDA_TRY(c, cudaMemcpy(c->d_blob[fmt], blob.data(), blob.size(), cudaMemcpyHostToDevice));

@@ -25,7 +25,6 @@ struct TcWeights {
     int nch_out;       // B chunks of the output layer (fp16 3, bf16 5)
     uint32_t bytes;    // blob size
     float l1_scale;    // 2^-s1 applied to layer-1 weights (fp16), 1 (bf16)
-    float w4s[kHidden];  // output weights w4 * 2^s3 (fp32, fused SIMT output layer)
     float b4;
     const uint8_t* blob;  // device
 };
