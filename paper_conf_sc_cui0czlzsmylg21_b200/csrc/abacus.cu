@@ -44,8 +44,8 @@ struct abacus_ctx {
     cudaStream_t stream = nullptr;      // stream of the blocking calls (default: own_stream)
     cudaStream_t own_stream = nullptr;
     Scratch* S = nullptr;         // device
-    Result* host_result = nullptr;  // pinned, host-mapped: the kernels write the decision here
-    Result* dev_result = nullptr;   // device alias of host_result
+    MappedRec* host_result = nullptr;  // pinned, host-mapped: the kernels write the decision here
+    MappedRec* dev_result = nullptr;   // device alias of host_result
     uint32_t seq = 0;
     std::string err;
     uint64_t launches = 0;
@@ -541,27 +541,40 @@ std::vector<uint8_t> build_blob(const abacus_ctx* c, int fmt, float* l1_scale, f
 cudaStream_t pick_stream(abacus_ctx* c, void* st) { return st ? (cudaStream_t)st : c->stream; }
 
 // Wait until the kernel-side publish of sequence number `seq` is visible in
-// the mapped result (spin; the stream is polled now and then so a failed or
-// finished-without-result launch is reported instead of hanging).
-// sequence numbers are unique per process, so a recycled pinned buffer can
-// never hold a matching stale tag
+// the mapped record and copy it out (spin; the stream is polled now and then
+// so a failed or finished-without-result launch is reported instead of
+// hanging). Sequence numbers are unique per process, so a recycled pinned
+// buffer can never hold chunks whose tags match a new number.
 std::atomic<uint32_t> g_seq{0};
-uint32_t next_seq(abacus_ctx* c) {
+uint32_t next_seq(abacus_ctx*) {
     uint32_t s = ++g_seq;
     if (s == 0) s = ++g_seq;
-    c->host_result->seq = 0;  // cleared before the launch that will publish `s`
     return s;
 }
 
-int wait_result(abacus_ctx* c, uint32_t seq) {
-    volatile uint32_t* s = &c->host_result->seq;
+// all four chunks of the record carry the tag of `seq` -> payload into *R
+bool read_record(const MappedRec* M, uint32_t seq, Result* R) {
+    const volatile uint32_t* w = M->w;
+    uint32_t p[12];
+    for (uint32_t i = 0; i < 4; i++) {
+        const uint32_t a = w[4 * i], b = w[4 * i + 1], cc = w[4 * i + 2], t = w[4 * i + 3];
+        if (t != rec_tag(seq, a, b, cc, i)) return false;
+        p[3 * i] = a;
+        p[3 * i + 1] = b;
+        p[3 * i + 2] = cc;
+    }
+    rec_unpayload(p, *R);
+    return true;
+}
+
+int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
     for (uint64_t spin = 1;; spin++) {
-        if (*s == seq) break;
+        if (read_record(c->host_result, seq, R)) break;
         if ((spin & 1023) == 0) {
             const cudaError_t e = cudaStreamQuery(c->stream);
             if (e != cudaSuccess && e != cudaErrorNotReady)
                 return fail(c, ABACUS_E_CUDA, "search kernel failed: %s", cudaGetErrorString(e));
-            if (e == cudaSuccess && *s != seq)
+            if (e == cudaSuccess && !read_record(c->host_result, seq, R))
                 return fail(c, ABACUS_E_CUDA, "search finished without publishing its result");
         }
     }
@@ -780,7 +793,7 @@ int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, in
     bool ok = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking) == cudaSuccess &&
               cudaMalloc(&c->S, sizeof(Scratch)) == cudaSuccess &&
               cudaMemset(c->S, 0, sizeof(Scratch)) == cudaSuccess &&
-              cudaHostAlloc(&c->host_result, sizeof(Result), cudaHostAllocMapped) == cudaSuccess &&
+              cudaHostAlloc(&c->host_result, sizeof(MappedRec), cudaHostAllocMapped) == cudaSuccess &&
               cudaHostGetDevicePointer(&c->dev_result, c->host_result, 0) == cudaSuccess &&
               cudaEventCreate(&c->ev0) == cudaSuccess && cudaEventCreate(&c->ev1) == cudaSuccess;
     if (ok) {
@@ -788,7 +801,7 @@ int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, in
         ok = cudaMemcpy(&c->S->y0, &nan, sizeof(float), cudaMemcpyHostToDevice) == cudaSuccess;
     }
     c->stream = c->own_stream;
-    if (ok) memset(c->host_result, 0, sizeof(Result));
+    if (ok) memset(c->host_result, 0, sizeof(MappedRec));
     if (!ok) {
         abacus_destroy(c);
         return ABACUS_E_CUDA;
@@ -985,9 +998,10 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
     CUDA_TRY(c, cudaSetDevice(c->device));
     rc = launch_fused(c, P);
     if (rc) return rc;
-    rc = wait_result(c, P.seq);
+    Result R;
+    rc = wait_result(c, P.seq, &R);
     if (rc) return rc;
-    *out = assemble_decision(*c->host_result, order, k, H, n_eval);
+    *out = assemble_decision(R, order, k, H, n_eval);
     return ABACUS_OK;
 }
 
@@ -1083,9 +1097,9 @@ int abacus_search_mway(abacus_ctx* c, const abacus_query_t* q, int32_t k, double
     CUDA_TRY(c, cudaSetDevice(c->device));
     CUDA_TRY(c, launch_mway(P, c->w234, c->d_w1b1, ways, c->S, c->stream));
     c->launches++;
-    rc = wait_result(c, P.seq);
+    Result R;
+    rc = wait_result(c, P.seq, &R);
     if (rc) return rc;
-    const Result R = *c->host_result;
     abacus_decision_t d{};
     d.critical = order[0];
     for (int j = 0; j < 4; j++) d.order[j] = j < k ? order[j] : -1;
@@ -1133,9 +1147,9 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
         CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->dev_result, seq, c->stream));
         c->launches++;
     }
-    rc = wait_result(c, seq);
+    Result R;
+    rc = wait_result(c, seq, &R);
     if (rc) return rc;
-    const Result R = *c->host_result;
     abacus_decision_t d{};
     d.critical = 0;
     for (int j = 0; j < 4; j++) d.order[j] = j < grid->k ? j : -1;

@@ -15,6 +15,7 @@
 // uniform: this is what lets a 128-row tile share one layer-1 operand.
 #pragma once
 #include <cstdint>
+#include <cstring>
 
 namespace abacus {
 
@@ -64,9 +65,49 @@ struct Result {
     int32_t end_op[kKMax];   // decoded t* per slot (grid order), 0 absent
     int32_t total_ops;
     int32_t status;          // 0 OK, 2 NONE (set by host for decisions)
-    uint32_t seq;            // mapped copy: written last, after a system fence
+    uint32_t seq;            // unused in device records (the mapped copy carries tags)
     uint32_t pad;
 };
+
+// Host-mapped copy of a Result: four 16-byte chunks of three payload words and
+// a tag, tag = seq ^ mix(payload, chunk index). The device writes it with four
+// vector stores and no system fence; the host accepts the record once all four
+// tags match the sequence number it waits for (a stale or torn chunk fails its
+// tag), so no store ordering across the PCIe writes is needed.
+struct alignas(64) MappedRec {
+    uint32_t w[16];
+};
+__host__ __device__ inline uint32_t rec_tag(uint32_t seq, uint32_t a, uint32_t b, uint32_t c, uint32_t i) {
+    uint32_t h = (a * 0x9E3779B1u) ^ ((b + 0x7F4A7C15u) * 0x85EBCA77u) ^ ((c + i) * 0xC2B2AE3Du) ^ (i * 0x27D4EB2Fu);
+    h ^= h >> 15;
+    h *= 0x2C1B3C6Du;
+    h ^= h >> 12;
+    return seq ^ h;
+}
+// payload words: key lo/hi, y_best, y0, evaluated lo/hi, end_op[4], total_ops,
+// status | pad << 8 (pad: m-way rounds, < 2^24)
+__host__ __device__ inline void rec_payload(const Result& R, uint32_t (&p)[12]) {
+    p[0] = (uint32_t)R.key;
+    p[1] = (uint32_t)(R.key >> 32);
+    memcpy(&p[2], &R.y_best, 4);
+    memcpy(&p[3], &R.y0, 4);
+    p[4] = (uint32_t)R.evaluated;
+    p[5] = (uint32_t)(R.evaluated >> 32);
+    for (int j = 0; j < kKMax; j++) p[6 + j] = (uint32_t)R.end_op[j];
+    p[10] = (uint32_t)R.total_ops;
+    p[11] = ((uint32_t)R.status & 0xFFu) | (R.pad << 8);
+}
+__host__ __device__ inline void rec_unpayload(const uint32_t (&p)[12], Result& R) {
+    R.key = (unsigned long long)p[0] | ((unsigned long long)p[1] << 32);
+    memcpy(&R.y_best, &p[2], 4);
+    memcpy(&R.y0, &p[3], 4);
+    R.evaluated = (unsigned long long)p[4] | ((unsigned long long)p[5] << 32);
+    for (int j = 0; j < kKMax; j++) R.end_op[j] = (int32_t)p[6 + j];
+    R.total_ops = (int32_t)p[10];
+    R.status = (int32_t)(p[11] & 0xFFu);
+    R.pad = p[11] >> 8;
+    R.seq = 0;
+}
 
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
 
@@ -81,7 +122,7 @@ struct PlanHdr {
     uint64_t T;             // size of the whole space
     uint64_t n_eval;        // candidates in this plan (this shard)
     uint64_t chain_cum[kKMax + 1];  // CHAIN: first u of block j
-    Result* mapped;         // host-mapped pinned result (device pointer) or null
+    MappedRec* mapped;      // host-mapped pinned result record (device pointer) or null
     unsigned long long* trace;  // optional %globaltimer stamps (tools only), null in production
     uint32_t seq;           // sequence number the mapped copy is tagged with
     uint32_t pad2;

@@ -305,21 +305,16 @@ __device__ __forceinline__ void trace_stamp(const PlanHdr& P, int slot) {
     }
 }
 
-// copy a result record to host-mapped pinned memory; the sequence number is
-// written last, after a system-scope fence, so a host that sees it sees the
-// whole record
-__device__ __forceinline__ void publish_mapped(const Result& R, Result* M, uint32_t seq) {
-    volatile Result* m = M;
-    m->key = R.key;
-    m->y_best = R.y_best;
-    m->y0 = R.y0;
-    m->evaluated = R.evaluated;
-    for (int j = 0; j < kKMax; j++) m->end_op[j] = R.end_op[j];
-    m->total_ops = R.total_ops;
-    m->status = R.status;
-    m->pad = R.pad;
-    // release at system scope: the record is visible before the tag
-    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(&M->seq), "r"(seq) : "memory");
+// copy a result record to host-mapped pinned memory as four tagged 16-byte
+// chunks (MappedRec, common.cuh): no fence, the host validates the tags
+__device__ __forceinline__ void publish_mapped(const Result& R, MappedRec* M, uint32_t seq) {
+    uint32_t p[12];
+    rec_payload(R, p);
+#pragma unroll
+    for (int i = 0; i < 4; i++)
+        asm volatile("st.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(&M->w[4 * i]), "r"(p[3 * i]), "r"(p[3 * i + 1]),
+                     "r"(p[3 * i + 2]), "r"(rec_tag(seq, p[3 * i], p[3 * i + 1], p[3 * i + 2], (uint32_t)i))
+                     : "memory");
 }
 
 static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratch* S, unsigned long long key, float y) {

@@ -40,7 +40,7 @@ cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const f
 cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,
                               cudaStream_t st, int* grid_out);
 cudaError_t launch_mway(const Plan& P, const W234& W, const float* w1b1, int ways, Scratch* S, cudaStream_t st);
-cudaError_t launch_finalize_gather(Scratch* S, int nranks, Result* mapped, uint32_t seq, cudaStream_t st);
+cudaError_t launch_finalize_gather(Scratch* S, int nranks, MappedRec* mapped, uint32_t seq, cudaStream_t st);
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out);

@@ -622,7 +622,7 @@ __global__ void __launch_bounds__(kFused2Threads, kFused2BlocksPerSM) fused_fp32
 // a6 tail: after the NCCL all-gather of the per-rank Result records, every
 // rank reduces the same records to the same global decision.
 // ---------------------------------------------------------------------------
-__global__ void finalize_gather_kernel(Scratch* S, int nranks, Result* mapped, uint32_t seq) {
+__global__ void finalize_gather_kernel(Scratch* S, int nranks, MappedRec* mapped, uint32_t seq) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     int best = 0;
     unsigned long long ev = 0;
@@ -1011,7 +1011,7 @@ cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, S
     return cudaGetLastError();
 }
 
-cudaError_t launch_finalize_gather(Scratch* S, int nranks, Result* mapped, uint32_t seq, cudaStream_t st) {
+cudaError_t launch_finalize_gather(Scratch* S, int nranks, MappedRec* mapped, uint32_t seq, cudaStream_t st) {
     finalize_gather_kernel<<<1, 32, 0, st>>>(S, nranks, mapped, seq);
     return cudaGetLastError();
 }
