@@ -23,6 +23,7 @@
 
 #include "../../include/abacus.h"
 #include "common.cuh"
+#include "device_common.cuh"
 #include "internal.h"
 #include "tc_ptx.cuh"
 
@@ -746,6 +747,12 @@ int grow_batch(abacus_ctx* c, int32_t n) {
 }
 
 // a7 for one decision from its result record (shared by the single and batched searches)
+// a7 on the host for records published to host-mapped memory: end op per slot of t*
+void host_decode(const Plan& P, Result& R) {
+    for (int j = 0; j < kKMax; j++)
+        R.end_op[j] = (R.key && j < P.k) ? decode_slot_ope(P, R.key & ((1ull << 40) - 1), j) : 0;
+}
+
 abacus_decision_t assemble_decision(const Result& R, const int32_t* order, int32_t k, float H, uint64_t n_eval) {
     abacus_decision_t d{};
     d.critical = order[0];
@@ -1001,6 +1008,7 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
     Result R;
     rc = wait_result(c, P.seq, &R);
     if (rc) return rc;
+    host_decode(P, R);
     *out = assemble_decision(R, order, k, H, n_eval);
     return ABACUS_OK;
 }
@@ -1150,6 +1158,7 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     Result R;
     rc = wait_result(c, seq, &R);
     if (rc) return rc;
+    if (!nccl_comm) host_decode(P, R);
     abacus_decision_t d{};
     d.critical = 0;
     for (int j = 0; j < 4; j++) d.order[j] = j < grid->k ? j : -1;

@@ -8,7 +8,7 @@
 namespace abacus {
 
 // grid digit -> ope (0 = absent); SlotP carries the ABI digit definition
-__device__ __forceinline__ int32_t digit_to_ope(const SlotP& s, uint32_t d) {
+__host__ __device__ __forceinline__ int32_t digit_to_ope(const SlotP& s, uint32_t d) {
     if (s.absent) return d == 0 ? 0 : s.end_lo + (int32_t)d - 1;
     return s.end_lo + (int32_t)d;
 }
@@ -270,7 +270,7 @@ __device__ __forceinline__ void fold_packed2(const Plan& P, int sx, uint32_t x1,
 // decodes the winning index into end ops per slot and resets the ticket.
 // ---------------------------------------------------------------------------
 // q = floor(a / b) for a < 2^40 via an fp64 reciprocal (exact after one correction)
-__device__ __forceinline__ unsigned long long div_rcp(unsigned long long a, unsigned long long b, double rb) {
+__host__ __device__ __forceinline__ unsigned long long div_rcp(unsigned long long a, unsigned long long b, double rb) {
     unsigned long long q = (unsigned long long)((double)a * rb);
     const long long rem = (long long)(a - q * b);
     if (rem < 0) q--;
@@ -280,8 +280,9 @@ __device__ __forceinline__ unsigned long long div_rcp(unsigned long long a, unsi
 
 // End op of slot `j` of the candidate with index idx (GRID: digit j of the
 // mixed-radix index, computed directly so lanes can decode slots in parallel;
-// CHAIN: block structure).  0 = absent.
-__device__ __forceinline__ int32_t decode_slot_ope(const PlanHdr& P, unsigned long long idx, int j) {
+// CHAIN: block structure).  0 = absent.  Also run by the host for searches
+// whose record goes to host-mapped memory (the kernel then skips the decode).
+__host__ __device__ __forceinline__ int32_t decode_slot_ope(const PlanHdr& P, unsigned long long idx, int j) {
     if (P.mode == kModeGrid) {
         const SlotP& s = P.slot[j];
         const unsigned long long q = div_rcp(idx, s.tstride, s.rtstride);
@@ -377,8 +378,9 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
             if (k2 > bk) { bk = k2; by = y2; }
         }
         trace_stamp(P, 9);
-        // a7: lane j decodes slot j's end op of t*
-        const int32_t my_ope = (threadIdx.x < (unsigned)P.k && bk)
+        // a7: lane j decodes slot j's end op of t*; a record that goes to host-mapped
+        // memory is decoded by the host instead (off the kernel's critical path)
+        const int32_t my_ope = (!P.mapped && threadIdx.x < (unsigned)P.k && bk)
                                    ? decode_slot_ope(P, bk & ((1ull << 40) - 1), (int)threadIdx.x)
                                    : 0;
         int32_t ope[kKMax];
