@@ -513,6 +513,15 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform for the compiler
     const int g = warp >> 2, wq = warp & 3;
     trace_stamp(P, 0);
+    // the mbarriers and the TMEM allocation are set up while the weights load
+    if (tid == 0) {
+        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
+        mbar_fence_init();
+    }
+    if (warp == 0) {
+        tmem_alloc(tmem_slot, 512);
+        tmem_relinquish();
+    }
     {
         const int4* src = reinterpret_cast<const int4*>(TP.blob);
         int4* dst = reinterpret_cast<int4*>(smem);
@@ -521,11 +530,22 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         float* s_w1 = reinterpret_cast<float*>(smem + L.stage);
         for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
     }
+    fence_before();
     __syncthreads();
+    fence_after();
     trace_stamp(P, 1);
+    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
     build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
                                blockDim.x);
-    const uint32_t tbase = fused_prologue_tmem<FMT, NG>(bars, tmem_slot, warp, g, wq);
+    if (g == 0) {  // the constant chunk (1, 1, 0, ...) of the bias rows
+        uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
+        tmem_st8(tbase + 480 + ((uint32_t)(wq * 32) << 16), c8);
+        tmem_wait_st();
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // weights and tables -> tensor core
+    fence_before();
+    __syncthreads();
+    fence_after();
     trace_stamp(P, 2);
 
     const uint32_t r = (uint32_t)(tid & 127);
