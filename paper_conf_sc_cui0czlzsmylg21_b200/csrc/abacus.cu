@@ -180,7 +180,7 @@ int validate_grid(abacus_ctx* c, const abacus_grid_t* g, uint64_t* T_out) {
 }
 
 // ---- plans ------------------------------------------------------------------
-__host__ __device__ void fill_strides(Plan& P) {
+__host__ __device__ void fill_strides(PlanHdr& P) {
     uint64_t b = 1;
     for (int j = kKMax - 1; j >= 0; j--) {
         P.slot[j].tstride = b;
@@ -189,7 +189,7 @@ __host__ __device__ void fill_strides(Plan& P) {
     }
 }
 
-__host__ __device__ void fill_slots(Plan& P, const abacus_grid_t* g) {
+__host__ __device__ void fill_slots(PlanHdr& P, const abacus_grid_t* g) {
     for (int j = 0; j < kKMax; j++) {
         SlotP& s = P.slot[j];
         if (j < g->k) {
@@ -246,7 +246,7 @@ __host__ __device__ Plan plan_whole_grid(int32_t n_models, int32_t D, const abac
 // number of elements of segment box `s` with index < a.  Per SLOT j the box
 // digit set is: present -> [dlo_j, dlo_j + cnt_j), absent -> {0}; elements
 // are ordered lexicographically by slot (index order).
-__host__ __device__ uint64_t box_count_lt(const Plan& P, const SegP& s, const uint32_t* dlo, const uint32_t* scnt, uint64_t a) {
+__host__ __device__ uint64_t box_count_lt(const PlanHdr& P, const SegP& s, const uint32_t* dlo, const uint32_t* scnt, uint64_t a) {
     if (a >= P.T) return box_size(s);
     uint32_t dig[kKMax] = {0, 0, 0, 0};
     uint64_t rem = a;
@@ -293,7 +293,7 @@ __host__ __device__ void order_digits(SegP& s, int k, const uint32_t* scnt, cons
     s.fast_carry = s.cnt[kKMax - 1] >= (uint32_t)kTileM ? 1u : 0u;
 }
 
-__host__ __device__ void set_positions(const Plan& P, SegP& s) {
+__host__ __device__ void set_positions(const PlanHdr& P, SegP& s) {
     for (int j = 0; j < kKMax; j++) {
         s.pos[j] = -1;
         if (j >= P.k || !((s.mask >> j) & 1u)) continue;
@@ -305,9 +305,14 @@ __host__ __device__ void set_positions(const Plan& P, SegP& s) {
 }
 
 // GRID / sweep: one segment per presence pattern, restricted to [first, last)
-__host__ __device__ Plan plan_grid_segments(int32_t n_models, int32_t D, const abacus_grid_t* g, uint64_t T,
-                                            uint64_t first, uint64_t last, float H) {
-    Plan P{};
+// The segments go to `put(index, segment)`: the Plan's own table (host and
+// single launches) or, on the device planner of a batch, straight to the
+// decision's slots in global memory (no 3.7 KB Plan on the thread's stack).
+template <class Put>
+__host__ __device__ void plan_grid_segments_into(PlanHdr& P, Put&& put, int32_t n_models, int32_t D,
+                                                 const abacus_grid_t* g, uint64_t T, uint64_t first, uint64_t last,
+                                                 float H) {
+    P = PlanHdr{};
     P.k = g->k;
     P.n_models = n_models;
     P.D = D;
@@ -358,17 +363,26 @@ __host__ __device__ Plan plan_grid_segments(int32_t n_models, int32_t D, const a
         s.tile0 = tiles;
         tiles += (s.u_end - s.u_begin + kTileM - 1) / kTileM;
         n_eval += s.u_end - s.u_begin;
-        P.seg[P.n_seg++] = s;
+        put(P.n_seg++, s);
     }
     P.n_tiles = tiles;
     P.n_eval = n_eval;
+}
+
+__host__ __device__ Plan plan_grid_segments(int32_t n_models, int32_t D, const abacus_grid_t* g, uint64_t T,
+                                            uint64_t first, uint64_t last, float H) {
+    Plan P{};
+    plan_grid_segments_into(static_cast<PlanHdr&>(P), [&](int i, const SegP& sg) { P.seg[i] = sg; }, n_models, D,
+                            g, T, first, last, H);
     return P;
 }
 
 // CHAIN (decision mode): u = 0 critical only; block j: slots < j full, slot j
 // grows op by op, later slots absent
-__host__ __device__ Plan plan_chain(int32_t n_models, int32_t D, const abacus_grid_t* g, float H, uint64_t* n_out) {
-    Plan P{};
+template <class Put>
+__host__ __device__ void plan_chain_into(PlanHdr& P, Put&& put, int32_t n_models, int32_t D, const abacus_grid_t* g,
+                                         float H, uint64_t* n_out) {
+    P = PlanHdr{};
     P.k = g->k;
     P.n_models = n_models;
     P.D = D;
@@ -407,13 +421,19 @@ __host__ __device__ Plan plan_chain(int32_t n_models, int32_t D, const abacus_gr
         s.tile0 = tiles;
         tiles += (s.u_end + kTileM - 1) / kTileM;
         cum += s.u_end;
-        P.seg[P.n_seg++] = s;
+        put(P.n_seg++, s);
     }
     P.chain_cum[g->k] = cum;
     P.T = cum;
     P.n_tiles = tiles;
     P.n_eval = cum;
     *n_out = cum;
+}
+
+__host__ __device__ Plan plan_chain(int32_t n_models, int32_t D, const abacus_grid_t* g, float H, uint64_t* n_out) {
+    Plan P{};
+    plan_chain_into(static_cast<PlanHdr&>(P), [&](int i, const SegP& sg) { P.seg[i] = sg; }, n_models, D, g, H,
+                    n_out);
     return P;
 }
 
@@ -666,16 +686,25 @@ __global__ void batch_plan_kernel(const BatchIn* __restrict__ in, int32_t n, int
     if (i >= n) return;
     const BatchIn b = in[i];
     uint64_t n_eval = 0;
-    Plan P = b.chain ? plan_chain(n_models, D, &b.g, b.H, &n_eval) : plan_grid_segments(n_models, D, &b.g, b.T, 0, b.T, b.H);
-    if (!b.chain) n_eval = P.n_eval;
+    // segments go straight to this decision's slots in global memory
+    SegP* my = segs + (size_t)kMaxSegBatch * i;
+    auto put = [&](int sg, const SegP& s) {
+        if (sg < kMaxSegBatch) my[sg] = s;
+    };
+    PlanHdr P;
+    if (b.chain) {
+        plan_chain_into(P, put, n_models, D, &b.g, b.H, &n_eval);
+    } else {
+        plan_grid_segments_into(P, put, n_models, D, &b.g, b.T, 0, b.T, b.H);
+        n_eval = P.n_eval;
+    }
     BatchDec& bd = decs[i];
-    bd.h = static_cast<const PlanHdr&>(P);
+    bd.h = P;
     bd.h.want_y0 = 1;
     bd.h.n_eval = n_eval;
     bd.h.mapped = nullptr;
     bd.h.trace = nullptr;
     bd.seg0 = (uint32_t)(kMaxSegBatch * i);
-    for (int sg = 0; sg < P.n_seg && sg < kMaxSegBatch; sg++) segs[(size_t)kMaxSegBatch * i + sg] = P.seg[sg];
     pairs[i] = (P.n_tiles + 1) / 2;  // tiles padded to pairs (lock-step slots never straddle decisions)
 }
 
