@@ -305,6 +305,12 @@ __host__ __device__ void set_positions(const PlanHdr& P, SegP& s) {
 }
 
 // GRID / sweep: one segment per presence pattern, restricted to [first, last)
+// segment sink of a full Plan (host and single launches)
+struct PlanSink {
+    Plan* P;
+    __host__ __device__ void operator()(int i, const SegP& s) const { P->seg[i] = s; }
+};
+
 // The segments go to `put(index, segment)`: the Plan's own table (host and
 // single launches) or, on the device planner of a batch, straight to the
 // decision's slots in global memory (no 3.7 KB Plan on the thread's stack).
@@ -372,8 +378,7 @@ __host__ __device__ void plan_grid_segments_into(PlanHdr& P, Put&& put, int32_t 
 __host__ __device__ Plan plan_grid_segments(int32_t n_models, int32_t D, const abacus_grid_t* g, uint64_t T,
                                             uint64_t first, uint64_t last, float H) {
     Plan P{};
-    plan_grid_segments_into(static_cast<PlanHdr&>(P), [&](int i, const SegP& sg) { P.seg[i] = sg; }, n_models, D,
-                            g, T, first, last, H);
+    plan_grid_segments_into(static_cast<PlanHdr&>(P), PlanSink{&P}, n_models, D, g, T, first, last, H);
     return P;
 }
 
@@ -432,8 +437,7 @@ __host__ __device__ void plan_chain_into(PlanHdr& P, Put&& put, int32_t n_models
 
 __host__ __device__ Plan plan_chain(int32_t n_models, int32_t D, const abacus_grid_t* g, float H, uint64_t* n_out) {
     Plan P{};
-    plan_chain_into(static_cast<PlanHdr&>(P), [&](int i, const SegP& sg) { P.seg[i] = sg; }, n_models, D, g, H,
-                    n_out);
+    plan_chain_into(static_cast<PlanHdr&>(P), PlanSink{&P}, n_models, D, g, H, n_out);
     return P;
 }
 
@@ -605,7 +609,7 @@ int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
 
 // a1 (Eq. 2 + Eq. 3, sort) and the decision's slots in headroom order
 int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
-                   int32_t* order, float* H_out, abacus_grid_t* g_out) {
+                   int32_t* order, float* H_out, abacus_grid_t* g_out, uint64_t* T_out = nullptr) {
     if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
     if (!q) return fail(c, ABACUS_E_INVALID, "NULL argument");
     if (k < 1 || k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
@@ -628,10 +632,16 @@ int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now
         h[i] = (a.qos_ms - (now_ms - a.t_start_ms)) - inflight_pred_ms;
         order[i] = i;
     }
-    std::stable_sort(order, order + k, [&](int a, int b) {
-        if (h[a] != h[b]) return h[a] < h[b];
-        return q[a].model_id < q[b].model_id;
-    });
+    // stable insertion sort of <= 4 entries (std::stable_sort would allocate a buffer per call)
+    for (int i = 1; i < k; i++) {
+        const int v = order[i];
+        int j = i - 1;
+        while (j >= 0 && (h[order[j]] > h[v] || (h[order[j]] == h[v] && q[order[j]].model_id > q[v].model_id))) {
+            order[j + 1] = order[j];
+            j--;
+        }
+        order[j + 1] = v;
+    }
     *H_out = (float)h[order[0]];
     // a2: slots in headroom order; the critical query is fully included
     abacus_grid_t& g = *g_out;
@@ -643,13 +653,14 @@ int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now
         g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? L : a.next_op, L, j == 0 ? 0 : 1};
     }
     uint64_t T = 0;
-    return validate_grid(c, &g, &T);
+    const int rc = validate_grid(c, &g, &T);
+    if (T_out) *T_out = T;
+    return rc;
 }
 
 unsigned long long* trace_ptr();
 
-int launch_fused(abacus_ctx* c, const Plan& Pin) {
-    Plan P = Pin;
+int launch_fused(abacus_ctx* c, Plan& P) {
     P.trace = trace_ptr();
     int grid = 0;
     cudaError_t e;
@@ -1014,18 +1025,18 @@ int abacus_search(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_
     int32_t order[ABACUS_K_MAX];
     float H = 0.0f;
     abacus_grid_t g{};
-    int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g);
-    if (rc) return rc;
     uint64_t T = 0;
-    rc = validate_grid(c, &g, &T);
+    int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g, &T);
     if (rc) return rc;
     const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
+    // the plan is built in place (the segment table is written once, not returned by value)
     Plan P;
+    const PlanSink put{&P};
     uint64_t n_eval = 0;
     if (chain) {
-        P = plan_chain(c->n_models, c->D, &g, H, &n_eval);
+        plan_chain_into(static_cast<PlanHdr&>(P), put, c->n_models, c->D, &g, H, &n_eval);
     } else {
-        P = plan_grid_segments(c->n_models, c->D, &g, T, 0, T, H);
+        plan_grid_segments_into(static_cast<PlanHdr&>(P), put, c->n_models, c->D, &g, T, 0, T, H);
         n_eval = P.n_eval;
     }
     P.want_y0 = 1;
@@ -1071,12 +1082,11 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     for (int32_t i = 0; i < n; i++) {
         BatchIn& b = c->h_in[i];
         rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], &c->b_order[4 * (size_t)i],
-                            &c->b_H[i], &b.g);
+                            &c->b_H[i], &b.g, &b.T);
         if (rc) {
             c->err = "decision " + std::to_string(i) + ": " + c->err;
             return rc;
         }
-        validate_grid(c, &b.g, &b.T);
         b.H = c->b_H[i];
         b.chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && b.T > grid_budget);
         // bounds the device plan cannot exceed: the widest segment digit (selects the
