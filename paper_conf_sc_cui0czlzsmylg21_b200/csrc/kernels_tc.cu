@@ -448,6 +448,18 @@ struct TcPipe {
             issue_next<LAYER, TWO>();
         }
     }
+    // the same with fixed issuer roles: stage p issued by warp wq == p of the group
+    template <bool TWO>
+    __device__ __forceinline__ void run_layers_fixed(int wq, uint32_t& yx, uint32_t& yy) {
+        stage_as<0, TWO>(wq == 0);
+        stage_as<1, TWO>(wq == 1);
+        stage_as<2, TWO>(wq == 2);
+        wait();
+        if (TWO) tmem_ld1x2(X.d + lane_off, Y.d + lane_off, yx, yy);
+        else tmem_ld1(X.d + lane_off, yx);
+        yx = add_b4(yx);
+        if (TWO) yy = add_b4(yy);
+    }
     // the three hidden stages, then wait for the output MMA and read y (column 0 of D)
     template <bool TWO, bool CONST = false>
     __device__ __forceinline__ void run_layers(uint32_t& yx, uint32_t& yy) {
@@ -911,7 +923,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
                 y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s;
                 store_a1_packed(pp.Y.a1 + pp.lane_off, W.a1, W.a2);
                 tmem_wait_st();
-                if (pp.handoff(pp.me[3])) {
+                if (pp.handoff(wq == 3)) {
                     issue_l1(pp.X, sX);
                     issue_l1(pp.Y, sY);
                     pp.commit();
@@ -921,10 +933,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             enter_pair(pb, true);
             for (uint64_t p = pb; p < pe; p++) {
                 uint32_t ybx, yby;
-                pp.template run_layers<true>(ybx, yby);
+                pp.template run_layers_fixed<true>(wq, ybx, yby);
                 if (ltX == 0 && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
-                fold_packed(P, sX, x1, x2, xs, __uint_as_float(ybx), best, best_y, bsn);
-                fold_packed(P, sY, y1, y2, ys, __uint_as_float(yby), best, best_y, bsn);
+                fold_packed2(P, sX, x1, x2, xs, __uint_as_float(ybx), sY, y1, y2, ys, __uint_as_float(yby), best,
+                             best_y, bsn);
                 if (p + 1 == dec_pair_end) {  // leaving decision d
                     flush();
                     bsn = 1u;
