@@ -30,11 +30,17 @@
 using namespace abacus;
 
 // one decision of a batch after a1 (host): its grid, threshold, size and space
-struct BatchIn {
-    abacus_grid_t g;
+// one decision of a batch as the caller gave it (copied to pinned memory, then to the device)
+struct BatchRaw {
+    abacus_query_t q[ABACUS_K_MAX];
+    double now, infl;
+    int32_t k, pad;
+};
+// a1 of one decision of a batch, computed on the device: headroom order, H, error
+struct BatchA1 {
+    int32_t order[ABACUS_K_MAX];
     float H;
-    uint32_t chain;
-    uint64_t T;
+    int32_t err;  // A1 code | query i << 8 | query j << 16 (0 = valid)
 };
 
 struct abacus_ctx {
@@ -68,10 +74,11 @@ struct abacus_ctx {
     BatchAcc* d_acc = nullptr;
     float* d_y0 = nullptr;
     Result* d_out = nullptr;
-    std::vector<int32_t> b_order;  // [4 n] headroom order per decision
-    std::vector<float> b_H;
-    BatchIn* h_in = nullptr;       // pinned: a1 results (grid, H, T, space) per decision
-    BatchIn* d_in = nullptr;
+    BatchRaw* h_raw = nullptr;     // pinned: the decisions as given
+    BatchRaw* d_raw = nullptr;
+    BatchA1* h_a1 = nullptr;       // pinned: a1 per decision (order, H, error), from the device
+    BatchA1* d_a1 = nullptr;
+    int32_t* d_L = nullptr;        // device copy of the registry's op counts
     uint64_t* d_pairs = nullptr;   // [n] tile pairs per decision, then [n] = total
     // NEXT-3 training state (abacus_train_begin)
     bool training = false;
@@ -607,28 +614,30 @@ int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
     return ABACUS_OK;
 }
 
-// a1 (Eq. 2 + Eq. 3, sort) and the decision's slots in headroom order
-int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
-                   int32_t* order, float* H_out, abacus_grid_t* g_out, uint64_t* T_out = nullptr) {
-    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
-    if (!q) return fail(c, ABACUS_E_INVALID, "NULL argument");
-    if (k < 1 || k > ABACUS_K_MAX) return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
-    if (!std::isfinite(now_ms) || !std::isfinite(inflight_pred_ms))
-        return fail(c, ABACUS_E_INVALID, "non-finite time");
+// a1 (Eq. 2 + Eq. 3, sort) and the decision's slots in headroom order, shared by
+// the host (single rounds) and the device planner of batches. Returns an A1_*
+// code (0 = valid) and the offending query indices in *qi, *qj.
+enum : int32_t { A1_OK = 0, A1_K, A1_TIME, A1_MODEL, A1_DUP, A1_NEXTOP, A1_SIZES, A1_QTIME, A1_T, A1_SUMN };
+__host__ __device__ int32_t a1_slots(const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                                     const int32_t* L, int32_t n_models, int32_t* order, float* H_out,
+                                     abacus_grid_t* g_out, uint64_t* T_out, int32_t* qi, int32_t* qj) {
+    *qi = *qj = 0;
+    if (k < 1 || k > ABACUS_K_MAX) return A1_K;
+    if (!isfinite(now_ms) || !isfinite(inflight_pred_ms)) return A1_TIME;
     // a1: Eq. 2 + Eq. 3 headroom per query; ascending order, ties by model id
     double h[ABACUS_K_MAX];
     for (int i = 0; i < k; i++) {
         const abacus_query_t& a = q[i];
-        if (a.model_id < 1 || a.model_id > c->n_models)
-            return fail(c, ABACUS_E_INVALID, "query %d: model_id %d", i, a.model_id);
+        *qi = i;
+        if (a.model_id < 1 || a.model_id > n_models) return A1_MODEL;
         for (int j = 0; j < i; j++)
-            if (q[j].model_id == a.model_id) return fail(c, ABACUS_E_DUP_MODEL, "queries %d, %d share a model", j, i);
-        const int32_t L = c->L[a.model_id - 1];
-        if (a.next_op < 1 || a.next_op > L) return fail(c, ABACUS_E_INVALID, "query %d: next_op %d", i, a.next_op);
-        if (a.batch < 1 || a.batch > 32767 || a.seqlen < 0 || a.seqlen > 32767)
-            return fail(c, ABACUS_E_INVALID, "query %d: batch/seqlen", i);
-        if (!std::isfinite(a.qos_ms) || !std::isfinite(a.t_start_ms))
-            return fail(c, ABACUS_E_INVALID, "query %d: non-finite time", i);
+            if (q[j].model_id == a.model_id) {
+                *qj = j;
+                return A1_DUP;
+            }
+        if (a.next_op < 1 || a.next_op > L[a.model_id - 1]) return A1_NEXTOP;
+        if (a.batch < 1 || a.batch > 32767 || a.seqlen < 0 || a.seqlen > 32767) return A1_SIZES;
+        if (!isfinite(a.qos_ms) || !isfinite(a.t_start_ms)) return A1_QTIME;
         h[i] = (a.qos_ms - (now_ms - a.t_start_ms)) - inflight_pred_ms;
         order[i] = i;
     }
@@ -647,15 +656,48 @@ int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now
     abacus_grid_t& g = *g_out;
     g = abacus_grid_t{};
     g.k = k;
+    uint64_t T = 1;
+    int64_t max_sum_n = 0;
     for (int j = 0; j < k; j++) {
         const abacus_query_t& a = q[order[j]];
-        const int32_t L = c->L[a.model_id - 1];
-        g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? L : a.next_op, L, j == 0 ? 0 : 1};
+        const int32_t Lm = L[a.model_id - 1];
+        g.slot[j] = abacus_slot_t{a.model_id, a.next_op, a.batch, a.seqlen, j == 0 ? Lm : a.next_op, Lm, j == 0 ? 0 : 1};
+        T *= (uint64_t)g.slot[j].allow_absent + (uint64_t)(g.slot[j].end_hi - g.slot[j].end_lo + 1);
+        if (T >= (1ull << 40)) return A1_T;
+        max_sum_n += Lm - a.next_op + 1;
     }
+    if (max_sum_n + 1 >= (1ll << 24)) return A1_SUMN;
+    *T_out = T;
+    return A1_OK;
+}
+
+// host: the same with the library's error text
+int a1_fail(abacus_ctx* c, int32_t code, int32_t qi, int32_t qj, const abacus_query_t* q, int32_t k) {
+    switch (code) {
+        case A1_K: return fail(c, ABACUS_E_INVALID, "k=%d outside [1,4]", k);
+        case A1_TIME: return fail(c, ABACUS_E_INVALID, "non-finite time");
+        case A1_MODEL: return fail(c, ABACUS_E_INVALID, "query %d: model_id %d", qi, q[qi].model_id);
+        case A1_DUP: return fail(c, ABACUS_E_DUP_MODEL, "queries %d, %d share a model", qj, qi);
+        case A1_NEXTOP: return fail(c, ABACUS_E_INVALID, "query %d: next_op %d", qi, q[qi].next_op);
+        case A1_SIZES: return fail(c, ABACUS_E_INVALID, "query %d: batch/seqlen", qi);
+        case A1_QTIME: return fail(c, ABACUS_E_INVALID, "query %d: non-finite time", qi);
+        case A1_T: return fail(c, ABACUS_E_INVALID, "grid size >= 2^40");
+        case A1_SUMN: return fail(c, ABACUS_E_INVALID, "sum_n + 1 >= 2^24");
+        default: return ABACUS_OK;
+    }
+}
+
+int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                   int32_t* order, float* H_out, abacus_grid_t* g_out, uint64_t* T_out = nullptr) {
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (!q) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    int32_t qi = 0, qj = 0;
     uint64_t T = 0;
-    const int rc = validate_grid(c, &g, &T);
+    const int32_t code = a1_slots(q, k, now_ms, inflight_pred_ms, c->L.data(), c->n_models, order, H_out, g_out, &T,
+                                  &qi, &qj);
+    if (code) return a1_fail(c, code, qi, qj, q, k);
     if (T_out) *T_out = T;
-    return rc;
+    return ABACUS_OK;
 }
 
 unsigned long long* trace_ptr();
@@ -691,22 +733,42 @@ unsigned long long* trace_ptr() { return g_trace_ptr; }
 // One thread per decision runs the same planner as the single-round path
 // (plan_grid_segments / plan_chain, __host__ __device__) and writes the
 // decision's header and segments (fixed slots of kMaxSegBatch) in place.
-__global__ void batch_plan_kernel(const BatchIn* __restrict__ in, int32_t n, int32_t n_models, int32_t D,
-                                  BatchDec* __restrict__ decs, SegP* __restrict__ segs, uint64_t* __restrict__ pairs) {
+__global__ void batch_plan_kernel(const BatchRaw* __restrict__ raw, int32_t n, int32_t n_models, int32_t D,
+                                  const int32_t* __restrict__ L, int32_t space, uint64_t grid_budget,
+                                  BatchDec* __restrict__ decs, SegP* __restrict__ segs, uint64_t* __restrict__ pairs,
+                                  BatchA1* __restrict__ a1) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
-    const BatchIn b = in[i];
+    const BatchRaw& rw = raw[i];
+    // a1 (the host's function): headroom order, H, slots, validation
+    BatchA1 r{};
+    abacus_grid_t g;
+    uint64_t T = 0;
+    int32_t qi = 0, qj = 0;
+    const int32_t code = a1_slots(rw.q, rw.k, rw.now, rw.infl, L, n_models, r.order, &r.H, &g, &T, &qi, &qj);
+    r.err = code ? (code | (qi << 8) | (qj << 16)) : 0;
+    a1[i] = r;
+    if (code) {
+        // an invalid decision gets a one-candidate placeholder plan (model 1 run to
+        // its end) so the batch's tile walk stays well formed; the call reports the
+        // error and writes no output
+        g = abacus_grid_t{};
+        g.k = 1;
+        g.slot[0] = abacus_slot_t{1, 1, 1, 0, L[0], L[0], 0};
+        T = 1;
+    }
+    const bool chain = !code && (space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget));
     uint64_t n_eval = 0;
     // segments go straight to this decision's slots in global memory
     SegP* my = segs + (size_t)kMaxSegBatch * i;
-    auto put = [&](int sg, const SegP& s) {
-        if (sg < kMaxSegBatch) my[sg] = s;
+    auto put = [&](int sg, const SegP& sp) {
+        if (sg < kMaxSegBatch) my[sg] = sp;
     };
     PlanHdr P;
-    if (b.chain) {
-        plan_chain_into(P, put, n_models, D, &b.g, b.H, &n_eval);
+    if (chain) {
+        plan_chain_into(P, put, n_models, D, &g, r.H, &n_eval);
     } else {
-        plan_grid_segments_into(P, put, n_models, D, &b.g, b.T, 0, b.T, b.H);
+        plan_grid_segments_into(P, put, n_models, D, &g, T, 0, T, r.H);
         n_eval = P.n_eval;
     }
     BatchDec& bd = decs[i];
@@ -756,11 +818,15 @@ int grow_batch(abacus_ctx* c, int32_t n) {
     cudaFree(c->d_acc);
     cudaFree(c->d_y0);
     cudaFree(c->d_out);
-    if (c->h_in) cudaFreeHost(c->h_in);
-    cudaFree(c->d_in);
+    if (c->h_raw) cudaFreeHost(c->h_raw);
+    cudaFree(c->d_raw);
+    if (c->h_a1) cudaFreeHost(c->h_a1);
+    cudaFree(c->d_a1);
     cudaFree(c->d_pairs);
-    c->h_in = nullptr;
-    c->d_in = nullptr;
+    c->h_raw = nullptr;
+    c->d_raw = nullptr;
+    c->h_a1 = nullptr;
+    c->d_a1 = nullptr;
     c->d_pairs = nullptr;
     c->h_out = nullptr;
     c->d_decs = nullptr;
@@ -776,11 +842,11 @@ int grow_batch(abacus_ctx* c, int32_t n) {
     CUDA_TRY(c, cudaMalloc(&c->d_acc, nd * sizeof(BatchAcc)));
     CUDA_TRY(c, cudaMalloc(&c->d_y0, nd * sizeof(float)));
     CUDA_TRY(c, cudaMalloc(&c->d_out, nd * sizeof(Result)));
-    CUDA_TRY(c, cudaHostAlloc(&c->h_in, nd * sizeof(BatchIn), cudaHostAllocDefault));
-    CUDA_TRY(c, cudaMalloc(&c->d_in, nd * sizeof(BatchIn)));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_raw, nd * sizeof(BatchRaw), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaMalloc(&c->d_raw, nd * sizeof(BatchRaw)));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_a1, nd * sizeof(BatchA1), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaMalloc(&c->d_a1, nd * sizeof(BatchA1)));
     CUDA_TRY(c, cudaMalloc(&c->d_pairs, (nd + 1) * sizeof(uint64_t)));
-    c->b_order.resize(4 * nd);
-    c->b_H.resize(nd);
 
     c->batch_cap = cap;
     return ABACUS_OK;
@@ -845,7 +911,10 @@ int abacus_create(int device, int32_t n_models, const int32_t* ops_per_model, in
               cudaEventCreate(&c->ev0) == cudaSuccess && cudaEventCreate(&c->ev1) == cudaSuccess;
     if (ok) {
         const float nan = NAN;
-        ok = cudaMemcpy(&c->S->y0, &nan, sizeof(float), cudaMemcpyHostToDevice) == cudaSuccess;
+        ok = cudaMemcpy(&c->S->y0, &nan, sizeof(float), cudaMemcpyHostToDevice) == cudaSuccess &&
+             cudaMalloc(&c->d_L, sizeof(int32_t) * (size_t)n_models) == cudaSuccess &&
+             cudaMemcpy(c->d_L, ops_per_model, sizeof(int32_t) * (size_t)n_models, cudaMemcpyHostToDevice) ==
+                 cudaSuccess;
     }
     c->stream = c->own_stream;
     if (ok) memset(c->host_result, 0, sizeof(MappedRec));
@@ -873,8 +942,11 @@ void abacus_destroy(abacus_ctx* c) {
     cudaFree(c->d_acc);
     cudaFree(c->d_y0);
     cudaFree(c->d_out);
-    if (c->h_in) cudaFreeHost(c->h_in);
-    cudaFree(c->d_in);
+    if (c->h_raw) cudaFreeHost(c->h_raw);
+    cudaFree(c->d_raw);
+    if (c->h_a1) cudaFreeHost(c->h_a1);
+    cudaFree(c->d_a1);
+    cudaFree(c->d_L);
     cudaFree(c->d_pairs);
     cudaFree(c->t_p);
     cudaFree(c->t_m);
@@ -1075,38 +1147,32 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     CUDA_TRY(c, cudaSetDevice(c->device));
     int rc = grow_batch(c, n);
     if (rc) return rc;
-    // a1 and validation on the host, in order (the first failing decision is
-    // reported and nothing is launched); everything after runs on the device
-    uint64_t pairs_ub = 0;
+    // The host copies the decisions to pinned memory and bounds the widest digit
+    // (it selects the tensor kernels' split layer-1 layout); a1, validation and
+    // planning run on the device, one thread per decision (batch_plan_kernel).
+    // A failing decision is reported by its index (the first one) after the
+    // launch; no output is written then.
     uint32_t maxcnt = 0;
     for (int32_t i = 0; i < n; i++) {
-        BatchIn& b = c->h_in[i];
-        rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], &c->b_order[4 * (size_t)i],
-                            &c->b_H[i], &b.g, &b.T);
-        if (rc) {
-            c->err = "decision " + std::to_string(i) + ": " + c->err;
-            return rc;
+        BatchRaw& rw = c->h_raw[i];
+        const int32_t ki = k[i];
+        const int32_t kc = ki < 0 ? 0 : (ki > ABACUS_K_MAX ? ABACUS_K_MAX : ki);
+        memcpy(rw.q, q + 4 * (size_t)i, sizeof(abacus_query_t) * ABACUS_K_MAX);
+        rw.now = now_ms[i];
+        rw.infl = inflight_pred_ms[i];
+        rw.k = ki;
+        for (int j = 0; j < kc; j++) {  // a slot's digit counts at most L - next_op + 1 end ops
+            const abacus_query_t& a = rw.q[j];
+            if (a.model_id >= 1 && a.model_id <= c->n_models && a.next_op >= 1) {
+                const int32_t w = c->L[a.model_id - 1] - a.next_op + 1;
+                if (w > 0 && (uint32_t)w > maxcnt) maxcnt = (uint32_t)w;
+            }
         }
-        b.H = c->b_H[i];
-        b.chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && b.T > grid_budget);
-        // bounds the device plan cannot exceed: the widest segment digit (selects the
-        // split layer-1 layout) and the tile pairs (<= one partial tile per segment)
-        uint64_t n_cand = b.T;
-        if (b.chain) {
-            n_cand = 1;
-            for (int j = 1; j < b.g.k; j++) n_cand += (uint64_t)(b.g.slot[j].end_hi - b.g.slot[j].start_op + 1);
-        }
-        for (int j = b.chain ? 1 : 0; j < b.g.k; j++) {  // CHAIN: the critical slot's digit is fixed
-            const abacus_slot_t& sl = b.g.slot[j];
-            const uint32_t w = (uint32_t)(sl.end_hi - (b.chain ? sl.start_op : sl.end_lo) + 1);
-            maxcnt = w > maxcnt ? w : maxcnt;
-        }
-        pairs_ub += (n_cand / kTileM + kMaxSegBatch + 1) / 2 + 1;
     }
     cudaStream_t st = c->stream;
-    CUDA_TRY(c, cudaMemcpyAsync(c->d_in, c->h_in, (size_t)n * sizeof(BatchIn), cudaMemcpyHostToDevice, st));
-    batch_plan_kernel<<<(n + 127) / 128, 128, 0, st>>>(c->d_in, n, c->n_models, c->D, c->d_decs, c->d_segs,
-                                                       c->d_pairs);
+    CUDA_TRY(c, cudaMemcpyAsync(c->d_raw, c->h_raw, (size_t)n * sizeof(BatchRaw), cudaMemcpyHostToDevice, st));
+    batch_plan_kernel<<<(n + 127) / 128, 128, 0, st>>>(c->d_raw, n, c->n_models, c->D, c->d_L, space, grid_budget,
+                                                       c->d_decs, c->d_segs, c->d_pairs, c->d_a1);
     batch_scan_kernel<<<1, kScanThreads, 0, st>>>(c->d_decs, c->d_pairs, n);
     CUDA_TRY(c, cudaGetLastError());
     c->launches += 2;
@@ -1114,15 +1180,26 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     CUDA_TRY(c, cudaMemsetAsync(c->d_y0, 0xFF, (size_t)n * sizeof(float), st));  // NaN
     if (c->timed) cudaEventRecord(c->ev0, st);
     const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
+    // the exact pair count is only known on the device: the grid covers every SM
+    const uint64_t pairs_ub = ~0ull >> 8;
     cudaError_t e = launch_batch_tc(c->d_decs, c->d_segs, n, c->d_pairs + n, pairs_ub, maxcnt, c->D, c->tw[fmt],
                                     c->d_w1b1, c->d_acc, c->d_y0, c->d_out, c->nsm, st);
     if (c->timed) cudaEventRecord(c->ev1, st);
     if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "batched search launch: %s", cudaGetErrorString(e));
     c->launches += 2;
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_a1, c->d_a1, (size_t)n * sizeof(BatchA1), cudaMemcpyDeviceToHost, st));
     CUDA_TRY(c, cudaMemcpyAsync(c->h_out, c->d_out, (size_t)n * sizeof(Result), cudaMemcpyDeviceToHost, st));
     CUDA_TRY(c, cudaStreamSynchronize(st));
+    for (int32_t i = 0; i < n; i++) {
+        const int32_t er = c->h_a1[i].err;
+        if (er) {
+            a1_fail(c, er & 0xFF, (er >> 8) & 0xFF, (er >> 16) & 0xFF, q + 4 * (size_t)i, k[i]);
+            c->err = "decision " + std::to_string(i) + ": " + c->err;
+            return (er & 0xFF) == A1_DUP ? ABACUS_E_DUP_MODEL : ABACUS_E_INVALID;
+        }
+    }
     for (int32_t i = 0; i < n; i++)
-        out[i] = assemble_decision(c->h_out[i], &c->b_order[4 * (size_t)i], k[i], c->b_H[i], c->h_out[i].evaluated);
+        out[i] = assemble_decision(c->h_out[i], c->h_a1[i].order, k[i], c->h_a1[i].H, c->h_out[i].evaluated);
     return ABACUS_OK;
 }
 
