@@ -584,29 +584,14 @@ uint32_t next_seq(abacus_ctx*) {
     return s;
 }
 
-// all four chunks of the record carry the tag of `seq` -> payload into *R
-bool read_record(const MappedRec* M, uint32_t seq, Result* R) {
-    const volatile uint32_t* w = M->w;
-    uint32_t p[12];
-    for (uint32_t i = 0; i < 4; i++) {
-        const uint32_t a = w[4 * i], b = w[4 * i + 1], cc = w[4 * i + 2], t = w[4 * i + 3];
-        if (t != rec_tag(seq, a, b, cc, i)) return false;
-        p[3 * i] = a;
-        p[3 * i + 1] = b;
-        p[3 * i + 2] = cc;
-    }
-    rec_unpayload(p, *R);
-    return true;
-}
-
 int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
     for (uint64_t spin = 1;; spin++) {
-        if (read_record(c->host_result, seq, R)) break;
+        if (rec_read(c->host_result, seq, R)) break;
         if ((spin & 1023) == 0) {
             const cudaError_t e = cudaStreamQuery(c->stream);
             if (e != cudaSuccess && e != cudaErrorNotReady)
                 return fail(c, ABACUS_E_CUDA, "search kernel failed: %s", cudaGetErrorString(e));
-            if (e == cudaSuccess && !read_record(c->host_result, seq, R))
+            if (e == cudaSuccess && !rec_read(c->host_result, seq, R))
                 return fail(c, ABACUS_E_CUDA, "search finished without publishing its result");
         }
     }

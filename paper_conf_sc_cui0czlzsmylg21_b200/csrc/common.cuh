@@ -109,6 +109,22 @@ __host__ __device__ inline void rec_unpayload(const uint32_t (&p)[12], Result& R
     R.seq = 0;
 }
 
+// host: all four chunks of a record carry the tag of `seq` -> payload into *R
+// (volatile reads: the device may be writing the record concurrently)
+inline bool rec_read(const MappedRec* M, uint32_t seq, Result* R) {
+    const volatile uint32_t* w = M->w;
+    uint32_t p[12];
+    for (uint32_t i = 0; i < 4; i++) {
+        const uint32_t a = w[4 * i], b = w[4 * i + 1], c = w[4 * i + 2], t = w[4 * i + 3];
+        if (t != rec_tag(seq, a, b, c, i)) return false;
+        p[3 * i] = a;
+        p[3 * i + 1] = b;
+        p[3 * i + 2] = c;
+    }
+    rec_unpayload(p, *R);
+    return true;
+}
+
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
 
 // header of a plan: everything but the segment table (decode of t*, a7)
