@@ -144,3 +144,54 @@ def test_batch_errors_name_the_decision():
         assert len(ab.abacus_search_batch(c.h, decs)) == 5
     finally:
         c.close()
+
+
+def _bad_variants(qs):
+    """One invalid version of a round per validation rule of a1 (the device
+    planner of a batch checks what abacus_search checks on the host)."""
+    m0 = qs[0]
+    L0 = synth.L(m0.model_id)
+    rep = lambda q, **kw: synth.Query(**{**q.__dict__, **kw})  # noqa: E731
+    return [
+        ("model_id", [rep(m0, model_id=99)] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("next_op", [rep(m0, next_op=L0 + 1)] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("next_op", [rep(m0, next_op=0)] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("batch", [rep(m0, batch=0)] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("seqlen", [rep(m0, seqlen=-1)] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("qos", [rep(m0, qos_ms=float("nan"))] + list(qs[1:]), ab.ABACUS_E_INVALID),
+        ("dup", list(qs) + [rep(qs[-1], next_op=1)], ab.ABACUS_E_DUP_MODEL),
+    ]
+
+
+@pytest.mark.parametrize("prec", TC)
+def test_batch_validation_matches_single_rounds(prec):
+    """Every validation rule, at several positions in a batch: the batch fails
+    with the single-round error code, names the first failing decision, and
+    leaves the context usable; non-finite now / in-flight times too."""
+    c = Ctx(params=synth.weights(1), precision=prec)
+    try:
+        decs = synth.cfg2_decisions(12)
+        for name, bad_qs, code in _bad_variants(decs[0][0]):
+            with pytest.raises(ab.AbacusError) as single:
+                ab.abacus_search(c.h, bad_qs, decs[0][1], decs[0][2])
+            assert single.value.code == code, name
+            for pos in (0, 5, 11):
+                batch = list(decs)
+                batch[pos] = (bad_qs, batch[pos][1], batch[pos][2])
+                if pos != 11:  # a second bad round later in the batch: the first one is named
+                    batch[11] = (bad_qs, batch[11][1], batch[11][2])
+                with pytest.raises(ab.AbacusError) as e:
+                    ab.abacus_search_batch(c.h, batch)
+                assert e.value.code == code, (name, pos)
+                assert ("decision %d:" % pos) in str(e.value), (name, pos, str(e.value))
+        for now, infl in ((float("inf"), 0.0), (0.0, float("nan"))):
+            batch = list(decs)
+            batch[3] = (batch[3][0], now, infl)
+            with pytest.raises(ab.AbacusError) as e:
+                ab.abacus_search_batch(c.h, batch)
+            assert e.value.code == ab.ABACUS_E_INVALID and "decision 3:" in str(e.value)
+        got = ab.abacus_search_batch(c.h, decs)
+        for (qs, now, infl), d in zip(decs, got):
+            _same(d, ab.abacus_search(c.h, qs, now, infl))
+    finally:
+        c.close()
