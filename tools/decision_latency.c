@@ -23,6 +23,10 @@ static int cmpd(const void* a, const void* b) {
     double x = *(const double*)a, y = *(const double*)b;
     return x < y ? -1 : x > y;
 }
+static int cmpu(const void* a, const void* b) {
+    const uint64_t x = *(const uint64_t*)a, y = *(const uint64_t*)b;
+    return x < y ? -1 : x > y;
+}
 #define RD(p, n, f) do { if (fread(p, 1, n, f) != (size_t)(n)) { fprintf(stderr, "short read\n"); return 2; } } while (0)
 
 int main(int argc, char** argv) {
@@ -105,11 +109,15 @@ int main(int argc, char** argv) {
     qsort(lat + warm, n, sizeof(double), cmpd);
     uint64_t evmax = 0, evsum = 0;
     for (int i = warm; i < ndec; i++) { evmax = ev[i] > evmax ? ev[i] : evmax; evsum += ev[i]; }
+    /* candidates evaluated per decision (grid / chain size): percentiles */
+    qsort(ev + warm, n, sizeof(uint64_t), cmpu);
     printf("{\"decisions\": %d, \"p50_us\": %.2f, \"p90_us\": %.2f, \"p99_us\": %.2f, \"p999_us\": %.2f, "
-           "\"max_us\": %.2f, \"evaluated_mean\": %.1f, \"evaluated_max\": %llu, \"drops\": %d, \"launches\": %llu}\n",
+           "\"max_us\": %.2f, \"evaluated_mean\": %.1f, \"evaluated_max\": %llu, \"evaluated_p50\": %llu, "
+           "\"evaluated_p90\": %llu, \"evaluated_p99\": %llu, \"drops\": %d, \"launches\": %llu}\n",
            n, lat[warm + n / 2], lat[warm + (int)(0.9 * n)], lat[warm + (int)(0.99 * n)],
-           lat[warm + (int)(0.999 * n)], lat[ndec - 1], (double)evsum / n, (unsigned long long)evmax, ndrop,
-           (unsigned long long)abacus_kernel_launches(ctx));
+           lat[warm + (int)(0.999 * n)], lat[ndec - 1], (double)evsum / n, (unsigned long long)evmax,
+           (unsigned long long)ev[warm + n / 2], (unsigned long long)ev[warm + (int)(0.9 * n)],
+           (unsigned long long)ev[warm + (int)(0.99 * n)], ndrop, (unsigned long long)abacus_kernel_launches(ctx));
     abacus_destroy(ctx);
     return 0;
 }
