@@ -1146,9 +1146,24 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
         rw.now = now_ms[i];
         rw.infl = inflight_pred_ms[i];
         rw.k = ki;
-        for (int j = 0; j < kc; j++) {  // a slot's digit counts at most L - next_op + 1 end ops
+        // widest digit = L - next_op + 1 over the non-critical queries (the critical
+        // query's slot is fixed): the same bound a single round derives from its
+        // plan, so a batch picks the same layer-1 layout (and the same arithmetic)
+        // as abacus_search of each of its rounds. The critical query is the
+        // smallest headroom, ties to the smaller model id (a1, reading c10).
+        int crit = 0;
+        double hc = 0.0;
+        for (int j = 0; j < kc; j++) {
             const abacus_query_t& a = rw.q[j];
-            if (a.model_id >= 1 && a.model_id <= c->n_models && a.next_op >= 1) {
+            const double h = (a.qos_ms - (rw.now - a.t_start_ms)) - rw.infl;
+            if (j == 0 || h < hc || (h == hc && a.model_id < rw.q[crit].model_id)) {
+                crit = j;
+                hc = h;
+            }
+        }
+        for (int j = 0; j < kc; j++) {
+            const abacus_query_t& a = rw.q[j];
+            if (j != crit && a.model_id >= 1 && a.model_id <= c->n_models && a.next_op >= 1) {
                 const int32_t w = c->L[a.model_id - 1] - a.next_op + 1;
                 if (w > 0 && (uint32_t)w > maxcnt) maxcnt = (uint32_t)w;
             }
