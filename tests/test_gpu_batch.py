@@ -195,3 +195,24 @@ def test_batch_validation_matches_single_rounds(prec):
             _same(d, ab.abacus_search(c.h, qs, now, infl))
     finally:
         c.close()
+
+
+def test_batch_layout_follows_single_round_bf16():
+    """bf16 splits the layer-1 digits above 257 end-op options. A long critical
+    query (whose slot is fixed) must not push a batch into the split layout
+    when every single round of it runs unsplit: the batch stays bit-identical."""
+    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_BF16)
+    try:
+        decs = []
+        for i in range(16):
+            # BERT-large (471 ops) from op 1 is critical (tiny headroom); the others
+            # have < 257 ops left, so no digit of the round exceeds 257 options
+            qs = [synth.Query(8, 1, 4, 128, 5.0 + 0.01 * i, 0.0),
+                  synth.Query(2, 241 - 100, 8, 0, 80.0, 0.0),
+                  synth.Query(4, 220 - 150, 8, 0, 90.0, 0.0)]
+            decs.append((qs, 0.0, 0.0))
+        got = ab.abacus_search_batch(c.h, decs)
+        for (qs, now, infl), d in zip(decs, got):
+            _same(d, ab.abacus_search(c.h, qs, now, infl))
+    finally:
+        c.close()
