@@ -1171,7 +1171,8 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     }
     cudaStream_t st = c->stream;
     CUDA_TRY(c, cudaMemcpyAsync(c->d_raw, c->h_raw, (size_t)n * sizeof(BatchRaw), cudaMemcpyHostToDevice, st));
-    batch_plan_kernel<<<(n + 127) / 128, 128, 0, st>>>(c->d_raw, n, c->n_models, c->D, c->d_L, space, grid_budget,
+    // one warp per block: the per-thread planner is latency-bound, so spread it over every SM
+    batch_plan_kernel<<<(n + 31) / 32, 32, 0, st>>>(c->d_raw, n, c->n_models, c->D, c->d_L, space, grid_budget,
                                                        c->d_decs, c->d_segs, c->d_pairs, c->d_a1);
     batch_scan_kernel<<<1, kScanThreads, 0, st>>>(c->d_decs, c->d_pairs, n);
     CUDA_TRY(c, cudaGetLastError());
