@@ -1546,6 +1546,10 @@ __global__ void __launch_bounds__(NG * 128, 1) predict24_tc_kernel(const __grid_
 // launchers
 // ---------------------------------------------------------------------------
 constexpr int kFusedNG = 5;
+#ifndef ABACUS_BATCH_NG
+#define ABACUS_BATCH_NG 5
+#endif
+constexpr int kBatchNG = ABACUS_BATCH_NG;  // groups per CTA of the batch search kernel
 constexpr int kPredictNG = 4;
 
 template <int FMT, bool SPLIT>
@@ -1598,14 +1602,14 @@ static cudaError_t launch_batch_fmt(const BatchDec* decs, const SegP* segs, int3
                                     uint64_t pairs_ub, int32_t D, const TcParams& tp, const float* w1b1,
                                     BatchAcc* acc, float* y0s, int nsm, cudaStream_t st) {
     uint32_t plans_off;
-    const TcSmem L = batch_smem_layout<FMT>(D, kFusedNG, &plans_off);
-    auto kern = fused_batch_tc_kernel<FMT, SPLIT, kFusedNG>;
+    const TcSmem L = batch_smem_layout<FMT>(D, kBatchNG, &plans_off);
+    auto kern = fused_batch_tc_kernel<FMT, SPLIT, kBatchNG>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (e != cudaSuccess) return e;
-    uint64_t g = (pairs_ub + kFusedNG - 1) / kFusedNG;  // the exact count is only known on the device
+    uint64_t g = (pairs_ub + kBatchNG - 1) / kBatchNG;  // the exact count is only known on the device
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
-    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(decs, segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s);
+    kern<<<(int)g, kBatchNG * 128, L.total, st>>>(decs, segs, n_dec, n_pairs, D, tp, w1b1, acc, y0s);
     return cudaGetLastError();
 }
 
