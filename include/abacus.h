@@ -48,7 +48,7 @@ extern "C" {
 
 #define ABACUS_K_MAX 4
 #define ABACUS_HIDDEN 32
-#define ABACUS_ABI_VERSION 2
+#define ABACUS_ABI_VERSION 3
 #define ABACUS_BATCH_MAX (1 << 20) /* decisions per abacus_search_batch call */
 #define ABACUS_TRAIN_MAX_BATCH 65536 /* samples per training step */
 
@@ -69,7 +69,11 @@ enum {
     ABACUS_BF16 = 1, /* tcgen05 kind::f16, bf16 operands (weights split hi+lo),     */
                      /* fp32 accumulation in TMEM                                   */
     ABACUS_FP16 = 2  /* tcgen05 kind::f16, fp16 operands with exact power-of-two    */
-                     /* layer scaling, fp32 accumulation in TMEM                    */
+                     /* layer scaling; accumulation in TMEM is fp32 for layer 1 and */
+                     /* the output layer but F16 for hidden layers 2 and 3 (their   */
+                     /* biases are added in f16 in the epilogue); the output bias   */
+                     /* is added in fp32.  Error vs the fp64 oracle on config 5:    */
+                     /* max 1.5e-3 relative (reading r2)                  */
 };
 
 /* candidate space of abacus_search (reading c13) */
@@ -287,12 +291,50 @@ int abacus_search_mway(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, doub
  * (an ncclComm_t on this device, e.g. from abacus_nccl_comm_init) the
  * per-rank results are combined with one collective so every rank returns
  * the same global decision (status OK or NONE, end_op per slot, pred_ms of
- * t*, evaluated summed over ranks).  Validation: 1 <= k <= 4, model ids in
+ * t*, evaluated summed over ranks, pred_critical_only_ms = y(index 0) from
+ * the rank whose shard holds index 0; see abacus_combine_decisions).
+ * Without a communicator pred_critical_only_ms = y(index 0) if
+ * first == 0 < count, else NaN.  Validation: 1 <= k <= 4, model ids in
  * [1, N] and distinct, 1 <= start_op <= end_lo <= end_hi <= L, batch >= 1,
  * seqlen >= 0, T < 2^40, max sum_n + 1 < 2^24.  Errors: E_INVALID,
  * E_DUP_MODEL, E_NOT_LOADED, E_CUDA, E_NCCL. */
 int abacus_search_grid(abacus_ctx* ctx, const abacus_grid_t* grid, float headroom_ms, uint64_t first,
                        uint64_t count, void* nccl_comm, abacus_decision_t* out);
+
+/* Per-decision sharded search (the paper's search is
+ * single-node): the decision of abacus_search(q, k, now_ms,
+ * inflight_pred_ms, space, grid_budget), computed by all ranks of `nccl_comm`
+ * together.  Every rank must pass the same arguments.  Each rank runs a1
+ * itself (deterministic: same order and H everywhere); a GRID decision's
+ * index space [0, T) is split into contiguous shards
+ * [floor(rT/G), floor((r+1)T/G)) over the G ranks, each rank searches its
+ * shard with the fused kernel, and one ncclAllGather of the per-rank records
+ * plus a 1-thread combine kernel (max key; y(0) for the drop test from the
+ * rank whose shard holds index 0) gives every rank the same decision.
+ * CHAIN decisions (incl. AUTO over the budget) are searched whole on every
+ * rank with no collective.  nccl_comm == NULL: exactly abacus_search.
+ * out->evaluated counts the candidates of all ranks.  Blocking.
+ * Errors: as abacus_search, plus E_NCCL. */
+int abacus_search_sharded(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double now_ms,
+                          double inflight_pred_ms, int32_t space, uint64_t grid_budget, void* nccl_comm,
+                          abacus_decision_t* out);
+
+/* The cross-GPU combine step (a6) on the host, no ctx and no device needed:
+ * per_rank[r] (host, nranks records, rank order) is rank r's
+ * abacus_search_grid result without a communicator over shard r of a
+ * contiguous partition of one grid under one headroom (status OK or NONE;
+ * pred_critical_only_ms is NaN unless the shard holds index 0).  *out =
+ * the global decision: the max key with its index, end_op, total_ops and
+ * pred_ms; evaluated summed; pred_critical_only_ms from the first record
+ * that holds index 0; status OK / NONE.  drop_test != 0 additionally applies
+ * the decision drop rule of abacus_search (reading c14): status
+ * DROP iff !(pred_critical_only_ms <= headroom_ms), then pred_ms = that
+ * value, end_op and total_ops zero.  The device combine of
+ * abacus_search_grid / abacus_search_sharded runs the same function.
+ * Errors: E_INVALID (NULL, nranks outside [1, 64], headroom_ms differing
+ * between records, status other than OK/NONE, key inconsistent with status). */
+int abacus_combine_decisions(const abacus_decision_t* per_rank, int32_t nranks, int32_t drop_test,
+                             abacus_decision_t* out);
 
 /* ------------------------------------------------------------------------ */
 /* NCCL bootstrap helpers (multi-GPU sweeps; one process per GPU)            */

@@ -29,7 +29,8 @@ K_MAX = 4
 
 EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load_predictor",
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
-            "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_nccl_unique_id",
+            "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_search_sharded",
+            "abacus_combine_decisions", "abacus_nccl_unique_id",
             "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
             "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version",
             "abacus_train_begin", "abacus_train_step", "abacus_train_epoch", "abacus_train_params"]
@@ -107,6 +108,9 @@ def lib():
                                          P(abacus_decision_t), P(C.c_int32)]
         L.abacus_search_grid.argtypes = [vp, P(abacus_grid_t), C.c_float, C.c_uint64, C.c_uint64, vp,
                                          P(abacus_decision_t)]
+        L.abacus_search_sharded.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
+                                            C.c_uint64, vp, P(abacus_decision_t)]
+        L.abacus_combine_decisions.argtypes = [P(abacus_decision_t), C.c_int32, C.c_int32, P(abacus_decision_t)]
         L.abacus_nccl_unique_id.argtypes = [P(C.c_uint8)]
         L.abacus_nccl_comm_init.argtypes = [vp, C.c_int32, C.c_int32, P(C.c_uint8), P(vp)]
         L.abacus_nccl_comm_destroy.argtypes = [vp]
@@ -255,6 +259,26 @@ def abacus_search_grid(ctx, grid: abacus_grid_t, headroom_ms: float, first: int,
     out = abacus_decision_t()
     _check(ctx, lib().abacus_search_grid(ctx, C.byref(grid), float(headroom_ms), first, count, nccl_comm,
                                          C.byref(out)))
+    return out
+
+
+def abacus_search_sharded(ctx, queries, now_ms: float, inflight_pred_ms: float, space: int = ABACUS_SPACE_GRID,
+                          grid_budget: int = 2**40, nccl_comm: Optional[int] = None) -> abacus_decision_t:
+    k = len(queries)
+    qa = (abacus_query_t * k)(*[abacus_query_t(q.model_id, q.next_op, q.batch, q.seqlen, q.qos_ms,
+                                               q.t_start_ms) for q in queries])
+    out = abacus_decision_t()
+    _check(ctx, lib().abacus_search_sharded(ctx, qa, k, float(now_ms), float(inflight_pred_ms), space, grid_budget,
+                                            nccl_comm, C.byref(out)))
+    return out
+
+
+def abacus_combine_decisions(per_rank: Sequence[abacus_decision_t], drop_test: bool = False) -> abacus_decision_t:
+    """Host-side a6 combine of per-rank sweep decisions (rank order); needs no GPU."""
+    n = len(per_rank)
+    arr = (abacus_decision_t * max(n, 1))(*per_rank)
+    out = abacus_decision_t()
+    _check(None, lib().abacus_combine_decisions(arr, n, 1 if drop_test else 0, C.byref(out)))
     return out
 
 

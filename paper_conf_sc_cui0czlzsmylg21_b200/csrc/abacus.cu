@@ -14,6 +14,8 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
+#include <cstdlib>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -116,6 +118,7 @@ struct NcclApi {
     ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
     ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
     ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
+    ncclResult_t (*CommUserRank)(const ncclComm_t, int*) = nullptr;
     ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
     const char* (*GetErrorString)(ncclResult_t) = nullptr;
 };
@@ -133,9 +136,10 @@ const NcclApi& nccl() {
     api.CommInitRank = (decltype(api.CommInitRank))dlsym(h, "ncclCommInitRank");
     api.CommDestroy = (decltype(api.CommDestroy))dlsym(h, "ncclCommDestroy");
     api.CommCount = (decltype(api.CommCount))dlsym(h, "ncclCommCount");
+    api.CommUserRank = (decltype(api.CommUserRank))dlsym(h, "ncclCommUserRank");
     api.AllGather = (decltype(api.AllGather))dlsym(h, "ncclAllGather");
     api.GetErrorString = (decltype(api.GetErrorString))dlsym(h, "ncclGetErrorString");
-    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.CommCount && api.AllGather &&
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.CommCount && api.CommUserRank && api.AllGather &&
              api.GetErrorString;
     return api;
 }
@@ -584,7 +588,20 @@ uint32_t next_seq(abacus_ctx*) {
     return s;
 }
 
+// A search that has not published after ABACUS_WAIT_TIMEOUT_S seconds (default
+// 300: a full config-4 sweep in fp32 takes about 1 s) is reported as E_CUDA
+// instead of spinning forever; the ctx's stream may still hold the hung work.
+double wait_timeout_s() {
+    static double t = [] {
+        const char* e = getenv("ABACUS_WAIT_TIMEOUT_S");
+        const double v = e ? atof(e) : 0.0;
+        return v > 0.0 ? v : 300.0;
+    }();
+    return t;
+}
+
 int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
+    const auto t0 = std::chrono::steady_clock::now();
     for (uint64_t spin = 1;; spin++) {
         if (rec_read(c->host_result, seq, R)) break;
         if ((spin & 1023) == 0) {
@@ -593,6 +610,10 @@ int wait_result(abacus_ctx* c, uint32_t seq, Result* R) {
                 return fail(c, ABACUS_E_CUDA, "search kernel failed: %s", cudaGetErrorString(e));
             if (e == cudaSuccess && !rec_read(c->host_result, seq, R))
                 return fail(c, ABACUS_E_CUDA, "search finished without publishing its result");
+            const double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            if (dt > wait_timeout_s())
+                return fail(c, ABACUS_E_CUDA, "search did not publish its result within %.0f s "
+                            "(ABACUS_WAIT_TIMEOUT_S); the ctx stream still holds the work", dt);
         }
     }
     std::atomic_thread_fence(std::memory_order_acquire);
@@ -844,6 +865,32 @@ void host_decode(const Plan& P, Result& R) {
         R.end_op[j] = (R.key && j < P.k) ? decode_slot_ope(P, R.key & ((1ull << 40) - 1), j) : 0;
 }
 
+// (nranks, rank) of an NCCL communicator (the NCCL copy the process already loaded)
+int comm_shape(abacus_ctx* c, void* comm, int* nranks, int* rank) {
+    if (!nccl().ok) return fail(c, ABACUS_E_NCCL, "libnccl.so.2 not available");
+    if (nccl().CommCount((ncclComm_t)comm, nranks) != ncclSuccess || *nranks < 1 || *nranks > 64 ||
+        nccl().CommUserRank((ncclComm_t)comm, rank) != ncclSuccess || *rank < 0 || *rank >= *nranks)
+        return fail(c, ABACUS_E_NCCL, "bad communicator");
+    return ABACUS_OK;
+}
+
+// a6 after a fused launch whose last CTA left this rank's record in S->result
+// (P.mapped == null, so end ops are decoded on the device): one ncclAllGather
+// of the 56-byte records on the ctx stream, then one 1-thread kernel runs
+// combine_results (common.cuh) and publishes the global record to the mapped
+// copy tagged `seq`.
+int combine_over_comm(abacus_ctx* c, void* comm, uint32_t seq) {
+    int nranks = 0, rank = 0;
+    int rc = comm_shape(c, comm, &nranks, &rank);
+    if (rc) return rc;
+    ncclResult_t nr =
+        nccl().AllGather(&c->S->result, c->S->gathered, sizeof(Result), ncclUint8, (ncclComm_t)comm, c->stream);
+    if (nr != ncclSuccess) return fail(c, ABACUS_E_NCCL, "ncclAllGather: %s", nccl().GetErrorString(nr));
+    CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->dev_result, seq, c->stream));
+    c->launches++;
+    return ABACUS_OK;
+}
+
 abacus_decision_t assemble_decision(const Result& R, const int32_t* order, int32_t k, float H, uint64_t n_eval) {
     abacus_decision_t d{};
     d.critical = order[0];
@@ -969,6 +1016,10 @@ int abacus_load_predictor(abacus_ctx* c, const float* params, size_t n_params, i
     for (size_t i = 0; i < n_params; i++)
         if (!std::isfinite(params[i])) return fail(c, ABACUS_E_INVALID, "param %zu is not finite", i);
     CUDA_TRY(c, cudaSetDevice(c->device));
+    // async predict / search work queued on any stream may still read the old
+    // weights (W2..W4 travel by value, W1/b1 and the blobs by pointer): finish
+    // it before the device copies are overwritten or freed
+    CUDA_TRY(c, cudaDeviceSynchronize());
     c->params.assign(params, params + n_params);
     const int D = c->D;
     const float* p = c->params.data();
@@ -1121,12 +1172,29 @@ int abacus_search_batch(abacus_ctx* c, const abacus_query_t* q, const int32_t* k
     if (space < ABACUS_SPACE_GRID || space > ABACUS_SPACE_AUTO) return fail(c, ABACUS_E_INVALID, "bad space");
     if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
     if (c->precision == ABACUS_FP32) {
-        // the fp32 SIMT path has no batched kernel: one fused launch per decision
+        // the fp32 SIMT path has no batched kernel: one fused launch per decision.
+        // Every decision is validated (a1) first and the results go to a scratch
+        // array, so an error names its decision and leaves `out` untouched.
+        for (int32_t i = 0; i < n; i++) {
+            int32_t order[ABACUS_K_MAX];
+            float H = 0.0f;
+            abacus_grid_t g{};
+            const int rc = decision_slots(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], order, &H, &g);
+            if (rc) {
+                c->err = "decision " + std::to_string(i) + ": " + c->err;
+                return rc;
+            }
+        }
+        std::vector<abacus_decision_t> tmp((size_t)n);
         for (int32_t i = 0; i < n; i++) {
             const int rc = abacus_search(c, q + 4 * (size_t)i, k[i], now_ms[i], inflight_pred_ms[i], space,
-                                         grid_budget, &out[i]);
-            if (rc) return rc;
+                                         grid_budget, &tmp[(size_t)i]);
+            if (rc) {
+                c->err = "decision " + std::to_string(i) + ": " + c->err;
+                return rc;
+            }
         }
+        memcpy(out, tmp.data(), sizeof(abacus_decision_t) * (size_t)n);
         return ABACUS_OK;
     }
     CUDA_TRY(c, cudaSetDevice(c->device));
@@ -1259,18 +1327,16 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     const uint32_t seq = next_seq(c);
     P.mapped = nccl_comm ? nullptr : c->dev_result;  // with a combine, the finalize kernel publishes
     P.seq = seq;
+    if (nccl_comm) {
+        int nranks = 0, rank = 0;
+        rc = comm_shape(c, nccl_comm, &nranks, &rank);
+        if (rc) return rc;
+    }
     rc = launch_fused(c, P);
     if (rc) return rc;
     if (nccl_comm) {
-        int nranks = 0;
-        ncclComm_t comm = (ncclComm_t)nccl_comm;
-        if (!nccl().ok) return fail(c, ABACUS_E_NCCL, "libnccl.so.2 not available");
-        if (nccl().CommCount(comm, &nranks) != ncclSuccess || nranks < 1 || nranks > 64)
-            return fail(c, ABACUS_E_NCCL, "bad communicator");
-        ncclResult_t nr = nccl().AllGather(&c->S->result, c->S->gathered, sizeof(Result), ncclUint8, comm, c->stream);
-        if (nr != ncclSuccess) return fail(c, ABACUS_E_NCCL, "ncclAllGather: %s", nccl().GetErrorString(nr));
-        CUDA_TRY(c, launch_finalize_gather(c->S, nranks, c->dev_result, seq, c->stream));
-        c->launches++;
+        rc = combine_over_comm(c, nccl_comm, seq);
+        if (rc) return rc;
     }
     Result R;
     rc = wait_result(c, seq, &R);
@@ -1288,6 +1354,89 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     d.pred_ms = R.key ? R.y_best : NAN;
     d.total_ops = R.total_ops;
     for (int j = 0; j < grid->k; j++) d.end_op[j] = R.end_op[j];
+    *out = d;
+    return ABACUS_OK;
+}
+
+// Per-decision sharded search: every rank runs a1 on the same
+// inputs (deterministic, so every rank derives the same grid, order and H), a
+// GRID decision's index space is split into the contiguous shard of this rank,
+// the fused kernel searches it, and one all-gather + combine_results gives every
+// rank the global record; the drop test uses y(0) from the rank whose shard holds
+// index 0.  A CHAIN decision (<= a few thousand candidates: launch-bound) is
+// searched whole on every rank, with no collective.
+int abacus_search_sharded(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now_ms, double inflight_pred_ms,
+                          int32_t space, uint64_t grid_budget, void* nccl_comm, abacus_decision_t* out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!out) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (space < ABACUS_SPACE_GRID || space > ABACUS_SPACE_AUTO) return fail(c, ABACUS_E_INVALID, "bad space");
+    if (!nccl_comm) return abacus_search(c, q, k, now_ms, inflight_pred_ms, space, grid_budget, out);
+    int32_t order[ABACUS_K_MAX];
+    float H = 0.0f;
+    abacus_grid_t g{};
+    uint64_t T = 0;
+    int rc = decision_slots(c, q, k, now_ms, inflight_pred_ms, order, &H, &g, &T);
+    if (rc) return rc;
+    const bool chain = space == ABACUS_SPACE_CHAIN || (space == ABACUS_SPACE_AUTO && T > grid_budget);
+    if (chain) return abacus_search(c, q, k, now_ms, inflight_pred_ms, space, grid_budget, out);
+    int nranks = 0, rank = 0;
+    rc = comm_shape(c, nccl_comm, &nranks, &rank);
+    if (rc) return rc;
+    const uint64_t first = (uint64_t)rank * T / (uint64_t)nranks;  // T < 2^40, nranks <= 64: no overflow
+    const uint64_t last = (uint64_t)(rank + 1) * T / (uint64_t)nranks;
+    Plan P;
+    plan_grid_segments_into(static_cast<PlanHdr&>(P), PlanSink{&P}, c->n_models, c->D, &g, T, first, last, H);
+    P.mapped = nullptr;  // the finalize kernel publishes the combined record
+    P.seq = next_seq(c);
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    rc = launch_fused(c, P);
+    if (rc) return rc;
+    rc = combine_over_comm(c, nccl_comm, P.seq);
+    if (rc) return rc;
+    Result R;
+    rc = wait_result(c, P.seq, &R);
+    if (rc) return rc;
+    *out = assemble_decision(R, order, k, H, R.evaluated);
+    return ABACUS_OK;
+}
+
+// a6 on the host (no device work): the same combine_results as the finalize
+// kernel, over per-rank sweep decisions.
+int abacus_combine_decisions(const abacus_decision_t* per_rank, int32_t nranks, int32_t drop_test,
+                             abacus_decision_t* out) {
+    if (!per_rank || !out || nranks < 1 || nranks > 64) return ABACUS_E_INVALID;
+    Result r[64];
+    for (int32_t i = 0; i < nranks; i++) {
+        const abacus_decision_t& d = per_rank[i];
+        if (memcmp(&d.headroom_ms, &per_rank[0].headroom_ms, sizeof(float)) != 0) return ABACUS_E_INVALID;
+        if (d.status != ABACUS_DECIDE_OK && d.status != ABACUS_DECIDE_NONE) return ABACUS_E_INVALID;
+        if ((d.key == 0) != (d.status == ABACUS_DECIDE_NONE)) return ABACUS_E_INVALID;
+        Result& R = r[i];
+        R = Result{};
+        R.key = d.key;
+        R.y_best = d.pred_ms;
+        R.y0 = d.pred_critical_only_ms;
+        R.evaluated = d.evaluated;
+        for (int j = 0; j < kKMax; j++) R.end_op[j] = d.end_op[j];
+        R.total_ops = d.total_ops;
+    }
+    const Result R = combine_results(r, nranks);
+    abacus_decision_t d = per_rank[0];
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    d.evaluated = R.evaluated;
+    d.pred_critical_only_ms = R.y0;
+    d.total_ops = R.key ? R.total_ops : 0;
+    d.pred_ms = R.key ? R.y_best : NAN;
+    for (int j = 0; j < 4; j++) d.end_op[j] = R.key ? R.end_op[j] : 0;
+    d.status = R.key ? ABACUS_DECIDE_OK : ABACUS_DECIDE_NONE;
+    if (drop_test && !(R.y0 <= d.headroom_ms)) {  // drop mechanism (reading c14)
+        d.status = ABACUS_DECIDE_DROP;
+        d.pred_ms = R.y0;
+        d.total_ops = 0;
+        for (int j = 0; j < 4; j++) d.end_op[j] = 0;
+    }
     *out = d;
     return ABACUS_OK;
 }
@@ -1440,10 +1589,15 @@ int abacus_internal_set_trace(void* d_stamps) {
 
 int abacus_set_stream(abacus_ctx* c, void* stream) {
     if (!c) return ABACUS_E_INVALID;
-    if (c->own_stream && c->stream != (cudaStream_t)stream && stream) {
+    // the blocking calls share the ctx's scratch, mapped record and batch /
+    // training buffers: whenever the effective stream changes (including the
+    // reset to the ctx's own stream), finish the work queued on the old one
+    const cudaStream_t next = stream ? (cudaStream_t)stream : c->own_stream;
+    if (next != c->stream) {
+        cudaSetDevice(c->device);
         cudaStreamSynchronize(c->stream);
     }
-    c->stream = stream ? (cudaStream_t)stream : c->own_stream;
+    c->stream = next;
     return ABACUS_OK;
 }
 

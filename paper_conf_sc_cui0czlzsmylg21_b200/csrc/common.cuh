@@ -69,6 +69,12 @@ struct Result {
     uint32_t pad;
 };
 
+__host__ __device__ inline float f32_from_bits(uint32_t b) {
+    float f;
+    memcpy(&f, &b, 4);
+    return f;
+}
+
 // Host-mapped copy of a Result: four 16-byte chunks of three payload words and
 // a tag, tag = seq ^ mix(payload, chunk index). The device writes it with four
 // vector stores and no system fence; the host accepts the record once all four
@@ -123,6 +129,34 @@ inline bool rec_read(const MappedRec* M, uint32_t seq, Result* R) {
     }
     rec_unpayload(p, *R);
     return true;
+}
+
+// a6: the global result of a contiguously sharded candidate space from the
+// per-rank records r[0..n) (rank order, shard r = [floor(rT/G), floor((r+1)T/G))).
+// Max key (a key embeds its index, so two records never tie unless both are 0),
+// y(t*) / end ops / total ops from the winning record, evaluated summed, and
+// y(0) -- the drop test's prediction (reading c14) -- from the
+// first record that evaluated index 0: only that rank's shard holds it, every
+// other rank publishes NaN there.  Shared by the device finalize kernel (after
+// the NCCL all-gather) and the host entry point abacus_combine_decisions.
+__host__ __device__ inline Result combine_results(const Result* r, int n) {
+    int best = 0;
+    unsigned long long ev = 0;
+    float y0 = f32_from_bits(0x7fc00000u);
+    bool have_y0 = false;
+    for (int i = 0; i < n; i++) {
+        ev += r[i].evaluated;
+        if (r[i].key > r[best].key) best = i;
+        if (!have_y0 && r[i].y0 == r[i].y0) {
+            y0 = r[i].y0;
+            have_y0 = true;
+        }
+    }
+    Result out = r[best];
+    out.evaluated = ev;
+    out.y0 = y0;
+    out.status = out.key ? 0 : 2;
+    return out;
 }
 
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };

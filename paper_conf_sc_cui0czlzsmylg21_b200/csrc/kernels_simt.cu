@@ -624,14 +624,7 @@ __global__ void __launch_bounds__(kFused2Threads, kFused2BlocksPerSM) fused_fp32
 // ---------------------------------------------------------------------------
 __global__ void finalize_gather_kernel(Scratch* S, int nranks, MappedRec* mapped, uint32_t seq) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    int best = 0;
-    unsigned long long ev = 0;
-    for (int r = 0; r < nranks; r++) {
-        ev += S->gathered[r].evaluated;
-        if (S->gathered[r].key > S->gathered[best].key) best = r;
-    }
-    S->result = S->gathered[best];
-    S->result.evaluated = ev;
+    S->result = combine_results(S->gathered, nranks);  // common.cuh, shared with the host
     if (mapped) publish_mapped(S->result, mapped, seq);
 }
 

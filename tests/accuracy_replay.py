@@ -8,7 +8,7 @@ oracle as the 'real' latency), a log-binned error histogram, and (bf16) the
 distance to the bf16-emulating oracle (rounding-point check).  Also times the
 standalone encode_groups / predict_batch kernels (CUDA events).
 
-  python tools/accuracy_replay.py [--n 1000000] [--out profiles/cfg5_accuracy.json]
+  python tests/accuracy_replay.py [--n 1000000] [--out profiles/cfg5_accuracy.json]
 """
 import argparse
 import json

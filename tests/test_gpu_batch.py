@@ -127,8 +127,9 @@ def test_batch_fp32_is_per_round():
         c.close()
 
 
-def test_batch_errors_name_the_decision():
-    c = Ctx(params=synth.weights(1), precision=ab.ABACUS_FP16)
+@pytest.mark.parametrize("prec", [ab.ABACUS_FP16, ab.ABACUS_BF16, ab.ABACUS_FP32], ids=["fp16", "bf16", "fp32"])
+def test_batch_errors_name_the_decision(prec):
+    c = Ctx(params=synth.weights(1), precision=prec)
     try:
         decs = synth.cfg2_decisions(5)
         bad = list(decs)

@@ -13,7 +13,7 @@ timeout 600 python tools/bench_kernels.py --out gpurun_out/${TAG}_kernels.json >
 for k in encode_grid24 select_kernel encode_groups24; do
   timeout 600 ncu --set full --clock-control none -k regex:$k -c 1 -o gpurun_out/${TAG}_$k python tools/bench_kernels.py --rows 16777216 --reps 1 > gpurun_out/${TAG}_ncu_$k.log 2>&1
 done
-timeout 600 python tools/accuracy_replay.py --out gpurun_out/${TAG}_acc.json > gpurun_out/${TAG}_acc.log 2>&1
+timeout 600 python tests/accuracy_replay.py --out gpurun_out/${TAG}_acc.json > gpurun_out/${TAG}_acc.log 2>&1
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err
 for p in bf16 fp32; do
   timeout 600 python bench.py --steps 5 --warmup 3 --precision $p --no-cpu-baseline --no-decisions > gpurun_out/${TAG}_bench_$p.json 2> gpurun_out/${TAG}_bench_$p.err

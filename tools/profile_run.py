@@ -37,9 +37,11 @@ for _ in range(1 + a.reps):
     d = ab.abacus_search_grid(ctx, g, synth.cfg4_headroom(), 0, T // a.frac)
 print("key", d.key, "evaluated", d.evaluated)
 if a.predict:
-    from oracle import encode_groups  # test infra: builds the input rows only
-    X = encode_groups(8, 4, [s.slots for s in synth.instance_samples(200_000, seed=15)])
-    x = torch.from_numpy(np.tile(X, (5, 1))).cuda()
+    G = [s.slots for s in synth.instance_samples(200_000, seed=15)]
+    gr = torch.frombuffer(bytearray(ab.make_groups(G)), dtype=torch.uint8).cuda()
+    X = torch.empty((len(G), 24), dtype=torch.int16, device="cuda")
+    ab.abacus_encode_groups(ctx, gr, len(G), X)  # the product's encoder builds the input rows
+    x = X.repeat(5, 1).contiguous()
     y = torch.empty(x.shape[0], device="cuda")
     for _ in range(2):
         ab.abacus_predict_batch(ctx, x, x.shape[0], y)
