@@ -15,9 +15,12 @@
  * replay, dyadic hand-computed MLP, brute-force enumeration, closed-form
  * counts, linear-predictor knapsack closed form, Eq. 2/3 worked example.
  * The bf16-emulating MLP (orc_mlp64_emu) is a secondary reference used only
- * to localise bf16 error; its rounding points are pinned by tests that
- * compare against numpy-free hand rounding of single values
- * (parity of the emulation itself beyond those points: unpinned).
+ * to localise bf16 error; its rounding points are pinned by hand-rounded
+ * single values, and the emulation as a whole against torch's independent
+ * fp32 -> bf16 conversion (tests/test_oracle_pins.py
+ * test_bf16_emulation_against_torch_rounding).  The determinism hash
+ * primitives (orc_splitmix64, orc_fnv1a64) are pinned by their published
+ * known answers.
  */
 #include <math.h>
 #include <stdint.h>

@@ -356,3 +356,93 @@ def test_multiway_equals_exhaustive_chain_under_monotone_predictor():
                 assert mw.u == ex.index and list(mw.end_op)[:k] == list(ex.end_op)[:k]
                 R = max(1, ex.evaluated)
                 assert mw.rounds <= 2 + int(np.ceil(np.log(R) / np.log(ways + 1)))
+
+
+# ------------------------------------------------- hash primitives ----
+def test_splitmix64_known_answers():
+    """SplitMix64 (Steele, Lea, Flood 2014; Vigna's reference generator) seeded
+    at 0: the state advances by the golden gamma 0x9E3779B97F4A7C15 and the
+    first three outputs are the published 0xE220A8397B1DCDAF,
+    0x6E789E6AA1B965F4, 0x06C45D188009454F.  orc_splitmix64(z) is one output
+    from state z (the gamma is added inside)."""
+    g = 0x9E3779B97F4A7C15
+    assert oracle.splitmix64(0) == 0xE220A8397B1DCDAF
+    assert oracle.splitmix64(g) == 0x6E789E6AA1B965F4
+    assert oracle.splitmix64((2 * g) % 2**64) == 0x06C45D188009454F
+
+
+def test_fnv1a64_known_answers():
+    """FNV-1a 64 (Fowler/Noll/Vo): the empty input gives the offset basis
+    0xcbf29ce484222325 and "foobar" the published 0x85944171f73967e8.  The
+    oracle hashes int16 feature values as little-endian bytes, so "foobar" is
+    the three int16 words 'fo' 'ob' 'ar'."""
+    assert oracle.fnv1a64(np.array([], dtype=np.int16)) == 0xCBF29CE484222325
+    words = np.frombuffer(b"foobar", dtype="<i2")
+    assert oracle.fnv1a64(words) == 0x85944171F73967E8
+    # byte order matters: the big-endian reading is a different string
+    assert oracle.fnv1a64(np.frombuffer(b"offbra", dtype="<i2")) != 0x85944171F73967E8
+
+
+def test_sweep_hash_is_the_sum_over_brute_force_rows():
+    """The sweep's determinism hash = sum_t splitmix64(t xor fnv1a64(x(t))) mod
+    2^64 over brute-force enumerated Fig.-8 rows (both primitives pinned above)."""
+    p = synth.raw_weights(2)
+    grid = [synth.GridSlot(2, 3, 4, 0, 3, 9, 1), synth.GridSlot(7, 1, 8, 64, 2, 6, 0)]
+    r, _, x, _ = oracle.sweep(p, grid, 0.0, want_x=True)
+    cands = brute.enumerate_grid(grid)
+    assert len(cands) == len(x)
+    h = 0
+    for t in range(len(x)):
+        h = (h + oracle.splitmix64(t ^ oracle.fnv1a64(x[t]))) % 2**64
+    assert r.hash == h
+
+
+# ------------------------------------------------ reading r2: why fp16, not plain bf16 ----
+def test_reading_r2_plain_bf16_misses_the_bar_on_config5():
+    """DESIGN.md reading r2: with plain bf16 (weights and post-ReLU activations
+    rounded RNE to bf16, fp64 accumulation: flags 1 | 8 of the emulation; the
+    integer features < 256 are exact and the larger ones round too with flag
+    4) the config-5 predictions miss the north star's 1e-2 relative bar
+    against the fp64 oracle (max 1.06e-2 / 1.08e-2 here), which is why the
+    tensor path uses fp16 operands (or split bf16 weights).  5e4
+    instance-based samples (Fig. 9)."""
+    params = synth.weights(1)
+    G = synth.instance_samples(50_000, seed=15)
+    X = oracle.encode_groups(8, 4, [g.slots for g in G])
+    y64 = oracle.mlp64_batch(params, X)
+    for flags in (1 | 8, 15):
+        ye = oracle.mlp64_emu_batch(params, X, flags=flags)
+        err = np.abs(ye - y64) / np.abs(y64)
+        assert err.max() > 1e-2, (flags, err.max())
+    # the weights alone (flags 1 | 2) already cost more than half the bar
+    ye = oracle.mlp64_emu_batch(params, X, flags=3)
+    assert (np.abs(ye - y64) / np.abs(y64)).max() > 5e-3
+
+
+def test_bf16_emulation_against_torch_rounding():
+    """orc_mlp64_emu pinned beyond single rounding points: flags 1|2 (weights,
+    biases) and 4 (features) equal the plain fp64 MLP evaluated on operands
+    pre-rounded by torch's own fp32 -> bf16 conversion (RNE), bit for bit; with
+    flag 8 (activations) a float64 numpy forward that rounds each post-ReLU
+    activation through torch bf16 agrees to fp64 rounding noise."""
+    torch = pytest.importorskip("torch")
+    params = synth.weights(1)
+    G = synth.instance_samples(3000, seed=5)
+    X = oracle.encode_groups(8, 4, [g.slots for g in G])
+    pr = torch.from_numpy(params.astype(np.float32)).to(torch.bfloat16).float().numpy()
+    assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=3), oracle.mlp64_batch(pr, X))
+    Xr = torch.from_numpy(X.astype(np.float32)).to(torch.bfloat16).float().numpy().astype(np.int16)
+    assert not np.array_equal(Xr, X)  # some features (>= 256) do round
+    assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=4), oracle.mlp64_batch(params, Xr))
+    W1, b1, W2, b2, W3, b3, w4, b4 = [a.astype(np.float64) for a in synth.split_params(params)]
+
+    def rb(a):  # fp64 -> bf16 via torch (the fp32 step is exact for these magnitudes up to 2^-24 rel)
+        return torch.from_numpy(a).to(torch.float32).to(torch.bfloat16).to(torch.float64).numpy()
+    h = rb(np.maximum(X.astype(np.float64) @ W1.T + b1, 0))
+    h = rb(np.maximum(h @ W2.T + b2, 0))
+    h = rb(np.maximum(h @ W3.T + b3, 0))
+    y = h @ w4 + b4[0]
+    ye = oracle.mlp64_emu_batch(params, X, flags=8)
+    d = np.abs(ye - y) / np.abs(y)
+    assert np.quantile(d, 0.99) <= 1e-12   # same roundings
+    assert d.max() <= 2 ** -7              # a rare tie flipped by fp64 summation order moves one activation by 1 ulp
