@@ -119,11 +119,13 @@ def cpu_oracle_rate_all_cores(params, slots, H, budget_s=8.0, chunk=50_000):
     counts = [0] * ncores
     t0 = time.perf_counter()
 
+    span = (T - T // 2) // ncores
+
     def work(w):
-        first = T // 2 + w * 10_000_000
+        first = T // 2 + w * span
         while time.perf_counter() - t0 < budget_s:
-            oracle.sweep(params, slots, H, first=first + counts[w], count=chunk)
-            counts[w] += chunk
+            r, _, _, _ = oracle.sweep(params, slots, H, first=first + counts[w], count=chunk)
+            counts[w] += r.evaluated
 
     ths = [threading.Thread(target=work, args=(w,)) for w in range(ncores)]
     for th in ths:
@@ -159,10 +161,16 @@ def run_reference(args, rank, world):
     T = oracle.grid_size(slots)
     ncores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
     per_thread = 100_000
+    # thread w sweeps its own contiguous range inside [T/2, T): starts spaced
+    # (T - T/2) / ncores apart (always inside the grid, whatever the core
+    # count); only the candidates the oracle actually evaluated are counted
+    span = (T - T // 2) // ncores
 
-    def step(i):
+    def step(i, counted):
         def work(w):
-            oracle.sweep(params, slots, H, first=T // 2 + w * 50_000_000 + i * per_thread, count=per_thread)
+            first = T // 2 + w * span + (i * per_thread) % max(1, span - per_thread)
+            r, _, _, _ = oracle.sweep(params, slots, H, first=first, count=per_thread)
+            counted[w] = r.evaluated
         ths = [threading.Thread(target=work, args=(w,)) for w in range(ncores)]
         for th in ths:
             th.start()
@@ -170,14 +178,18 @@ def run_reference(args, rank, world):
             th.join()
 
     for i in range(args.warmup):
-        step(i)
+        step(i, [0] * ncores)
+    counts = []
     t0 = time.perf_counter()
     for i in range(args.steps):
-        step(args.warmup + i)
+        c = [0] * ncores
+        step(args.warmup + i, c)
+        counts.append(sum(c))
     dt = time.perf_counter() - t0
-    per_step = per_thread * ncores
-    rate = per_step * args.steps / dt
-    sample = "%d config-4 candidates per step: %d threads x %d contiguous from T/2" % (per_step, ncores, per_thread)
+    per_step = int(np.mean(counts))
+    rate = sum(counts) / dt
+    sample = "%d config-4 candidates per step: %d threads x %d contiguous, spread over [T/2, T)" % (
+        per_step, ncores, per_thread)
     line = {"impl": "reference", "metric": METRIC, "value": rate, "unit": "candidates/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
@@ -197,6 +209,7 @@ def main():
     ap.add_argument("--precision", default="fp16", choices=list(PREC))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-decisions", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the bf16 / fp32 sweep keys")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -271,10 +284,20 @@ def main():
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_rate = T * e2e_steps / float(te[0])
 
+    # ---- per-decision sharded search (config 3 pure GRID, all ranks) --------
+    sharded = None
+    if not args.no_decisions:
+        sharded = sharded_decision_latency(ab, ctx, comm, world, rank)
+
     # ---- per-decision latency (config 2, 3-way; 1 GPU each) -----------------
     dec = None
     if rank == 0 and not args.no_decisions:
         dec = decision_latency(ab, ctx, precision=args.precision)
+
+    # ---- the other arithmetic paths on the same sweep (secondary keys) ------
+    secondary = None
+    if world == 1 and not args.no_secondary:
+        secondary = secondary_paths(ab, ctx, params, grid, H, T, args.precision, stream)
 
     if rank == 0:
         pk, src = peaks()
@@ -319,6 +342,8 @@ def main():
             "gpu_launches": launches,
             "clocks": clk.summary(),
             "decision_latency": dec,
+            "decision_latency_sharded": sharded,
+            "secondary_paths": secondary,
         }
         print(json.dumps(line))
     if comm:
@@ -326,6 +351,82 @@ def main():
     ab.abacus_destroy(ctx)
     if world > 1:
         dist.destroy_process_group()
+
+
+def fp32_fma_peak_tflops(sm_mhz):
+    """SIMT fp32 ceiling: 148 SMs x 128 FP32 lanes x 2 FLOP per FFMA x clock
+    (B200_PROFILING.md unit counts)."""
+    return 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
+
+
+def secondary_paths(ab, ctx, params, grid, H, T, headline, stream, steps=(("bf16", 6), ("fp32", 3))):
+    """The same config-4 sweep in the other arithmetic paths (DESIGN.md r2):
+    device time per sweep (CUDA events on the launching stream) and each
+    path's own roofline: the tensor paths against the measured bf16 peak
+    (fp16 = bf16 dense rate), fp32 SIMT against the FP32 FMA ceiling."""
+    import torch
+    out = {}
+    pk, src = peaks()
+    for name, n in steps:
+        if name == headline:
+            continue
+        ab.abacus_load_predictor(ctx, params, PREC[name])
+        d = ab.abacus_search_grid(ctx, grid, H, 0, T)  # warm-up
+        kms = []
+        with Clocks(0) as clk:
+            for _ in range(n):
+                d = ab.abacus_search_grid(ctx, grid, H, 0, T)
+                kms.append(ab.abacus_last_kernel_ms(ctx))
+        cs = clk.summary()
+        k = float(np.mean(kms))
+        achieved = FLOP_PER_CAND * T / (k / 1e3) / 1e12
+        if name == "fp32":
+            mhz = cs.get("sm_mhz") or 1965.0
+            peak, unit, bound, psrc = fp32_fma_peak_tflops(mhz), "TFLOP/s", "alu", \
+                "148 SM x 128 FFMA x 2 x %.0f MHz (median SM clock under load)" % mhz
+        else:
+            peak, unit, bound, psrc = pk["bf16_tflops"], "TFLOP/s", "tensor", src + ", burst"
+        out[name] = {"value": T / (k / 1e3), "unit": "candidates/s", "kernel_ms": k, "steps": n,
+                     "dtype": DTYPE[name], "selected_key": d.key,
+                     "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+                                  "frac": achieved / peak, "flop_per_candidate": FLOP_PER_CAND,
+                                  "peak_source": psrc},
+                     "clocks": cs}
+    ab.abacus_load_predictor(ctx, params, PREC[headline])
+    torch.cuda.synchronize()
+    return out
+
+
+def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50):
+    """Per-decision latency of abacus_search_sharded on config-3 4-way pure
+    GRID decisions (up to 4.1e7 candidates each): every rank searches its
+    contiguous shard of each decision's grid and one all-gather combines them
+    (SURVEY §8(d)/(e)).  At N = 1 there is no communicator (the local search).
+    Host clock around each blocking call on every rank; the per-decision time
+    is the max over ranks."""
+    import torch
+    import torch.distributed as dist
+    decs = synth.cfg3_decisions(n + warm)
+    lat = np.zeros(n)
+    ev = np.zeros(n)
+    for i, (qs, now, infl) in enumerate(decs):
+        t0 = time.perf_counter()
+        d = ab.abacus_search_sharded(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID, 2**40, comm)
+        t1 = time.perf_counter()
+        if i >= warm:
+            lat[i - warm] = (t1 - t0) * 1e6
+            ev[i - warm] = d.evaluated
+    t = torch.tensor(lat, dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    a = t.cpu().numpy()
+    return {"decisions": n, "n_gpus": world, "space": "grid (pure, config 3, 4-way)",
+            "p50_us": float(np.percentile(a, 50)), "p90_us": float(np.percentile(a, 90)),
+            "p99_us": float(np.percentile(a, 99)), "p999_us": float(np.percentile(a, 99.9)),
+            "max_us": float(a.max()), "grid_p50": float(np.percentile(ev, 50)), "grid_p99": float(np.percentile(ev, 99)),
+            "grid_max": float(ev.max()),
+            "path": "Python binding -> abacus_search_sharded (%s)" % (
+                "NCCL all-gather over %d ranks" % world if world > 1 else "1 GPU, no collective")}
 
 
 def decision_latency(ab, ctx, n=10_000, warm=100, precision="fp16"):
@@ -338,7 +439,7 @@ def decision_latency(ab, ctx, n=10_000, warm=100, precision="fp16"):
         sys.path.insert(0, os.path.join(ROOT, "tools"))
         import decision_latency as dl
         for cfg, space, budget in (("cfg2", "grid", 0), ("cfg3", "chain", 0), ("cfg3", "auto", 1 << 20),
-                                   ("cfg3", "auto", 1 << 22)):
+                                   ("cfg3", "auto", 1 << 22), ("cfg3", "grid", 0)):
             key = "%s_%s" % (cfg, space) + ("_%d" % budget if space == "auto" else "")
             out[key] = dl.run(cfg, space, precision, n, warm, budget or 4_194_304)
         # NEXT-4: many rounds per call (abacus_search_batch), decisions/s
