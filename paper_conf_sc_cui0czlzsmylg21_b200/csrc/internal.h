@@ -17,6 +17,12 @@ struct W234 {
     float b4;
 };
 
+// layer 1 in fp32 for the D = 24 SIMT predictor (kernel parameter, constant bank)
+struct W1P {
+    float W1[kHidden][24];
+    float b1[kHidden];
+};
+
 // tensor-core weight blob: layer 2 / layer 3 / output chunks in the shared
 // memory B-operand layout (tc_ptx.cuh b_offset), prepared at load time
 struct TcWeights {
@@ -33,8 +39,8 @@ cudaError_t launch_encode_grid(const Plan& P, uint64_t first, uint64_t count, in
                                cudaStream_t st);
 cudaError_t launch_encode_groups(const void* groups, uint64_t count, int32_t n_models, int32_t D, int16_t* out,
                                  uint32_t* bad, int nsm, cudaStream_t st);
-cudaError_t launch_predict_fp32(const W234& W, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
-                                float* y, int nsm, cudaStream_t st);
+cudaError_t launch_predict_fp32(const W234& W, const W1P* w1p, const float* w1b1, int32_t D, const int16_t* x,
+                                uint64_t count, float* y, int nsm, cudaStream_t st);
 cudaError_t launch_select(const Plan& P, uint64_t first, uint64_t count, const float* lat, float H,
                           unsigned long long* best, int nsm, cudaStream_t st);
 cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, Scratch* S, int nsm,

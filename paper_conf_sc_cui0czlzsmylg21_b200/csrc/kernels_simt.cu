@@ -300,6 +300,87 @@ __global__ void __launch_bounds__(kPredThreads) predict_fp32_kernel(const __grid
     }
 }
 
+// D = 24 (the registry's canonical width): layer 1 from the kernel parameters
+// too, so every FFMA of the row takes its weight from the constant bank (no
+// shared-memory load per FMA, which bound the generic kernel at 0.36 of the
+// FP32 FMA rate).  Each thread runs R = 2 consecutive rows so every weight
+// brought into a uniform register (LDCU) feeds two FFMAs; the 2 x 48-byte rows
+// are read with six 16-byte streaming loads.
+constexpr int kPred24Rows = 2;
+
+__global__ void __launch_bounds__(kPredThreads) predict24_fp32_kernel(const __grid_constant__ W1P A,
+                                                                      const __grid_constant__ W234 W,
+                                                                      const int16_t* __restrict__ x, uint64_t count,
+                                                                      float* __restrict__ y) {
+    constexpr int D = 24, R = kPred24Rows;
+    const uint64_t npair = (count + R - 1) / R;
+    for (uint64_t pi = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; pi < npair;
+         pi += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t row0 = pi * R;
+        float xv[R][D];
+#pragma unroll
+        for (int rr = 0; rr < R; rr++) {
+            // a missing last row re-reads row0 (its result is not stored)
+            const uint64_t row = row0 + rr < count ? row0 + rr : row0;
+            const uint4* rp = reinterpret_cast<const uint4*>(x + row * D);
+#pragma unroll
+            for (int q = 0; q < 3; q++) {
+                const uint4 v = __ldcs(rp + q);
+                const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                for (int i = 0; i < 4; i++) {
+                    xv[rr][8 * q + 2 * i] = (float)(int16_t)(w[i] & 0xFFFFu);
+                    xv[rr][8 * q + 2 * i + 1] = (float)(int16_t)(w[i] >> 16);
+                }
+            }
+        }
+        float h[R][kHidden];
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) {
+            float s[R];
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) s[rr] = 0.0f;
+#pragma unroll
+            for (int j = 0; j < D; j++)
+#pragma unroll
+                for (int rr = 0; rr < R; rr++) s[rr] = fmaf(A.W1[i][j], xv[rr][j], s[rr]);
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) h[rr][i] = fmaxf(s[rr] + A.b1[i], 0.0f);
+        }
+        float h2[R][kHidden];
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) {
+            float s[R];
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) s[rr] = W.b2[i];
+#pragma unroll
+            for (int j = 0; j < kHidden; j++)
+#pragma unroll
+                for (int rr = 0; rr < R; rr++) s[rr] = fmaf(W.W2[i][j], h[rr][j], s[rr]);
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) h2[rr][i] = fmaxf(s[rr], 0.0f);
+        }
+        float acc[R];
+#pragma unroll
+        for (int rr = 0; rr < R; rr++) acc[rr] = W.b4;
+#pragma unroll
+        for (int i = 0; i < kHidden; i++) {
+            float s[R];
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) s[rr] = W.b3[i];
+#pragma unroll
+            for (int j = 0; j < kHidden; j++)
+#pragma unroll
+                for (int rr = 0; rr < R; rr++) s[rr] = fmaf(W.W3[i][j], h2[rr][j], s[rr]);
+#pragma unroll
+            for (int rr = 0; rr < R; rr++) acc[rr] = fmaf(W.w4[i], fmaxf(s[rr], 0.0f), acc[rr]);
+        }
+#pragma unroll
+        for (int rr = 0; rr < R; rr++)
+            if (row0 + rr < count) __stcs(y + row0 + rr, acc[rr]);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // a5: headroom mask + largest-group key over a grid range.  Each thread walks
 // kSelPer consecutive candidates (two 16-byte loads of y), decoding only the
@@ -960,9 +1041,15 @@ cudaError_t launch_encode_groups(const void* groups, uint64_t count, int32_t n_m
     return cudaGetLastError();
 }
 
-cudaError_t launch_predict_fp32(const W234& W, const float* w1b1, int32_t D, const int16_t* x, uint64_t count,
-                                float* y, int nsm, cudaStream_t st) {
+cudaError_t launch_predict_fp32(const W234& W, const W1P* w1p, const float* w1b1, int32_t D, const int16_t* x,
+                                uint64_t count, float* y, int nsm, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
+    if (D == 24 && w1p && (reinterpret_cast<uintptr_t>(x) & 15u) == 0) {
+        const uint64_t blocks = ((count + kPred24Rows - 1) / kPred24Rows + kPredThreads - 1) / kPredThreads;
+        const int grid = (int)(blocks < (uint64_t)nsm * 16 ? blocks : (uint64_t)nsm * 16);
+        predict24_fp32_kernel<<<grid, kPredThreads, 0, st>>>(*w1p, W, x, count, y);
+        return cudaGetLastError();
+    }
     const uint64_t blocks = (count + kPredThreads - 1) / kPredThreads;
     const int grid = (int)(blocks < (uint64_t)nsm * 8 ? blocks : (uint64_t)nsm * 8);
     const size_t smem = (size_t)(kHidden * D + kHidden) * sizeof(float);

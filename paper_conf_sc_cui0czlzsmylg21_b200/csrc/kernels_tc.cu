@@ -46,7 +46,7 @@ struct TcParams {
 
 template <int FMT>
 struct TcCfg {
-    static constexpr int kNchL1 = FMT == 0 ? 1 : 2;      // layer-1 B chunks per segment (fused)
+    static constexpr int kNchL1 = 1;                     // layer-1 B chunks per segment (fused; fp16 table)
     static constexpr int kNchHid = FMT == 0 ? 3 : 5;     // hidden-layer B chunks
     static constexpr int kNchOut = FMT == 0 ? 3 : 5;     // output-layer B chunks
     static constexpr uint32_t kOne2 = FMT == 0 ? 0x3C003C00u : 0x3F803F80u;  // (1, 1)
@@ -63,7 +63,8 @@ __device__ __forceinline__ void split16(float v, uint16_t& hi, uint16_t& lo) {
 //   k0 = c_hi, k1 = c_lo, then per slot j:
 //     SPLIT:   k(2+2j) = 256 w_j, k(3+2j) = w_j   (digit = 256 hi + lo)
 //     !SPLIT:  k(2+j)  = w_j                      (digit exact in the format)
-//   bf16: chunk 1 holds the lo halves of the w_j columns (weights split hi+lo).
+// The table is fp16 for both paths (FMT = 0 here; the bf16 path switches to
+// bf16 operands from layer 2 on).
 // c = b1 + W1 x0 (Fig.-8 vector of the segment's v = 0 group), w_j = the
 // W1 column of slot j's ope at its Fig.-8 position.
 template <int FMT, bool SPLIT>
@@ -117,55 +118,6 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
             *reinterpret_cast<uint16_t*>(base + b_offset(n, k)) = v0;
             if (NCH > 1) *reinterpret_cast<uint16_t*>(base + kChunkBytesN32 + b_offset(n, k)) = v1;
         }
-    }
-}
-
-// issue the MMAs of one hidden layer (N = 32) or the output layer (N = 16)
-template <int FMT>
-__device__ __forceinline__ void issue_layer(uint32_t tD, uint32_t tA, uint32_t tC, uint32_t wbase,
-                                            uint32_t chunk_bytes, uint32_t idesc) {
-    if (FMT == 0) {
-        mma_ts(tD, tA, smem_desc(wbase + 0 * chunk_bytes), idesc, 0u);
-        mma_ts(tD, tA + 8, smem_desc(wbase + 1 * chunk_bytes), idesc, 1u);
-        mma_ts(tD, tC, smem_desc(wbase + 2 * chunk_bytes), idesc, 1u);
-    } else {
-        mma_ts(tD, tA, smem_desc(wbase + 0 * chunk_bytes), idesc, 0u);
-        mma_ts(tD, tA + 8, smem_desc(wbase + 1 * chunk_bytes), idesc, 1u);
-        mma_ts(tD, tA, smem_desc(wbase + 2 * chunk_bytes), idesc, 1u);
-        mma_ts(tD, tA + 8, smem_desc(wbase + 3 * chunk_bytes), idesc, 1u);
-        mma_ts(tD, tC, smem_desc(wbase + 4 * chunk_bytes), idesc, 1u);
-    }
-}
-
-template <int FMT>
-__device__ __forceinline__ void issue_layer_e(uint32_t tD, uint32_t tA, uint32_t tC, const uint64_t* d,
-                                              uint32_t idesc) {
-    if (FMT == 0) {
-        mma_ts_elect(tD, tA, d[0], idesc, 0u);
-        mma_ts_elect(tD, tA + 8, d[1], idesc, 1u);
-        mma_ts_elect(tD, tC, d[2], idesc, 1u);
-    } else {
-        mma_ts_elect(tD, tA, d[0], idesc, 0u);
-        mma_ts_elect(tD, tA + 8, d[1], idesc, 1u);
-        mma_ts_elect(tD, tA, d[2], idesc, 1u);
-        mma_ts_elect(tD, tA + 8, d[3], idesc, 1u);
-        mma_ts_elect(tD, tC, d[4], idesc, 1u);
-    }
-}
-
-template <int FMT>
-__device__ __forceinline__ void issue_layer_p(uint32_t pred, uint32_t tD, uint32_t tA, uint32_t tC,
-                                              const uint64_t* d, uint32_t idesc) {
-    if (FMT == 0) {
-        mma_ts_p(pred, tD, tA, d[0], idesc, 0u);
-        mma_ts_p(pred, tD, tA + 8, d[1], idesc, 1u);
-        mma_ts_p(pred, tD, tC, d[2], idesc, 1u);
-    } else {
-        mma_ts_p(pred, tD, tA, d[0], idesc, 0u);
-        mma_ts_p(pred, tD, tA + 8, d[1], idesc, 1u);
-        mma_ts_p(pred, tD, tA, d[2], idesc, 1u);
-        mma_ts_p(pred, tD, tA + 8, d[3], idesc, 1u);
-        mma_ts_p(pred, tD, tC, d[4], idesc, 1u);
     }
 }
 
@@ -279,7 +231,7 @@ struct TcPipe {
     bool outbias = false;
     float b4 = 0.0f;
     __device__ __forceinline__ void set_outbias(float bias) {
-        outbias = FMT == 0;
+        outbias = true;  // both formats: b4 in fp32 at the read of y, no output bias chunk
         b4 = bias;
     }
     __device__ __forceinline__ uint32_t add_b4(uint32_t ybits) const {
@@ -349,11 +301,13 @@ struct TcPipe {
         ph ^= 1u;
         fence_after();
     }
-    // layer-1 MMA(s) of one tile against its segment's B operand (no commit)
+    // layer-1 MMA of one tile against its segment's B operand (no commit).  Both
+    // formats: fp16 operands (the digits enter as the exact fp16 1024 + v, the
+    // segment table is fp16, fp32 accumulation); the bf16 path switches to bf16
+    // operands from layer 2 on (its layer-1 epilogue packs bf16)
     __device__ __forceinline__ void issue_l1(const TileIO& T, uint64_t db) const {
-        constexpr uint32_t id32 = idesc_f16(FMT, 32);
+        constexpr uint32_t id32 = idesc_f16(0, 32);
         mma_ts_elect(T.d, T.a1, db, id32, 0u);
-        if (TcCfg<FMT>::kNchL1 > 1) mma_ts_elect(T.d, T.a1, db + (kChunkBytesN32 >> 4), id32, 1u);
     }
     __device__ __forceinline__ void commit() const { mma_commit_elect(bar); }
     // layer LAYER (0: layer 2, 1: layer 3, 2: output) of X (and Y), one commit
@@ -365,26 +319,24 @@ struct TcPipe {
         // the output layer accumulate in fp32
         constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32, FMT != 0 || LAYER == 2);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
-        if (FMT == 0 && TWO) {
-            if (LAYER < 2 || outbias) {
-                issue_layer2_asm<0, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
-                return;
+        if (FMT == 1) {
+            // bf16 (DESIGN.md r2): layer 2 = hi weights + bias chunk (chunks 0, 1, 4),
+            // layer 3 = hi + lo weights + bias chunk (0..4), output = hi weights (0, 1),
+            // b4 added in fp32 when y is read
+            if (TWO) {
+                if (LAYER == 0) issue_layer2_asm<1, ID, CH, true, 4>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+                else if (LAYER == 1) issue_layer2x5_asm<ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+                else issue_layer2_asm<1, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+            } else {
+                if (LAYER == 0) issue_layer_asm<1, ID, CH, true, 4, false>(X.d, X.a, tCx, db, bar);
+                else if (LAYER == 1) issue_layer_asm<1, ID, CH, true, 4, true>(X.d, X.a, tCx, db, bar);
+                else issue_layer_asm<1, ID, CH, false, 2, false>(X.d, X.a, tCx, db, bar);
             }
-            issue_layer2_asm<0, ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
-        } else if (!TWO) {
-            if (FMT == 0 && (LAYER < 2 || outbias)) {
-                issue_layer_asm<FMT, ID, CH, false>(X.d, X.a, tCx, db, bar);
-                return;
-            }
-            issue_layer_asm<FMT, ID, CH>(X.d, X.a, tCx, db, bar);
-        } else {
-            uint64_t d[5];
-#pragma unroll
-            for (int i = 0; i < 5; i++) d[i] = db + (uint64_t)(i * (CH >> 4));
-            issue_layer_e<FMT>(X.d, X.a, tCx, d, ID);
-            issue_layer_e<FMT>(Y.d, Y.a, tCy, d, ID);
-            mma_commit_elect(bar);
+            return;
         }
+        // fp16: no bias MMA in any layer (hidden biases in the f16 epilogue, b4 in fp32)
+        if (TWO) issue_layer2_asm<0, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+        else issue_layer_asm<0, ID, CH, false>(X.d, X.a, tCx, db, bar);
     }
     // wait for the previous layer's MMAs, ReLU + pack into A, hand off, issue layer LAYER
     // CONST: also (re)write the per-tile constant chunks (layouts where the
@@ -547,7 +499,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_after();
     trace_stamp(P, 1);
     const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
-    build_b1_fused<FMT, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
+    build_b1_fused<0, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
                                blockDim.x);
     if (g == 0) {  // the constant chunk (1, 1, 0, ...) of the bias rows
         uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
@@ -579,7 +531,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     float best_y = __int_as_float(0x7fc00000);
     uint64_t wb, we;
     work_range(P.n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
-    if constexpr (FMT == 0 && !SPLIT) {
+    if constexpr (!SPLIT) {
         if (wb < we) {
 #ifdef EXP_STAGETRACE
             if (blockIdx.x == 0 && g == 0) pp.tr = P.trace;
@@ -714,11 +666,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
         // prologue: tile wb in slot X and (if the group has it) wb + 1 in slot Y
         const bool yLive = wb + 1 < we;  // warp-uniform
         take(vX, sX, okX, zX);
-        store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
+        store_a1<0, SPLIT>(pp.X.a1 + pp.lane_off, vX);
         if (yLive) {
             walker_next(P, W, wb + 1, r);
             take(vY, sY, okY, zY);
-            store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
+            store_a1<0, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
         }
         tmem_wait_st();
         if (pp.handoff(pp.me[3])) {
@@ -741,11 +693,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             if (w + 2 < we) {
                 walker_next(P, W, w + 2, r);
                 take(vX, sX, okX, zX);
-                store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
+                store_a1<0, SPLIT>(pp.X.a1 + pp.lane_off, vX);
                 if (NTWO) {
                     walker_next(P, W, w + 3, r);
                     take(vY, sY, okY, zY);
-                    store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
+                    store_a1<0, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
                 }
                 tmem_wait_st();
                 if (pp.handoff(pp.me[3])) {
@@ -886,7 +838,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             dec_pair0 = bd.pair0;
             dec_pair_end = d + 1 < n_dec ? decs[d + 1].pair0 : n_pairs;
             named_bar_sync(pp.bar_id, 128);
-            build_b1_fused<FMT, SPLIT>(P, s_w1, TP.l1_scale, my_b1, (int)r, 128);
+            build_b1_fused<0, SPLIT>(P, s_w1, TP.l1_scale, my_b1, (int)r, 128);
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             named_bar_sync(pp.bar_id, 128);
         };
@@ -902,7 +854,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             if ((tid & 31) == 0 && best) acc_fold(&acc[d], best, best_y);
             best = 0;
         };
-        if constexpr (FMT == 0 && !SPLIT) {
+        if constexpr (!SPLIT) {
             // packed walker + three-instruction fold (as fused_tc_kernel)
             PackedWalker W{};
             uint32_t x1 = 0, x2 = 0, xs = 0, y1 = 0, y2 = 0, ys = 0, bsn = 1u;
@@ -973,10 +925,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             if (fresh) walker_begin(P, W, lt, r);
             else walker_next(P, W, lt, r);
             take(vX, sX, okX, zX);
-            store_a1<FMT, SPLIT>(pp.X.a1 + pp.lane_off, vX);
+            store_a1<0, SPLIT>(pp.X.a1 + pp.lane_off, vX);
             walker_next(P, W, lt + 1, r);
             take(vY, sY, okY, zY);
-            store_a1<FMT, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
+            store_a1<0, SPLIT>(pp.Y.a1 + pp.lane_off, vY);
             tmem_wait_st();
             if (pp.handoff(pp.me[3])) {
                 issue_l1(pp.X, sX);
@@ -1392,13 +1344,14 @@ __device__ __forceinline__ float predict_row_fp32(const W234& W, const float* __
     return acc;
 }
 
-template <int NG>
+// FMT 1 (bf16): the same fp16 layer-1 operand and table; layers 2, 3 and the
+// output in bf16 (TcPipe<1>), as in the fused bf16 search.
+template <int FMT, int NG>
 __global__ void __launch_bounds__(NG * 128, 1) predict24_tc_kernel(const __grid_constant__ TcParams TP,
                                                                    const __grid_constant__ W234 W,
                                                                    const float* __restrict__ w1b1,
                                                                    const int16_t* __restrict__ x, uint64_t count,
                                                                    float* __restrict__ y) {
-    constexpr int FMT = 0;
     extern __shared__ __align__(1024) uint8_t smem[];
     // stages: per group X0 X1 Y0 Y1 (4 x 6 KB); TMA mbarriers after the TMEM slot
     const TcSmem L = tc_smem_layout<FMT>(2, kChunkBytesN32, NG, 4 * kStage24);
@@ -1457,11 +1410,11 @@ __global__ void __launch_bounds__(NG * 128, 1) predict24_tc_kernel(const __grid_
         bad = (o & 0xFC00FC00u) != 0u ? 1u : 0u;  // a feature < 0 or >= 1024: recomputed in fp32
 #pragma unroll
         for (int i = 0; i < 12; i++) a[i] |= 0x64006400u;
-        a[12] = TcCfg<FMT>::kOne2;
+        a[12] = TcCfg<0>::kOne2;  // fp16 (1, 1): the layer-1 operand is fp16 in both formats
         a[13] = a[14] = a[15] = 0u;
     };
     auto issue_l1 = [&](const TileIO& T) {
-        constexpr uint32_t id32 = idesc_f16(FMT, 32);
+        constexpr uint32_t id32 = idesc_f16(0, 32);
         mma_ts_elect(T.d, T.a1, d1, id32, 0u);
         mma_ts_elect(T.d, T.a1 + 8, d1 + (kChunkBytesN32 >> 4), id32, 1u);
     };
@@ -1579,8 +1532,9 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
     return cudaGetLastError();
 }
 
-// digits are < cnt: unsplit when exact -- fp16 1024 + v up to v = 1024, bf16 v up to 256
-static bool need_split(int fmt, uint32_t maxcnt) { return fmt == 0 ? maxcnt > 1025 : maxcnt > 257; }
+// digits are < cnt: unsplit when exact as the fp16 1024 + v (v up to 1024); both
+// formats enter layer 1 through the same fp16 digit operand
+static bool need_split(int, uint32_t maxcnt) { return maxcnt > 1025; }
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
                             cudaStream_t st, int* grid_out) {
@@ -1655,11 +1609,12 @@ cudaError_t launch_predict_tc(const TcWeights& TW, const W234& W, const float* w
     if (count == 0) return cudaSuccess;
     if (D > 31) return cudaErrorInvalidValue;  // layer-1 operand: 4 K-chunks = the 32-column U region
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
-    if (TW.fmt == 0 && D == 24 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0) {
+    if (D == 24 && (reinterpret_cast<uintptr_t>(x) & 15u) == 0) {
         constexpr int NG = kPred24NG;
-        const TcSmem L = tc_smem_layout<0>(2, kChunkBytesN32, NG, 4 * kStage24);
+        const TcSmem L = TW.fmt == 0 ? tc_smem_layout<0>(2, kChunkBytesN32, NG, 4 * kStage24)
+                                     : tc_smem_layout<1>(2, kChunkBytesN32, NG, 4 * kStage24);
         const uint32_t total = L.total + 8u * 4u * NG;  // + TMA mbarriers
-        auto kern = predict24_tc_kernel<NG>;
+        auto kern = TW.fmt == 0 ? predict24_tc_kernel<0, NG> : predict24_tc_kernel<1, NG>;
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)total);
         if (e != cudaSuccess) return e;
         const uint64_t n_tiles = (count + kTileM - 1) / kTileM;

@@ -153,11 +153,12 @@ __device__ __forceinline__ void mma_commit_elect(uint64_t* bar) {
 // immediate, one elected lane issues the MMAs and the commit.
 //   FMT 0 (fp16):  D  = A[0:8) W_c0 + A[8:16) W_c1 + C bias
 //   FMT 1 (bf16):  D  = A[0:8) Whi_c0 + A[8:16) Whi_c1 + A[0:8) Wlo_c0 + A[8:16) Wlo_c1 + C bias
-template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
+// LO (bf16 only): also the lo chunks 2, 3; the bias chunk is then 4, else BCH.
+template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true, uint32_t BCH = 2, bool LO = (FMT == 1)>
 __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32_t tC, uint64_t dbase,
                                                 uint64_t* bar) {
     constexpr uint32_t U = CHUNK >> 4;
-    if (FMT == 0 && !BIAS) {  // the two data chunks only (the bias is added outside)
+    if (!LO && !BIAS) {  // the two data chunks only (the bias is added outside)
         asm volatile(
             "{\n\t"
             ".reg .pred e, pf, pt;\n\t"
@@ -176,7 +177,31 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
             : "memory");
         return;
     }
-    if (FMT == 0) {
+    if (LO && !BIAS) {  // hi + lo weight chunks, no bias
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1, d2, d3;\n\t"
+            ".reg .b32 a8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %2, %4;\n\t"
+            "add.s64 d2, %2, %5;\n\t"
+            "add.s64 d3, %2, %6;\n\t"
+            "add.u32 a8, %1, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %7, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d1, %7, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %7, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d3, %7, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%3];\n\t"
+            "}" ::"r"(tD),
+            "r"(tA), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(2 * U)),
+            "n"((uint64_t)(3 * U)), "n"(IDESC)
+            : "memory");
+        return;
+    }
+    if (!LO) {
         asm volatile(
             "{\n\t"
             ".reg .pred e, pf, pt;\n\t"
@@ -193,7 +218,7 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
             "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], d2, %7, pt;\n\t"
             "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%4];\n\t"
             "}" ::"r"(tD),
-            "r"(tA), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(2 * U)),
+            "r"(tA), "r"(tC), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(BCH * U)),
             "n"(IDESC)
             : "memory");
     } else {
@@ -223,11 +248,14 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
     }
 }
 
-// the MMAs of one layer for TWO tiles (same B operand) and ONE commit
-template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
+// the MMAs of one layer for TWO tiles (same B operand) and ONE commit:
+// chunks 0, 1 (the two K halves of the weights) and, with BIAS, the bias chunk
+// BCH against the constant chunk (fp16 blob: BCH = 2; bf16 blob: BCH = 4, the
+// lo chunks 2, 3 skipped -- layer 2 of the bf16 path runs hi weights only).
+// IDESC carries the operand format (f16 or bf16).
+template <int FMT, uint32_t IDESC, uint32_t CHUNK, bool BIAS = true, uint32_t BCH = 2>
 __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
                                                  uint32_t tCx, uint32_t tCy, uint64_t dbase, uint64_t* bar) {
-    static_assert(FMT == 0, "lock-step pair issue: fp16 layout");
     constexpr uint32_t U = CHUNK >> 4;
     if (!BIAS) {  // the two data chunks only (the bias is added outside)
         asm volatile(
@@ -272,7 +300,73 @@ __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uin
         "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t"
         "}" ::"r"(tDx),
         "r"(tAx), "r"(tDy), "r"(tAy), "r"(tCx), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
-        "n"((uint64_t)(2 * U)), "n"(IDESC), "r"(tCy)
+        "n"((uint64_t)(BCH * U)), "n"(IDESC), "r"(tCy)
+        : "memory");
+}
+
+// bf16 layer for TWO tiles: hi chunks 0, 1, lo chunks 2, 3 (W = W_hi + W_lo)
+// and (BIAS) the bias chunk 4, one commit
+template <uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
+__device__ __forceinline__ void issue_layer2x5_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
+                                                   uint32_t tCx, uint32_t tCy, uint64_t dbase, uint64_t* bar) {
+    constexpr uint32_t U = CHUNK >> 4;
+    if (!BIAS) {
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d1, d2, d3;\n\t"
+            ".reg .b32 ax8, ay8;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d1, %4, %6;\n\t"
+            "add.s64 d2, %4, %7;\n\t"
+            "add.s64 d3, %4, %8;\n\t"
+            "add.u32 ax8, %1, 8;\n\t"
+            "add.u32 ay8, %3, 8;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %4, %9, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d1, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d3, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %4, %9, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], d2, %9, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d3, %9, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%5];\n\t"
+            "}" ::"r"(tDx),
+            "r"(tAx), "r"(tDy), "r"(tAy), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
+            "n"((uint64_t)(2 * U)), "n"((uint64_t)(3 * U)), "n"(IDESC)
+            : "memory");
+        return;
+    }
+    asm volatile(
+        "{\n\t"
+        ".reg .pred e, pf, pt;\n\t"
+        ".reg .b64 d1, d2, d3, d4;\n\t"
+        ".reg .b32 ax8, ay8;\n\t"
+        "setp.ne.b32 pf, 0, 0;\n\t"
+        "setp.eq.b32 pt, 0, 0;\n\t"
+        "add.s64 d1, %5, %7;\n\t"
+        "add.s64 d2, %5, %8;\n\t"
+        "add.s64 d3, %5, %9;\n\t"
+        "add.s64 d4, %5, %10;\n\t"
+        "add.u32 ax8, %1, 8;\n\t"
+        "add.u32 ay8, %3, 8;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %5, %11, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d1, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d3, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%4], d4, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %5, %11, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], d2, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d3, %11, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%12], d4, %11, pt;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%6];\n\t"
+        "}" ::"r"(tDx),
+        "r"(tAx), "r"(tDy), "r"(tAy), "r"(tCx), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
+        "n"((uint64_t)(2 * U)), "n"((uint64_t)(3 * U)), "n"((uint64_t)(4 * U)), "n"(IDESC), "r"(tCy)
         : "memory");
 }
 

@@ -59,6 +59,7 @@ def timed(fn):
     return min(ms)
 
 
+FLOP_PER_ROW = 2 * (synth.D * 32 + 32 * 32 + 32 * 32 + 32)  # 5,696 (D = 24)
 res = {"rows": n, "hbm_peak_gbs": HBM, "peak_source": "MEASURED_PEAKS.json hbm_gbs"}
 ms = timed(lambda: ab.abacus_encode_candidates(ctx, grid, first, n, X, st))
 gb = n * synth.D * 2 / (ms * 1e-3) / 1e9
@@ -71,6 +72,12 @@ for name, prec in (("predict_fp32", ab.ABACUS_FP32), ("predict_fp16", ab.ABACUS_
     gb = n * (synth.D * 2 + 4) / (ms * 1e-3) / 1e9
     res[name] = {"ms": ms, "GB_per_s": gb, "frac": gb / HBM, "bytes_per_unit": synth.D * 2 + 4,
                  "units_per_s": n / (ms * 1e-3)}
+    if prec == ab.ABACUS_FP32:
+        # FP32 SIMT bound: 5,696 algorithmic FLOP per row against 148 SMs x 128 FFMA x 2 x 1965 MHz
+        fma_peak = 148 * 128 * 2 * 1965e6 / 1e12
+        tf = n * FLOP_PER_ROW / (ms * 1e-3) / 1e12
+        res[name].update({"bound": "alu", "TFLOP_per_s": tf, "alu_peak_tflops": fma_peak,
+                          "alu_frac": tf / fma_peak, "flop_per_unit": FLOP_PER_ROW})
 H = synth.cfg4_headroom()
 ms = timed(lambda: ab.abacus_select_group(ctx, grid, first, n, y, H, best, st))
 gb = n * 4 / (ms * 1e-3) / 1e9
