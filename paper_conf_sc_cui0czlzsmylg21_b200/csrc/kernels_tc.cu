@@ -24,6 +24,7 @@
 #include <cuda_runtime.h>
 #include <math.h>
 
+#include <cstdlib>
 #include <type_traits>
 
 #include "common.cuh"
@@ -317,7 +318,7 @@ struct TcPipe {
         // fp16: hidden layers 2 and 3 accumulate in f16 (their epilogues then read
         // half the TMEM bytes); layer 1 (the 1024 + v digits cancel there) and
         // the output layer accumulate in fp32
-        constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 16 : 32, FMT != 0 || LAYER == 2);
+        constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 8 : 32, FMT != 0 || LAYER == 2);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 1) {
             // bf16 (DESIGN.md r2): layer 2 = hi weights + bias chunk (chunks 0, 1, 4),
@@ -349,6 +350,17 @@ struct TcPipe {
     // constant in the fused kernel's role-specialised loop)
     template <int LAYER, bool TWO, bool CONST = false>
     __device__ __forceinline__ void stage_as(bool mine) {
+        epilogue<LAYER, TWO, CONST>();
+        tmem_wait_st();
+        stamp(LAYER, 1);
+        if (handoff(mine)) {
+            stamp(LAYER, 2);
+            issue_next<LAYER, TWO>();
+        }
+    }
+    // wait for the previous layer's MMAs, ReLU + pack into A (no st wait)
+    template <int LAYER, bool TWO, bool CONST = false>
+    __device__ __forceinline__ void epilogue() {
         uint32_t hbw[16];
         // layer 3's bias words sit one hidden-layer blob (kNchHid chunks) after layer 2's
         if (FMT == 0 && LAYER >= 1)
@@ -392,12 +404,6 @@ struct TcPipe {
             uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
             tmem_st8(tCx + lane_off, c8);
             if (TWO) tmem_st8(tCy + lane_off, c8);
-        }
-        tmem_wait_st();
-        stamp(LAYER, 1);
-        if (handoff(mine)) {
-            stamp(LAYER, 2);
-            issue_next<LAYER, TWO>();
         }
     }
     // the same with fixed issuer roles: stage p issued by warp wq == p of the group

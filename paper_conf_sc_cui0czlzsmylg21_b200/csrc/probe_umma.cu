@@ -10,6 +10,8 @@
 // variant 3: as 0, and the same A/B issued twice with accumulate (D = 2 A B^T)
 // variant 4: as 0 with an f16 accumulator (idesc c_format = F16); raw D words
 // variant 5: as 4, issued twice with accumulate
+// variant 6: as 0 with D columns [0, 32) pre-filled with a sentinel: an N < 32
+//            MMA must leave columns [N, 32) untouched (N = 8 at M = 128)
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -48,6 +50,12 @@ __global__ void probe_kernel(int fmt, int variant, int N, const uint32_t* __rest
     uint32_t a[8];
     for (int c = 0; c < 8; c++) a[c] = a_words[tid * 8 + c];
     tmem_st8(tb + acol + lane_off, a);
+    if (variant == 6) {
+        uint32_t z[16];
+        for (int c = 0; c < 16; c++) z[c] = __float_as_uint(-777.0f);
+        tmem_st16(tb + lane_off, z);
+        tmem_st16(tb + 16 + lane_off, z);
+    }
     tmem_wait_st();
     fence_before();
     __syncthreads();
@@ -56,7 +64,7 @@ __global__ void probe_kernel(int fmt, int variant, int N, const uint32_t* __rest
         const uint32_t saddr = smem_u32(sb);
         const uint64_t desc = variant == 1 ? smem_desc(saddr, 256, 128) : smem_desc(saddr, 128, 256);
         uint32_t id = idesc_f16(fmt, N);
-        if (variant >= 4) id &= ~(3u << 4);  // D format F16
+        if (variant == 4 || variant == 5) id &= ~(3u << 4);  // D format F16
         mma_ts(tb, tb + acol, desc, id, 0u);
         if (variant == 3 || variant == 5) mma_ts(tb, tb + acol, desc, id, 1u);
         mma_commit(&bar);
@@ -65,7 +73,8 @@ __global__ void probe_kernel(int fmt, int variant, int N, const uint32_t* __rest
     fence_after();
     uint32_t r[32];
     tmem_ld32(tb + lane_off, r);
-    for (int n = 0; n < N; n++) d_out[tid * N + n] = __uint_as_float(r[n]);
+    const int nout = variant == 6 ? 32 : N;
+    for (int n = 0; n < nout; n++) d_out[tid * nout + n] = __uint_as_float(r[n]);
     fence_before();
     __syncthreads();
     fence_after();
@@ -80,12 +89,13 @@ extern "C" int abacus_probe_mma(int fmt, int variant, int N, const uint32_t* a_w
     cudaError_t e = cudaSuccess;
     if ((e = cudaMalloc(&da, 128 * 8 * 4)) != cudaSuccess) return (int)e;
     if ((e = cudaMalloc(&db, N * 16 * 2)) != cudaSuccess) return (int)e;
-    if ((e = cudaMalloc(&dd, 128 * N * 4)) != cudaSuccess) return (int)e;
+    const int nout = variant == 6 ? 32 : N;
+    if ((e = cudaMalloc(&dd, 128 * nout * 4)) != cudaSuccess) return (int)e;
     cudaMemcpy(da, a_words_host, 128 * 8 * 4, cudaMemcpyHostToDevice);
     cudaMemcpy(db, b_host, N * 16 * 2, cudaMemcpyHostToDevice);
     probe_kernel<<<1, 128>>>(fmt, variant, N, da, db, dd);
     e = cudaDeviceSynchronize();
-    if (e == cudaSuccess) e = cudaMemcpy(d_host, dd, 128 * N * 4, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(d_host, dd, 128 * nout * 4, cudaMemcpyDeviceToHost);
     cudaFree(da);
     cudaFree(db);
     cudaFree(dd);

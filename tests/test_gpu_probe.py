@@ -46,3 +46,22 @@ def test_umma_layouts(fmt, N):
     assert np.array_equal(res[0], want), "descriptor (LBO=128 K-dir, SBO=256 N-dir) / A packing"
     assert np.array_equal(res[2], want), "A at a TMEM column offset of 8"
     assert np.array_equal(res[3], 2 * want), "accumulate flag"
+
+
+@pytest.mark.parametrize("fmt", [0, 1])
+def test_umma_m128_n8(fmt):
+    """M = 128 with N = 8 (the output layer's width): the MMA computes the 8
+    columns and leaves the rest of the 32-column D region untouched."""
+    L = _lib()
+    rng = np.random.default_rng(5 + fmt)
+    N = 8
+    A = rng.integers(-3, 4, size=(128, 16)).astype(np.float32)
+    B = rng.integers(-2, 3, size=(N, 16)).astype(np.float32)
+    ab = _bits(A, fmt).astype(np.uint32)
+    words = np.ascontiguousarray((ab[:, 1::2] << 16) | ab[:, 0::2], dtype=np.uint32)
+    bb = np.ascontiguousarray(_bits(B, fmt))
+    out = np.zeros((128, 32), dtype=np.float32)
+    rc = L.abacus_probe_mma(fmt, 6, N, words.ctypes.data, bb.ctypes.data, out.ctypes.data)
+    assert rc == 0
+    assert np.array_equal(out[:, :8], A @ B.T)
+    assert np.all(out[:, 8:] == -777.0)
