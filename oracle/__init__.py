@@ -241,6 +241,35 @@ def sweep(params, grid, H, first=0, count=None, eps=1e-4, n_models=8, kmax=4, em
     return r, y, x, o
 
 
+def whatif(params, grid, variants, H, eps=1e-4, n_models=8, kmax=4):
+    """What-if sweep (SURVEY §8(f) NEXT-4: bs / seqlen as swept grid dimensions;
+    the batch size is chosen by the load balancer at run time and inputs differ
+    in length).  ``variants`` is a list of (batch per slot, seqlen
+    per slot); variant v replaces the grid slots' bs and seqlen (Fig.-8
+    features) and its candidates take the indices
+    v * T + t (variant the most significant digit, T = |grid|).  The selection
+    rule is the grid's (max sum_n, then max index, reading c12) over all
+    variants: among groups of equal size the later variant wins.
+    Returns (per-variant SweepResults, (best key over all variants, its
+    variant or -1, its grid index t), (maxkey_strict, maxkey_loose) with the
+    per-variant acceptance keys lifted to global indices)."""
+    T = grid_size(grid)
+    per = []
+    best = (0, -1, 0)
+    strict = loose = 0
+    for v, (bss, sls) in enumerate(variants):
+        g = [type(s)(s.model_id, s.start_op, int(bss[j]), int(sls[j]), s.end_lo, s.end_hi, s.allow_absent)
+             for j, s in enumerate(grid)]
+        r, _, _, _ = sweep(params, g, H, eps=eps, n_models=n_models, kmax=kmax)
+        per.append(r)
+        lift = lambda key: ((key >> 40) << 40) | (v * T + (key & ((1 << 40) - 1))) if key else 0  # noqa: E731
+        if r.best_key and lift(r.best_key) > best[0]:
+            best = (lift(r.best_key), v, r.best_index)
+        strict = max(strict, lift(r.maxkey_strict))
+        loose = max(loose, lift(r.maxkey_loose))
+    return per, best, (strict, loose)
+
+
 def sweep_shell(params, grid, H, nsum_min, eps=1e-4, n_models=8, kmax=4, emu_flags=0):
     """The whole grid restricted to candidates with sum_n >= nsum_min (orc_sweep_shell)."""
     p, pp = _f32(params)

@@ -446,3 +446,57 @@ def test_bf16_emulation_against_torch_rounding():
     d = np.abs(ye - y) / np.abs(y)
     assert np.quantile(d, 0.99) <= 1e-12   # same roundings
     assert d.max() <= 2 ** -7              # a rare tie flipped by fp64 summation order moves one activation by 1 ulp
+
+
+# ------------------------------------------ NEXT-4: bs / seqlen as swept dims ----
+def test_whatif_vs_bruteforce_exact():
+    """The what-if sweep (bs and seqlen per slot as an outer variant digit,
+    P:513-520) against brute force: itertools over (variant, end ops), the
+    brute Fig.-8 encoder with the variant's bs / seqlen, exact rational MLP,
+    direct scan for max (sum_n, v T + t) under H."""
+    rng = np.random.default_rng(41)
+    p = synth.raw_weights(4)
+    for trial in range(6):
+        grid = synth.tiny_grids(1, seed=300 + trial, max_len=4)[0]
+        k = len(grid)
+        nv = int(rng.integers(1, 4))
+        variants = [([int(rng.integers(1, 33)) for _ in range(k)],
+                     [int(rng.choice([0, 16, 128, 512])) for _ in range(k)]) for _ in range(nv)]
+        T = oracle.grid_size(grid)
+        cands = brute.enumerate_grid(grid)
+        ys, meta = [], []
+        for v, (bss, sls) in enumerate(variants):
+            for t, opes in enumerate(cands):
+                pres = [(s.model_id, s.start_op, e, bss[j], sls[j]) for j, (s, e) in enumerate(zip(grid, opes)) if e]
+                ys.append(brute.mlp_exact(p, brute.encode(8, 4, pres), synth.D))
+                meta.append((v, t, brute.sum_n(grid, opes)))
+        sy = sorted(ys)
+        m = len(sy) // 2
+        H = Fraction(float((sy[m] + (sy[m + 1] if m + 1 < len(sy) else sy[m] + 1)) / 2))  # between values: no tie
+        best = (-1, -1, -1)
+        for (v, t, sn), y in zip(meta, ys):
+            if y <= H and (sn, v * T + t) > (best[2], best[0] * T + best[1] if best[0] >= 0 else -1):
+                best = (v, t, sn)
+        per, (key, bv, bt), _ = oracle.whatif(p, grid, variants, float(H))
+        assert (bv, bt) == best[:2], (trial, (bv, bt), best)
+        assert key == ((best[2] + 1) << 40) | (best[0] * T + best[1])
+        for v in range(nv):  # per variant: the plain grid scan of that variant
+            yv = ys[v * T:(v + 1) * T]
+            tv, sv = brute.best_by_scan(cands, grid, yv, H)
+            assert (per[v].best_index if per[v].best_key else -1) == tv
+
+
+def test_whatif_larger_batch_never_fits_more_under_monotone_predictor():
+    """With a predictor increasing in every slot's bs (linear, non-negative
+    coefficients, ReLU-transparent), the largest fitting group of a variant can
+    only shrink as the batch sizes grow."""
+    lp = LinearPredictor(8, 4, c0=2.0, beta=[0.5] * 8, a=[0.25, 0.125, 0.5, 0.75])
+    p = lp.params()
+    o = offsets(synth.D)
+    for q in range(4):  # bs coefficient of slot position q
+        p[o["W1"] + 0 * synth.D + 8 + 4 * q + 2] = 0.0625
+    grid = [synth.GridSlot(1, 1, 1, 0, 1, 60, 1), synth.GridSlot(5, 1, 1, 0, 1, 40, 1)]
+    variants = [([b, b], [0, 0]) for b in (1, 2, 4, 8, 16, 32)]
+    per, _, _ = oracle.whatif(p, grid, variants, 20.0)
+    sns = [(r.best_key >> 40) if r.best_key else 0 for r in per]
+    assert all(a >= b for a, b in zip(sns, sns[1:])) and sns[0] > sns[-1], sns
