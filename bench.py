@@ -296,7 +296,9 @@ def main():
 
     # ---- the other arithmetic paths on the same sweep (secondary keys) ------
     secondary = None
+    whatif = None
     if world == 1 and not args.no_secondary:
+        whatif = whatif_sweep(ab, ctx, slots, H, T)
         secondary = secondary_paths(ab, ctx, params, grid, H, T, args.precision, stream)
 
     if rank == 0:
@@ -344,6 +346,7 @@ def main():
             "decision_latency": dec,
             "decision_latency_sharded": sharded,
             "secondary_paths": secondary,
+            "whatif": whatif,
         }
         print(json.dumps(line))
     if comm:
@@ -395,6 +398,25 @@ def secondary_paths(ab, ctx, params, grid, H, T, headline, stream, steps=(("bf16
     ab.abacus_load_predictor(ctx, params, PREC[headline])
     torch.cuda.synchronize()
     return out
+
+
+def whatif_sweep(ab, ctx, slots, H, T, reps=3):
+    """NEXT-4 what-if sweep on the config-4 grid: BERT-large's batch size
+    swept over {1, 2, 4, 8} (4 x 9.19e9 candidates in one batched launch,
+    abacus_search_whatif).  Device time of the launch (CUDA events)."""
+    variants = [([8, 8, 8, b], [0, 0, 128, 512]) for b in (1, 2, 4, 8)]
+    g = ab.make_grid(slots)
+    ab.abacus_search_whatif(ctx, g, variants, H)  # warm-up (grows the buffers)
+    kms = []
+    for _ in range(reps):
+        per, best, bv = ab.abacus_search_whatif(ctx, g, variants, H)
+        kms.append(ab.abacus_last_kernel_ms(ctx))
+    k = float(np.mean(kms))
+    n = T * len(variants)
+    return {"grid": "config 4, BERT-large bs in {1, 2, 4, 8}", "variants": len(variants), "candidates": n,
+            "kernel_ms": k, "candidates_per_s": n / (k / 1e3), "best_variant": bv, "best_key": best.key,
+            "per_variant_total_ops": [d.total_ops for d in per],
+            "path": "abacus_search_whatif: one fused_batch_tc_kernel launch (4 plans) + finalize"}
 
 
 def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50):

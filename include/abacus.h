@@ -122,6 +122,14 @@ typedef struct {
     } slot[ABACUS_K_MAX];            /* any order; encoded by model id       */
 } abacus_group_t;
 
+/* One what-if variant of a grid (abacus_search_whatif): the batch size and
+ * sequence length of every grid slot (slot j uses batch[j], seqlen[j]; the
+ * grid's own values are replaced). */
+typedef struct {
+    int32_t batch[ABACUS_K_MAX];  /* >= 1 */
+    int32_t seqlen[ABACUS_K_MAX]; /* >= 0 (0 for non-Bert models, reading c8) */
+} abacus_variant_t;
+
 /* One active query (Fig. 4, Eq. 2). */
 typedef struct {
     int32_t model_id; /* 1..N                                  */
@@ -300,6 +308,29 @@ int abacus_search_mway(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, doub
  * E_DUP_MODEL, E_NOT_LOADED, E_CUDA, E_NCCL. */
 int abacus_search_grid(abacus_ctx* ctx, const abacus_grid_t* grid, float headroom_ms, uint64_t first,
                        uint64_t count, void* nccl_comm, abacus_decision_t* out);
+
+/* What-if sweep (batch size and sequence length as
+ * swept grid dimensions; the paper: "the batch size of query processing is
+ * determined by the upper-level load balancer at runtime" and inputs vary in
+ * length).  The candidates are every (variant v, end-op candidate
+ * t) with v in [0, n_var), t in [0, T) of `grid` (host) whose slots take
+ * variant v's batch sizes and sequence lengths (Fig.-8 features);
+ * their index is v * T + t (the variant is the most significant digit, so
+ * among groups of equal size the later variant wins, reading c12).
+ * per_variant (host, n_var, may be NULL): variant v's own sweep decision,
+ * exactly abacus_search_grid(variant grid v, headroom_ms, 0, T, NULL).
+ * best (host, may be NULL): the largest feasible group over all variants --
+ * key ((sum_n + 1) << 40) | (v T + t), index v T + t, end_op / pred_ms /
+ * total_ops of that candidate, evaluated n_var T, pred_critical_only_ms =
+ * y(index 0) of variant 0; status OK or NONE.  *best_variant (may be NULL)
+ * = its v, -1 if nothing fits.  1 <= n_var <= ABACUS_BATCH_MAX and
+ * n_var T < 2^40.  Tensor precisions: one batched launch for all variants
+ * (each variant a plan of the NEXT-4 batch kernel); fp32: one fused launch
+ * per variant.  Blocking.  Errors: as abacus_search_grid, plus E_INVALID for
+ * a variant's batch outside [1, 32767] or seqlen outside [0, 32767]. */
+int abacus_search_whatif(abacus_ctx* ctx, const abacus_grid_t* grid, const abacus_variant_t* variants,
+                         int32_t n_var, float headroom_ms, abacus_decision_t* per_variant,
+                         abacus_decision_t* best, int32_t* best_variant);
 
 /* Per-decision sharded search (the paper's search is
  * single-node): the decision of abacus_search(q, k, now_ms,

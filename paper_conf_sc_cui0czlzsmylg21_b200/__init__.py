@@ -29,7 +29,7 @@ K_MAX = 4
 
 EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load_predictor",
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
-            "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_search_sharded",
+            "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_search_sharded", "abacus_search_whatif",
             "abacus_combine_decisions", "abacus_nccl_unique_id",
             "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
             "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version",
@@ -57,6 +57,10 @@ class _gslot(C.Structure):
 
 class abacus_group_t(C.Structure):
     _fields_ = [("k", C.c_int32), ("slot", _gslot * K_MAX)]
+
+
+class abacus_variant_t(C.Structure):
+    _fields_ = [("batch", C.c_int32 * K_MAX), ("seqlen", C.c_int32 * K_MAX)]
 
 
 class abacus_query_t(C.Structure):
@@ -110,6 +114,8 @@ def lib():
                                          P(abacus_decision_t)]
         L.abacus_search_sharded.argtypes = [vp, P(abacus_query_t), C.c_int32, C.c_double, C.c_double, C.c_int32,
                                             C.c_uint64, vp, P(abacus_decision_t)]
+        L.abacus_search_whatif.argtypes = [vp, P(abacus_grid_t), P(abacus_variant_t), C.c_int32, C.c_float,
+                                           P(abacus_decision_t), P(abacus_decision_t), P(C.c_int32)]
         L.abacus_combine_decisions.argtypes = [P(abacus_decision_t), C.c_int32, C.c_int32, P(abacus_decision_t)]
         L.abacus_nccl_unique_id.argtypes = [P(C.c_uint8)]
         L.abacus_nccl_comm_init.argtypes = [vp, C.c_int32, C.c_int32, P(C.c_uint8), P(vp)]
@@ -271,6 +277,23 @@ def abacus_search_sharded(ctx, queries, now_ms: float, inflight_pred_ms: float, 
     _check(ctx, lib().abacus_search_sharded(ctx, qa, k, float(now_ms), float(inflight_pred_ms), space, grid_budget,
                                             nccl_comm, C.byref(out)))
     return out
+
+
+def abacus_search_whatif(ctx, grid: abacus_grid_t, variants, headroom_ms: float):
+    """variants: sequence of (batch per slot, seqlen per slot).  Returns
+    (per-variant decisions, best decision, best variant index or -1)."""
+    n = len(variants)
+    va = (abacus_variant_t * max(n, 1))()
+    for i, (bs, sl) in enumerate(variants):
+        for j in range(min(len(bs), K_MAX)):
+            va[i].batch[j] = int(bs[j])
+            va[i].seqlen[j] = int(sl[j])
+    per = (abacus_decision_t * max(n, 1))()
+    best = abacus_decision_t()
+    bv = C.c_int32()
+    _check(ctx, lib().abacus_search_whatif(ctx, C.byref(grid), va, n, float(headroom_ms), per, C.byref(best),
+                                           C.byref(bv)))
+    return list(per)[:n], best, int(bv.value)
 
 
 def abacus_combine_decisions(per_rank: Sequence[abacus_decision_t], drop_test: bool = False) -> abacus_decision_t:

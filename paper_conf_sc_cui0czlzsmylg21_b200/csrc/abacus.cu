@@ -83,6 +83,11 @@ struct abacus_ctx {
     BatchA1* d_a1 = nullptr;
     int32_t* d_L = nullptr;        // device copy of the registry's op counts
     uint64_t* d_pairs = nullptr;   // [n] tile pairs per decision, then [n] = total
+    // what-if sweeps (NEXT-4): host-planned grid plans of up to kMaxSeg segments
+    int32_t whatif_cap = 0;
+    BatchDec* h_wdecs = nullptr;   // pinned
+    SegP* h_wsegs = nullptr;       // pinned, kMaxSeg per variant
+    SegP* d_wsegs = nullptr;
     // NEXT-3 training state (abacus_train_begin)
     bool training = false;
     abacus_adam_t adam{};
@@ -898,6 +903,23 @@ int combine_over_comm(abacus_ctx* c, void* comm, uint32_t seq) {
     return ABACUS_OK;
 }
 
+// a sweep's decision from its result record (status OK / NONE, no drop test)
+abacus_decision_t sweep_decision(const Result& R, int32_t k, float H) {
+    abacus_decision_t d{};
+    d.critical = 0;
+    for (int j = 0; j < 4; j++) d.order[j] = j < k ? j : -1;
+    d.headroom_ms = H;
+    d.pred_critical_only_ms = R.y0;
+    d.evaluated = R.evaluated;
+    d.key = R.key;
+    d.index = R.key & ((1ull << 40) - 1);
+    d.status = R.key ? ABACUS_DECIDE_OK : ABACUS_DECIDE_NONE;
+    d.pred_ms = R.key ? R.y_best : NAN;
+    d.total_ops = R.key ? R.total_ops : 0;
+    for (int j = 0; j < k; j++) d.end_op[j] = R.key ? R.end_op[j] : 0;
+    return d;
+}
+
 abacus_decision_t assemble_decision(const Result& R, const int32_t* order, int32_t k, float H, uint64_t n_eval) {
     abacus_decision_t d{};
     d.critical = order[0];
@@ -987,6 +1009,9 @@ void abacus_destroy(abacus_ctx* c) {
     cudaFree(c->d_a1);
     cudaFree(c->d_L);
     cudaFree(c->d_pairs);
+    if (c->h_wdecs) cudaFreeHost(c->h_wdecs);
+    if (c->h_wsegs) cudaFreeHost(c->h_wsegs);
+    cudaFree(c->d_wsegs);
     cudaFree(c->t_p);
     cudaFree(c->t_m);
     cudaFree(c->t_v);
@@ -1354,19 +1379,7 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     rc = wait_result(c, seq, &R);
     if (rc) return rc;
     if (!nccl_comm) host_decode(P, R);
-    abacus_decision_t d{};
-    d.critical = 0;
-    for (int j = 0; j < 4; j++) d.order[j] = j < grid->k ? j : -1;
-    d.headroom_ms = headroom_ms;
-    d.pred_critical_only_ms = R.y0;
-    d.evaluated = R.evaluated;
-    d.key = R.key;
-    d.index = R.key & ((1ull << 40) - 1);
-    d.status = R.key ? ABACUS_DECIDE_OK : ABACUS_DECIDE_NONE;
-    d.pred_ms = R.key ? R.y_best : NAN;
-    d.total_ops = R.total_ops;
-    for (int j = 0; j < grid->k; j++) d.end_op[j] = R.end_op[j];
-    *out = d;
+    *out = sweep_decision(R, grid->k, headroom_ms);
     return ABACUS_OK;
 }
 
@@ -1450,6 +1463,150 @@ int abacus_combine_decisions(const abacus_decision_t* per_rank, int32_t nranks, 
         for (int j = 0; j < 4; j++) d.end_op[j] = 0;
     }
     *out = d;
+    return ABACUS_OK;
+}
+
+// ---- NEXT-4: what-if sweeps over bs / seqlen ---------------------------------
+namespace {
+int grow_whatif(abacus_ctx* c, int32_t n) {
+    int rc = grow_batch(c, n);
+    if (rc) return rc;
+    if (n <= c->whatif_cap) return ABACUS_OK;
+    if (c->h_wdecs) cudaFreeHost(c->h_wdecs);
+    if (c->h_wsegs) cudaFreeHost(c->h_wsegs);
+    cudaFree(c->d_wsegs);
+    c->h_wdecs = nullptr;
+    c->h_wsegs = nullptr;
+    c->d_wsegs = nullptr;
+    c->whatif_cap = 0;
+    const int32_t cap = c->batch_cap;  // grow_batch rounded n up
+    CUDA_TRY(c, cudaHostAlloc(&c->h_wdecs, (size_t)cap * sizeof(BatchDec), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaHostAlloc(&c->h_wsegs, (size_t)cap * kMaxSeg * sizeof(SegP), cudaHostAllocDefault));
+    CUDA_TRY(c, cudaMalloc(&c->d_wsegs, (size_t)cap * kMaxSeg * sizeof(SegP)));
+    c->whatif_cap = cap;
+    return ABACUS_OK;
+}
+
+// segment sink into a what-if variant's fixed slots (host staging)
+struct ArraySink {
+    SegP* segs;
+    void operator()(int i, const SegP& sg) const { segs[i] = sg; }
+};
+}  // namespace
+
+// What-if sweep (the load balancer picks
+// batch sizes at run time and inputs vary in length): the grid's candidates
+// under every (bs, seqlen) variant.  Tensor paths: every variant is one plan
+// of a single batched search launch (the NEXT-4 batch kernel), planned on the
+// host; fp32: one fused launch per variant.
+int abacus_search_whatif(abacus_ctx* c, const abacus_grid_t* grid, const abacus_variant_t* variants, int32_t n_var,
+                         float headroom_ms, abacus_decision_t* per_variant, abacus_decision_t* best,
+                         int32_t* best_variant) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
+    if (!variants || (!per_variant && !best)) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    if (n_var < 1 || n_var > ABACUS_BATCH_MAX)
+        return fail(c, ABACUS_E_INVALID, "n_var=%d outside [1,%d]", n_var, ABACUS_BATCH_MAX);
+    if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
+    uint64_t T = 0;
+    int rc = validate_grid(c, grid, &T);
+    if (rc) return rc;
+    if ((unsigned __int128)T * (unsigned __int128)n_var >= ((unsigned __int128)1 << 40))
+        return fail(c, ABACUS_E_INVALID, "n_var * |grid| >= 2^40");
+    for (int32_t v = 0; v < n_var; v++)
+        for (int j = 0; j < grid->k; j++) {
+            const int32_t b = variants[v].batch[j], l = variants[v].seqlen[j];
+            if (b < 1 || b > 32767 || l < 0 || l > 32767)
+                return fail(c, ABACUS_E_INVALID, "variant %d slot %d: batch %d / seqlen %d", v, j, b, l);
+        }
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    auto variant_grid = [&](int32_t v) {
+        abacus_grid_t g = *grid;
+        for (int j = 0; j < g.k; j++) {
+            g.slot[j].batch = variants[v].batch[j];
+            g.slot[j].seqlen = variants[v].seqlen[j];
+        }
+        return g;
+    };
+    std::vector<Result> res((size_t)n_var);
+    if (c->precision == ABACUS_FP32) {
+        for (int32_t v = 0; v < n_var; v++) {
+            const abacus_grid_t g = variant_grid(v);
+            Plan P = plan_grid_segments(c->n_models, c->D, &g, T, 0, T, headroom_ms);
+            P.mapped = c->dev_result;
+            P.seq = next_seq(c);
+            rc = launch_fused(c, P);
+            if (rc) return rc;
+            rc = wait_result(c, P.seq, &res[(size_t)v]);
+            if (rc) return rc;
+            host_decode(P, res[(size_t)v]);
+        }
+    } else {
+        rc = grow_whatif(c, n_var);
+        if (rc) return rc;
+        uint64_t pairs = 0;
+        uint32_t maxcnt = 0;
+        for (int32_t v = 0; v < n_var; v++) {
+            const abacus_grid_t g = variant_grid(v);
+            BatchDec& bd = c->h_wdecs[v];
+            SegP* segs = c->h_wsegs + (size_t)kMaxSeg * v;
+            plan_grid_segments_into(bd.h, ArraySink{segs}, c->n_models, c->D, &g, T, 0, T, headroom_ms);
+            bd.h.want_y0 = 1;
+            bd.h.mapped = nullptr;
+            bd.h.trace = nullptr;
+            bd.pair0 = pairs;
+            bd.seg0 = (uint32_t)(kMaxSeg * v);
+            pairs += (bd.h.n_tiles + 1) / 2;  // tiles padded to pairs, as for decision batches
+            for (int i = 0; i < bd.h.n_seg; i++)
+                for (int j = 0; j < kKMax; j++) maxcnt = segs[i].cnt[j] > maxcnt ? segs[i].cnt[j] : maxcnt;
+        }
+        cudaStream_t st = c->stream;
+        CUDA_TRY(c, cudaMemcpyAsync(c->d_decs, c->h_wdecs, (size_t)n_var * sizeof(BatchDec), cudaMemcpyHostToDevice,
+                                    st));
+        CUDA_TRY(c, cudaMemcpyAsync(c->d_wsegs, c->h_wsegs, (size_t)n_var * kMaxSeg * sizeof(SegP),
+                                    cudaMemcpyHostToDevice, st));
+        CUDA_TRY(c, cudaMemcpyAsync(c->d_pairs + n_var, &pairs, sizeof(uint64_t), cudaMemcpyHostToDevice, st));
+        CUDA_TRY(c, cudaMemsetAsync(c->d_acc, 0, (size_t)n_var * sizeof(BatchAcc), st));
+        CUDA_TRY(c, cudaMemsetAsync(c->d_y0, 0xFF, (size_t)n_var * sizeof(float), st));  // NaN
+        if (c->timed) cudaEventRecord(c->ev0, st);
+        const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
+        cudaError_t e = launch_batch_tc(c->d_decs, c->d_wsegs, n_var, c->d_pairs + n_var, pairs, maxcnt, c->D,
+                                        c->tw[fmt], c->d_w1b1, c->d_acc, c->d_y0, c->d_out, c->nsm, st);
+        if (c->timed) cudaEventRecord(c->ev1, st);
+        if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "what-if search launch: %s", cudaGetErrorString(e));
+        c->launches += 2;
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_out, c->d_out, (size_t)n_var * sizeof(Result), cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(c, cudaStreamSynchronize(st));
+        memcpy(res.data(), c->h_out, (size_t)n_var * sizeof(Result));
+    }
+    // the global best: max (sum_n, v T + t) over the variants (NEXT-4 reading: the
+    // variant is the most significant index digit)
+    uint64_t bkey = 0;
+    int32_t bv = -1;
+    for (int32_t v = 0; v < n_var; v++) {
+        const Result& R = res[(size_t)v];
+        if (per_variant) per_variant[v] = sweep_decision(R, grid->k, headroom_ms);
+        if (!R.key) continue;
+        const uint64_t lifted = (R.key & ~((1ull << 40) - 1)) | ((uint64_t)v * T + (R.key & ((1ull << 40) - 1)));
+        if (lifted > bkey) {
+            bkey = lifted;
+            bv = v;
+        }
+    }
+    if (best) {
+        Result R{};
+        uint64_t ev = 0;
+        for (int32_t v = 0; v < n_var; v++) ev += res[(size_t)v].evaluated;
+        if (bv >= 0) R = res[(size_t)bv];
+        R.y0 = res[0].y0;
+        R.evaluated = ev;
+        abacus_decision_t d = sweep_decision(R, grid->k, headroom_ms);
+        d.key = bkey;
+        d.index = bkey & ((1ull << 40) - 1);
+        *best = d;
+    }
+    if (best_variant) *best_variant = bv;
     return ABACUS_OK;
 }
 

@@ -737,8 +737,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
 // CTA can be in five different decisions.  On leaving a decision it folds its
 // best (key, y) into the decision's accumulator with a 128-bit CAS.
 // ---------------------------------------------------------------------------
-constexpr uint32_t kPlanBatchBytes =
-    (uint32_t)((sizeof(Plan) - kMaxSeg * sizeof(SegP) + kMaxSegBatch * sizeof(SegP) + 15) & ~size_t(15));
+// a group's plan slot holds up to kMaxSeg segments: decision batches use <= 8
+// (kMaxSegBatch), what-if sweeps (NEXT-4) whole grid plans of <= 16
+constexpr int kMaxSegSlot = kMaxSeg;
+constexpr uint32_t kPlanBatchBytes = (uint32_t)((sizeof(Plan) + 15) & ~size_t(15));
 
 __device__ __forceinline__ void acc_fold(BatchAcc* a, unsigned long long key, float y) {
     unsigned long long ok = a->key, oy = __float_as_uint(a->y);
@@ -764,7 +766,7 @@ __device__ __forceinline__ void acc_fold(BatchAcc* a, unsigned long long key, fl
 
 template <int FMT>
 __host__ __device__ inline TcSmem batch_smem_layout(int D, int ng, uint32_t* plans_off) {
-    TcSmem L = tc_smem_layout<FMT>(ng * kMaxSegBatch, TcCfg<FMT>::kNchL1 * kChunkBytesN32, ng,
+    TcSmem L = tc_smem_layout<FMT>(ng * kMaxSegSlot, TcCfg<FMT>::kNchL1 * kChunkBytesN32, ng,
                                    w1_stage_bytes(D, ng));
     *plans_off = (L.total + 15u) & ~15u;
     L.total = *plans_off + (uint32_t)ng * kPlanBatchBytes;
@@ -805,8 +807,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
     pp.set_outbias(TP.b4);
     pp.zero_a();
     constexpr uint32_t kTable = C::kNchL1 * kChunkBytesN32;
-    uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegBatch * kTable;
-    const uint64_t d1base = smem_desc(sbase + L.b1 + (uint32_t)g * kMaxSegBatch * kTable);
+    uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegSlot * kTable;
+    const uint64_t d1base = smem_desc(sbase + L.b1 + (uint32_t)g * kMaxSegSlot * kTable);
     constexpr uint32_t kSegStep = kTable >> 4;
     Plan& P = *reinterpret_cast<Plan*>(smem + plans_off + (size_t)g * kPlanBatchBytes);
     auto issue_l1 = [&](const TileIO& T, int s) {
