@@ -891,22 +891,57 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             };
             load_decision();
             enter_pair(pb, true);
-            for (uint64_t p = pb; p < pe; p++) {
+            // 32-bit loop state: pairs left in this group's range and in the current decision
+            uint32_t left = (uint32_t)(pe - pb), in_dec = (uint32_t)(dec_pair_end - pb);
+            bool first_pair = ltX == 0;
+            while (left) {
+                pp.template stage_as<0, true>(wq == 0);
+                pp.template stage_as<1, true>(wq == 1);
+                pp.template stage_as<2, true>(wq == 2);
+                // the next pair's rows are walked while the output MMA runs (inside a decision)
+                const bool same = in_dec > 1 && left > 1;  // warp-uniform
+                uint32_t n1 = 0, n2 = 0, ns = 0, m1 = 0, m2 = 0, ms = 0;
+                int nsX = 0, nsY = 0;
+                if (same) {
+                    ltX += 2;
+                    adv(ltX);
+                    n1 = W.a1; n2 = W.a2; ns = W.sn; nsX = W.s;
+                    adv(ltX + 1);
+                    m1 = W.a1; m2 = W.a2; ms = W.sn; nsY = W.s;
+                }
+                pp.wait();
                 uint32_t ybx, yby;
-                pp.template run_layers_fixed<true>(wq, ybx, yby);
-                if (ltX == 0 && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
+                tmem_ld1x2(pp.X.d + pp.lane_off, pp.Y.d + pp.lane_off, ybx, yby);
+                ybx = pp.add_b4(ybx);
+                yby = pp.add_b4(yby);
+                if (first_pair && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
+                first_pair = false;
                 fold_packed2(P, sX, x1, x2, xs, __uint_as_float(ybx), sY, y1, y2, ys, __uint_as_float(yby), best,
                              best_y, bsn);
-                if (p + 1 == dec_pair_end) {  // leaving decision d
+                left--;
+                in_dec--;
+                if (same) {
+                    x1 = n1; x2 = n2; xs = ns; sX = nsX;
+                    y1 = m1; y2 = m2; ys = ms; sY = nsY;
+                    store_a1_packed(pp.X.a1 + pp.lane_off, x1, x2);
+                    store_a1_packed(pp.Y.a1 + pp.lane_off, y1, y2);
+                    tmem_wait_st();
+                    if (pp.handoff(wq == 3)) {
+                        issue_l1(pp.X, sX);
+                        issue_l1(pp.Y, sY);
+                        pp.commit();
+                    }
+                } else if (in_dec == 0) {  // leaving decision d
                     flush();
                     bsn = 1u;
-                    if (p + 1 < pe) {
+                    if (left) {
+                        const uint64_t p = pe - left;  // the next pair, first of decision d + 1
                         d++;
                         load_decision();
-                        enter_pair(p + 1, true);
+                        in_dec = (uint32_t)(dec_pair_end - p);
+                        enter_pair(p, true);
+                        first_pair = ltX == 0;
                     }
-                } else if (p + 1 < pe) {
-                    enter_pair(p + 1, false);
                 }
             }
             flush();
