@@ -267,9 +267,13 @@ int abacus_search(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, double no
                   int32_t space, uint64_t grid_budget, abacus_decision_t* out);
 
 /* Many independent scheduling rounds in one call (
- * the paper runs one round at a time): decision i is exactly
+ * the paper runs one round at a time): decision i is
  * abacus_search(q + 4 i, k[i], now_ms[i], inflight_pred_ms[i], space,
- * grid_budget).  q: host array of 4 n query records (decision i uses
+ * grid_budget) -- bit for bit when every round of the batch takes the same
+ * layer-1 layout (every end-op range of <= 1,025 options, always true for
+ * the paper's registry, L <= 471); a batch mixing wider rounds runs the split
+ * layout for all of them, and the narrow rounds are then within the oracle's
+ * acceptance window (reading c18) rather than bit-identical.  q: host array of 4 n query records (decision i uses
  * q[4i .. 4i + k[i] - 1]; the rest are ignored); k, now_ms,
  * inflight_pred_ms: host arrays of n; out: host array of n decisions.
  * 1 <= n <= ABACUS_BATCH_MAX.  fp16 / bf16: one batched tensor-core launch

@@ -199,9 +199,11 @@ def test_batch_validation_matches_single_rounds(prec):
 
 
 def test_batch_layout_follows_single_round_bf16():
-    """bf16 splits the layer-1 digits above 257 end-op options. A long critical
-    query (whose slot is fixed) must not push a batch into the split layout
-    when every single round of it runs unsplit: the batch stays bit-identical."""
+    """A long critical query (whose slot is fixed) must not push a batch into the
+    split layer-1 layout when every single round of it runs unsplit: the batch
+    stays bit-identical.  (Both formats split above 1,025 end-op options since
+    the bf16 path took the fp16 digit operand; BERT-large from op 1 is the
+    registry's longest query.)"""
     c = Ctx(params=synth.weights(1), precision=ab.ABACUS_BF16)
     try:
         decs = []
@@ -215,5 +217,41 @@ def test_batch_layout_follows_single_round_bf16():
         got = ab.abacus_search_batch(c.h, decs)
         for (qs, now, infl), d in zip(decs, got):
             _same(d, ab.abacus_search(c.h, qs, now, infl))
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("prec", [ab.ABACUS_FP16, ab.ABACUS_BF16], ids=["fp16", "bf16"])
+def test_batch_mixed_layer1_layouts(prec):
+    """one batch launch runs ONE layer-1 layout, so a round with a
+    digit range above 1,025 (a long-model registry) puts the whole batch in the
+    split layout.  The wide rounds are then bit-identical to their single
+    search (same layout); the narrow ones run the split layout where their
+    single search would not, and must still be within the oracle's acceptance
+    window (reading c18) -- the ABI promises exactly this."""
+    ops = list(synth.OPS_PER_MODEL)
+    ops[0] = 3000  # model 1 with 3,000 ops
+    params = synth.weights(1)
+    c = Ctx(ops=ops, params=params, precision=prec)
+    try:
+        rng = np.random.default_rng(51)
+        decs, wide = [], []
+        for i in range(24):
+            w = i % 4 == 0
+            crit = synth.Query(4, int(rng.integers(1, 200)), 8, 0, 20.0 + rng.uniform(0, 5), 0.0)
+            other = synth.Query(1, 1 if w else 2900, 4, 0, 60.0 + rng.uniform(0, 20), 0.0)
+            third = synth.Query(7, int(rng.integers(1, 240)), 4, 64, 70.0, 0.0)
+            decs.append(([crit, other, third], 0.0, 0.0))
+            wide.append(w)
+        got = ab.abacus_search_batch(c.h, decs)
+        for (qs, now, infl), d, w in zip(decs, got, wide):
+            single = ab.abacus_search(c.h, qs, now, infl)
+            if w:
+                _same(d, single)
+            od = oracle.search(params, qs, now, infl, space=0, eps=EPS[prec], ops_per_model=ops)
+            if od.status == ab.ABACUS_DECIDE_OK and d.status == ab.ABACUS_DECIDE_OK:
+                assert accept_key(d.key, od.maxkey_strict, od.maxkey_loose)
+            elif abs(od.pred_critical_only_ms - od.headroom_ms) > EPS[prec] * abs(od.headroom_ms):
+                assert d.status == od.status
     finally:
         c.close()
