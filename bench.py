@@ -108,6 +108,39 @@ def cpu_oracle_rate(params, slots, H, budget_s=12.0, chunk=100_000):
     return n / dt, n, dt
 
 
+def cpu_oracle_other_configs(params):
+    """The fp64 oracle (1 thread, as it stands) on the other BASELINE configs
+    (SURVEY §8(d)): config 1 (all five 5,043-candidate grids), config 2 (100
+    3-way GRID decisions, oracle.search: a1 + exhaustive GRID + drop test),
+    config 5 (1e5 instance-based predictions, oracle.mlp64_batch).  Each
+    bounded to a few seconds."""
+    import oracle
+    out = {}
+    t0 = time.perf_counter()
+    n = 0
+    for _, g in synth.cfg1_grids():
+        r, _, _, _ = oracle.sweep(params, g, 15.0)
+        n += r.evaluated
+    dt = time.perf_counter() - t0
+    out["cfg1"] = {"candidates": n, "s": dt, "candidates_per_s": n / dt}
+    decs = synth.cfg2_decisions(100)
+    t0 = time.perf_counter()
+    n = 0
+    for qs, now, infl in decs:
+        n += oracle.search(params, qs, now, infl, space=0).evaluated
+    dt = time.perf_counter() - t0
+    out["cfg2"] = {"decisions": len(decs), "candidates": n, "s": dt, "candidates_per_s": n / dt,
+                   "decisions_per_s": len(decs) / dt, "space": "grid"}
+    G = synth.instance_samples(100_000, seed=15)
+    X = oracle.encode_groups(synth.N_MODELS, synth.K_MAX, [g.slots for g in G])
+    t0 = time.perf_counter()
+    oracle.mlp64_batch(params, X)
+    dt = time.perf_counter() - t0
+    out["cfg5"] = {"predictions": len(G), "s": dt, "predictions_per_s": len(G) / dt}
+    out["cores"] = 1
+    return out
+
+
 def cpu_oracle_rate_all_cores(params, slots, H, budget_s=8.0, chunk=50_000):
     """The same oracle on every host core the process may use: one Python
     thread per core, each sweeping its own contiguous sub-range (ctypes
@@ -323,6 +356,8 @@ def main():
             cpu_all = {"value": ra, "unit": "candidates/s", "cores": nc, "kind": "oracle",
                        "sample": "%d config-4 candidates in %d contiguous ranges from T/2 (%.1f s, %d threads)"
                                  % (na, nc, dta, nc)}
+            if world == 1:
+                cpu["other_configs"] = cpu_oracle_other_configs(params)
         value = T * args.steps / elapsed
         line = {
             "metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world, "steps": args.steps,
