@@ -36,7 +36,7 @@ import synth  # noqa: E402
 FLOP_PER_CAND = 2 * (synth.D * 32 + 32 * 32 + 32 * 32 + 32)  # 5,696 algorithmic FLOP (D = 24)
 METRIC = "predictor candidates/sec (config 4 exhaustive overlap sweep, abacus_search_grid)"
 PREC = {"fp32": 0, "bf16": 1, "fp16": 2}
-DTYPE = {"fp32": "f32", "bf16": "bf16 (weights hi+lo), f32 accum", "fp16": "f16 (layers 1 + output: f32 accum; layers 2-3: f16 accum)"}
+DTYPE = {"fp32": "f32", "bf16": "bf16 (layers 2, 3, output bf16 operands, W3 hi+lo; layer-1 digit operand f16), f32 accum", "fp16": "f16 (layers 1 + output: f32 accum; layers 2-3: f16 accum)"}
 
 
 def peaks():
@@ -437,21 +437,29 @@ def secondary_paths(ab, ctx, params, grid, H, T, headline, stream, steps=(("bf16
 
 def whatif_sweep(ab, ctx, slots, H, T, reps=3):
     """NEXT-4 what-if sweep on the config-4 grid: BERT-large's batch size
-    swept over {1, 2, 4, 8} (4 x 9.19e9 candidates in one batched launch,
-    abacus_search_whatif).  Device time of the launch (CUDA events)."""
+    swept over {1, 2, 4, 8} (4 x 9.19e9 candidates, abacus_search_whatif).
+    Time of the whole blocking call between CUDA events on the current
+    stream (the ctx runs on it)."""
     variants = [([8, 8, 8, b], [0, 0, 128, 512]) for b in (1, 2, 4, 8)]
     g = ab.make_grid(slots)
     ab.abacus_search_whatif(ctx, g, variants, H)  # warm-up (grows the buffers)
+    import torch
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     kms = []
     for _ in range(reps):
+        torch.cuda.synchronize()
+        e0.record()
         per, best, bv = ab.abacus_search_whatif(ctx, g, variants, H)
-        kms.append(ab.abacus_last_kernel_ms(ctx))
+        e1.record()
+        torch.cuda.synchronize()
+        kms.append(e0.elapsed_time(e1))
     k = float(np.mean(kms))
     n = T * len(variants)
     return {"grid": "config 4, BERT-large bs in {1, 2, 4, 8}", "variants": len(variants), "candidates": n,
-            "kernel_ms": k, "candidates_per_s": n / (k / 1e3), "best_variant": bv, "best_key": best.key,
+            "call_ms": k, "candidates_per_s": n / (k / 1e3), "best_variant": bv, "best_key": best.key,
             "per_variant_total_ops": [d.total_ops for d in per],
-            "path": "abacus_search_whatif: one fused_batch_tc_kernel launch (4 plans) + finalize"}
+            "path": "abacus_search_whatif: 4 variant grids of 9.19e9 candidates (>= 2^24: one fused search "
+                    "launch each)"}
 
 
 def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50):

@@ -328,9 +328,9 @@ int abacus_search_grid(abacus_ctx* ctx, const abacus_grid_t* grid, float headroo
  * total_ops of that candidate, evaluated n_var T, pred_critical_only_ms =
  * y(index 0) of variant 0; status OK or NONE.  *best_variant (may be NULL)
  * = its v, -1 if nothing fits.  1 <= n_var <= ABACUS_BATCH_MAX and
- * n_var T < 2^40.  Tensor precisions: one batched launch for all variants
- * (each variant a plan of the NEXT-4 batch kernel); fp32: one fused launch
- * per variant.  Blocking.  Errors: as abacus_search_grid, plus E_INVALID for
+ * n_var T < 2^40.  Tensor precisions with T < 2^24: one batched launch for
+ * all variants (each variant a plan of the NEXT-4 batch kernel); fp32, or
+ * T >= 2^24: one fused search launch per variant.  Blocking.  Errors: as abacus_search_grid, plus E_INVALID for
  * a variant's batch outside [1, 32767] or seqlen outside [0, 32767]. */
 int abacus_search_whatif(abacus_ctx* ctx, const abacus_grid_t* grid, const abacus_variant_t* variants,
                          int32_t n_var, float headroom_ms, abacus_decision_t* per_variant,

@@ -1530,7 +1530,13 @@ int abacus_search_whatif(abacus_ctx* c, const abacus_grid_t* grid, const abacus_
         return g;
     };
     std::vector<Result> res((size_t)n_var);
-    if (c->precision == ABACUS_FP32) {
+    // Large variant grids run one fused single-search launch each: at >= 2^24
+    // candidates the ~10 us launch + prologue is < 10 % of a variant, and the
+    // single kernel's inner loop (plan in the constant bank, unrolled by two)
+    // is ~1.2x the batch kernel's per candidate on the same grid
+    // (tools/exp_whatif.py).  Smaller grids share one batched launch.
+    const bool per_launch = c->precision == ABACUS_FP32 || T >= (1ull << 24);
+    if (per_launch) {
         for (int32_t v = 0; v < n_var; v++) {
             const abacus_grid_t g = variant_grid(v);
             Plan P = plan_grid_segments(c->n_models, c->D, &g, T, 0, T, headroom_ms);

@@ -892,14 +892,15 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             load_decision();
             enter_pair(pb, true);
             // 32-bit loop state: pairs left in this group's range and in the current decision
-            uint32_t left = (uint32_t)(pe - pb), in_dec = (uint32_t)(dec_pair_end - pb);
-            bool first_pair = ltX == 0;
+            // bit 31 of in_dec: this pair's X row 0 is the decision's index 0 (y(0) owed)
+            constexpr uint32_t kOweY0 = 0x80000000u;
+            uint32_t left = (uint32_t)(pe - pb), in_dec = (uint32_t)(dec_pair_end - pb) | (ltX == 0 ? kOweY0 : 0u);
             while (left) {
                 pp.template stage_as<0, true>(wq == 0);
                 pp.template stage_as<1, true>(wq == 1);
                 pp.template stage_as<2, true>(wq == 2);
                 // the next pair's rows are walked while the output MMA runs (inside a decision)
-                const bool same = in_dec > 1 && left > 1;  // warp-uniform
+                const bool same = (in_dec & ~kOweY0) > 1 && left > 1;  // warp-uniform
                 uint32_t n1 = 0, n2 = 0, ns = 0, m1 = 0, m2 = 0, ms = 0;
                 int nsX = 0, nsY = 0;
                 if (same) {
@@ -914,8 +915,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
                 tmem_ld1x2(pp.X.d + pp.lane_off, pp.Y.d + pp.lane_off, ybx, yby);
                 ybx = pp.add_b4(ybx);
                 yby = pp.add_b4(yby);
-                if (first_pair && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
-                first_pair = false;
+                if ((in_dec & kOweY0) && r == 0 && P.want_y0) y0s[d] = __uint_as_float(ybx);
+                in_dec &= ~kOweY0;
                 fold_packed2(P, sX, x1, x2, xs, __uint_as_float(ybx), sY, y1, y2, ys, __uint_as_float(yby), best,
                              best_y, bsn);
                 left--;
@@ -940,7 +941,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
                         load_decision();
                         in_dec = (uint32_t)(dec_pair_end - p);
                         enter_pair(p, true);
-                        first_pair = ltX == 0;
+                        if (ltX == 0) in_dec |= kOweY0;
                     }
                 }
             }

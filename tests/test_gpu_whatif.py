@@ -93,3 +93,28 @@ def test_whatif_errors(ctx):
     big = synth.cfg4_grid()  # 9.19e9 candidates: 120 variants exceed 2^40 indices
     with pytest.raises(ab.AbacusError):
         ab.abacus_search_whatif(ctx.h, ab.make_grid(big), [([8, 8, 8, 4], [0, 0, 128, 512])] * 120, 30.0)
+
+
+@pytest.mark.parametrize("prec", [ab.ABACUS_FP16, ab.ABACUS_BF16], ids=["fp16", "bf16"])
+def test_whatif_large_grid_takes_per_variant_launches(ctx, prec):
+    """Variant grids of >= 2^24 candidates run one fused search launch each:
+    every variant equals abacus_search_grid of its grid, and the global best is
+    the max over the variants' keys lifted to v T + t."""
+    ctx.load(ctx.params, prec)
+    slots = [synth.GridSlot(3, 200, 8, 0, 200, 360, 1), synth.GridSlot(4, 100, 8, 0, 100, 220, 1),
+             synth.GridSlot(7, 100, 8, 128, 100, 243, 1), synth.GridSlot(8, 400, 4, 512, 400, 471, 1)]
+    T = oracle.grid_size(slots)
+    assert T >= 1 << 24
+    variants = [([8, 8, 8, b], [0, 0, 128, 512]) for b in (1, 4, 16)]
+    H = synth.cfg4_headroom()
+    per, best, bv = ab.abacus_search_whatif(ctx.h, ab.make_grid(slots), variants, H)
+    lifted = []
+    for v, (bss, sls) in enumerate(variants):
+        gv = [synth.GridSlot(s.model_id, s.start_op, bss[j], sls[j], s.end_lo, s.end_hi, s.allow_absent)
+              for j, s in enumerate(slots)]
+        single = ab.abacus_search_grid(ctx.h, ab.make_grid(gv), H, 0, T)
+        assert (per[v].key, list(per[v].end_op), per[v].evaluated) == (single.key, list(single.end_op), T)
+        k = per[v].key
+        lifted.append(((k >> 40) << 40) | (v * T + (k & ((1 << 40) - 1))) if k else 0)
+    assert best.key == max(lifted) and (bv == int(np.argmax(lifted)) if best.key else bv == -1)
+    ctx.load(ctx.params, ab.ABACUS_FP32)
