@@ -153,12 +153,20 @@ __device__ __forceinline__ bool walker_is_index0(const Walker& W, uint32_t r) {
 // accepts (every candidate has sn >= 1).  The digits themselves are unpacked
 // only when a fold has to build a key.
 // ---------------------------------------------------------------------------
-struct PackedWalker {
+// GEN (the batch kernel): one add / compare / subtract chain for every
+// segment (the tile advance as mixed-radix digits D_j < cnt_j, at most one
+// carry per digit).  !GEN (the single search kernel, at its 96-register cap,
+// where the three extra increment words spill): the chain for segments whose
+// fastest digit has >= 128 options (D = (128, 0, 0, 0)), a radix division per
+// digit otherwise.
+template <bool GEN>
+struct PackedWalkerT {
     uint32_t a1, a2, sn;  // per row: the most recently taken tile
     int32_t s;            // segment (uniform)
     uint32_t tl;          // tiles of the segment left, the current one included (uniform)
     uint32_t last_rows;   // valid rows of the segment's last tile (uniform)
-    uint32_t fast;        // cnt3 >= 128: one carry at most per tile advance
+    uint32_t fast;        // !GEN: cnt3 >= 128 (one carry at most per tile advance)
+    uint32_t inc2, inc1, incsn;  // GEN: +128 rows as box digits, packed (v3, v2), (v1, v0) words and their sum
     uint32_t lim3, dec3, dsn3, lim2, cnt2, dsn2, lim1, dec1, dsn1;  // carry constants (uniform)
     uint64_t ub;          // box ordinal of the current tile's row 0 (general advance only)
 
@@ -178,6 +186,21 @@ struct PackedWalker {
         last_rows = (uint32_t)(n - (nt - 1) * kTileM);
         ub = g.u_begin + o * kTileM;
         fast = g.fast_carry;
+        // GEN: the tile advance (+128 box ordinals) as mixed-radix digits D_j <
+        // cnt_j: adding them digit by digit needs at most one carry per digit
+        // (v_j + D_j + 1 < 2 cnt_j), so every segment takes the same add /
+        // compare / subtract chain
+        if (GEN) {
+            uint32_t rem = (uint32_t)kTileM, d[kKMax];
+#pragma unroll
+            for (int j = kKMax - 1; j >= 0; j--) {
+                d[j] = j > 0 ? rem % g.cnt[j] : rem;
+                rem = j > 0 ? rem / g.cnt[j] : 0u;
+            }
+            inc2 = (d[3] << 16) + d[2];
+            inc1 = (d[1] << 16) + d[0];
+            incsn = d[0] + d[1] + d[2] + d[3];
+        }
         lim3 = (0x6400u + g.cnt[3]) << 16;
         dec3 = (g.cnt[3] << 16) - 1u;
         dsn3 = g.cnt[3] - 1u;
@@ -201,10 +224,16 @@ struct PackedWalker {
         }
         tl--;
         ub += kTileM;
-        if (fast) {
-            a2 += (uint32_t)kTileM << 16;
-            sn += kTileM;
-            const bool c3 = a2 >= lim3;  // the low half (0x6400 + v2) never reaches bit 16
+        if (GEN || fast) {
+            if (GEN) {
+                a2 += inc2;  // v3 += D3, v2 += D2 (low half stays below bit 16: v2 + D2 + 1 < 2 cnt2 <= 2050)
+                a1 += inc1;  // v1 += D1, v0 += D0
+                sn += incsn;
+            } else {
+                a2 += (uint32_t)kTileM << 16;
+                sn += kTileM;
+            }
+            const bool c3 = a2 >= lim3;  // v3 >= cnt3 (the low half never reaches bit 16)
             if (c3) { a2 -= dec3; sn -= dsn3; }  // v3 -= cnt3, v2 += 1
             const bool c2 = (a2 & 0xFFFFu) >= lim2;
             if (c2) { a2 -= cnt2; a1 += 0x10000u; sn -= dsn2; }  // v2 -= cnt2, v1 += 1
@@ -229,6 +258,8 @@ struct PackedWalker {
         if (tl == 1 && last_rows < (uint32_t)kTileM && r >= last_rows) sn = 0u;
     }
 };
+
+using PackedWalker = PackedWalkerT<false>;
 
 // fold one row of a packed tile: the key is built only when the row fits the
 // headroom and its sum_n can reach the running best

@@ -864,7 +864,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
         };
         if constexpr (!SPLIT) {
             // packed walker + three-instruction fold (as fused_tc_kernel)
-            PackedWalker W{};
+            PackedWalkerT<true> W{};
             uint32_t x1 = 0, x2 = 0, xs = 0, y1 = 0, y2 = 0, ys = 0, bsn = 1u;
             int sX = 0, sY = 0;
             uint64_t ltX = 0;
