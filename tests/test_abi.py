@@ -58,10 +58,10 @@ def test_struct_layouts_match_header(built):
 #include <stddef.h>
 #include "abacus.h"
 int main(void) {
-  printf("%zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(abacus_slot_t), sizeof(abacus_grid_t),
+  printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(abacus_slot_t), sizeof(abacus_grid_t),
          sizeof(abacus_group_t), sizeof(abacus_query_t), sizeof(abacus_decision_t),
          offsetof(abacus_decision_t, key), offsetof(abacus_decision_t, total_ops),
-         offsetof(abacus_query_t, qos_ms));
+         offsetof(abacus_query_t, qos_ms), sizeof(abacus_variant_t), offsetof(abacus_variant_t, seqlen));
   return 0;
 }'''
     with tempfile.TemporaryDirectory() as d:
@@ -72,7 +72,8 @@ int main(void) {
         got = [int(v) for v in subprocess.check_output([exe]).decode().split()]
     want = [C.sizeof(ab.abacus_slot_t), C.sizeof(ab.abacus_grid_t), C.sizeof(ab.abacus_group_t),
             C.sizeof(ab.abacus_query_t), C.sizeof(ab.abacus_decision_t), ab.abacus_decision_t.key.offset,
-            ab.abacus_decision_t.total_ops.offset, ab.abacus_query_t.qos_ms.offset]
+            ab.abacus_decision_t.total_ops.offset, ab.abacus_query_t.qos_ms.offset, C.sizeof(ab.abacus_variant_t),
+            ab.abacus_variant_t.seqlen.offset]
     assert got == want
 
 
