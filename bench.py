@@ -383,7 +383,11 @@ def main():
             "secondary_paths": secondary,
             "whatif": whatif,
         }
-        print(json.dumps(line))
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        # rank 0 ran the single-GPU latency and CPU legs alone: every rank tears
+        # down the library's communicator together (ncclCommDestroy finalizes)
+        dist.barrier()
     if comm:
         ab.abacus_nccl_comm_destroy(comm)
     ab.abacus_destroy(ctx)
