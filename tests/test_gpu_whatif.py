@@ -118,3 +118,41 @@ def test_whatif_large_grid_takes_per_variant_launches(ctx, prec):
         lifted.append(((k >> 40) << 40) | (v * T + (k & ((1 << 40) - 1))) if k else 0)
     assert best.key == max(lifted) and (bv == int(np.argmax(lifted)) if best.key else bv == -1)
     ctx.load(ctx.params, ab.ABACUS_FP32)
+
+
+@pytest.mark.parametrize("prec", [ab.ABACUS_FP16, ab.ABACUS_BF16], ids=["fp16", "bf16"])
+def test_whatif_small_radix_grids(ctx, prec):
+    """Grids whose digits all have few options (2..23), so one tile advance
+    (+128 rows) wraps several digits at once: the batch kernel's walker adds
+    the advance as mixed-radix digits with one carry per digit, the single
+    search divides by each radix.  Every variant must equal abacus_search_grid
+    bit for bit and be acceptable to the oracle; the whole grid spans many
+    tiles and a ragged tail."""
+    ctx.load(ctx.params, prec)
+    rng = np.random.default_rng(61)
+    for it in range(12):
+        k = int(rng.integers(2, 5))
+        models = [int(m) for m in rng.choice(np.arange(1, 9), size=k, replace=False)]
+        slots = []
+        for m in models:
+            L = synth.L(m)
+            n = int(rng.integers(1, 23))
+            lo = int(rng.integers(1, L - n + 2))
+            slots.append(synth.GridSlot(m, lo, int(rng.choice([1, 8, 32])), synth.seqlen_for(m, 128), lo,
+                                        lo + n - 1, int(rng.integers(0, 2))))
+        T = oracle.grid_size(slots)
+        _, y, _, _ = oracle.sweep(ctx.params, slots, 0.0, want_y=True)
+        H = float(np.float32(np.quantile(y, rng.uniform(0.2, 0.9))))
+        variants = [([int(b)] * k, [synth.seqlen_for(m, int(s)) for m in models])
+                    for b, s in ((1, 16), (8, 128), (32, 512))]
+        per, best, bv = ab.abacus_search_whatif(ctx.h, ab.make_grid(slots), variants, H)
+        oper, _, (strict, loose) = oracle.whatif(ctx.params, slots, variants, H, eps=EPS[prec])
+        for v, (bss, sls) in enumerate(variants):
+            gv = [synth.GridSlot(s.model_id, s.start_op, bss[j], sls[j], s.end_lo, s.end_hi, s.allow_absent)
+                  for j, s in enumerate(slots)]
+            single = ab.abacus_search_grid(ctx.h, ab.make_grid(gv), H, 0, T)
+            assert (per[v].key, list(per[v].end_op), per[v].evaluated) == \
+                   (single.key, list(single.end_op), single.evaluated), (it, v, T)
+            assert accept_key(per[v].key, oper[v].maxkey_strict, oper[v].maxkey_loose), (it, v)
+        assert accept_key(best.key, strict, loose)
+    ctx.load(ctx.params, ab.ABACUS_FP32)
