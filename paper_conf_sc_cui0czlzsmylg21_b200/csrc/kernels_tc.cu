@@ -225,6 +225,7 @@ struct TcPipe {
     uint32_t tCx, tCy, lane_off, bar_id, ph;  // bias constant chunk of X / Y (may be shared)
     uint64_t* bar;
     uint64_t db2, db3, db4;
+
     uint32_t hb_smem;  // fp16: shared address of layer 2's bias words (layer 3's follow one blob later)
     bool me[4];
     // fp16: the output layer runs without its bias K chunk and b4 is added to y
@@ -272,6 +273,13 @@ struct TcPipe {
         db2 = d2;
         db3 = d3;
         db4 = d4;
+        // opaque copies: the compiler keeps the descriptors live instead of
+        // rebuilding them from the shared-memory base at every issue (~7 uniform
+        // instructions per stage on the issuing warp: +1.3 % on config 4)
+        asm volatile("mov.b64 %0, %0;" : "+l"(db2));
+        asm volatile("mov.b64 %0, %0;" : "+l"(db3));
+        asm volatile("mov.b64 %0, %0;" : "+l"(db4));
+
         // fp16: the bias chunk of each hidden layer holds its 16 f16 bias pairs instead
         hb_smem = ((uint32_t)(d2 & 0x3FFFu) << 4) + 2u * kChunkBytesN32;
 #pragma unroll
