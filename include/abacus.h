@@ -66,8 +66,13 @@ enum {
 /* predictor arithmetic (reading c16) */
 enum {
     ABACUS_FP32 = 0, /* SIMT FFMA, fp32 weights and activations                     */
-    ABACUS_BF16 = 1, /* tcgen05 kind::f16, bf16 operands (weights split hi+lo),     */
-                     /* fp32 accumulation in TMEM                                   */
+    ABACUS_BF16 = 1, /* tcgen05 kind::f16, fp32 accumulation in TMEM; bf16 operands */
+                     /* for layers 2, 3 and the output (W3 split hi + lo, layer-2   */
+                     /* and output weights hi only, hidden biases as hi + lo rows  */
+                     /* of a bias K chunk, b4 in fp32); layer 1 of the fused search */
+                     /* and of the D = 24 predictor enters through the fp16 operand */
+                     /* of exact features / digits (1024 + v).  Error vs the fp64  */
+                     /* oracle on config 5: max 8.1e-3 relative (DESIGN.md r2)      */
     ABACUS_FP16 = 2  /* tcgen05 kind::f16, fp16 operands with exact power-of-two    */
                      /* layer scaling; accumulation in TMEM is fp32 for layer 1 and */
                      /* the output layer but F16 for hidden layers 2 and 3 (their   */

@@ -1,26 +1,34 @@
 // kernels_tc.cu -- tensor-core (tcgen05 / TMEM) kernels of the Abacus search.
 //
-//   fused_tc_kernel    a2..a5 fused: enumerate -> layer-1 operand in TMEM ->
-//                      3 hidden MMAs + output MMA (bias via a constant-1 K
-//                      column, ReLU + fp16/bf16 pack in the epilogue) ->
-//                      headroom mask -> running max key
-//   predict_tc_kernel  a4 alone: int16 Fig.-8 rows from HBM -> same MLP
+//   fused_tc_kernel        a2..a5 fused: enumerate -> layer-1 operand in TMEM ->
+//                          layer 1, 2, 3 and output MMAs (ReLU + pack in the
+//                          epilogues) -> headroom mask -> running max key
+//
+//   fused_batch_tc_kernel  the same for many independent plans per launch
+//                          (NEXT-4 decision batches and what-if variants)
+//   predict24_tc_kernel    a4 alone, D = 24: int16 Fig.-8 rows from HBM (TMA)
+//   predict_tc_kernel      a4 alone, any D <= 31
 //
 // CTA = NG groups of 4 warps.  A group owns 128 candidate rows = the 128 TMEM
 // lanes (warp q of a group reaches lanes 32q..32q+31) and a private slice of
-// TMEM columns; its first thread issues the group's MMAs (M = 128, N = 32,
-// K = 16 per instruction, A from TMEM, B = weights resident in shared memory)
-// and commits them to the group's mbarrier.  Groups run independently, so
-// while one group waits on its MMA the others run their epilogues.
+// TMEM columns; one elected thread issues the group's MMAs (M = 128, N = 32,
+// or 8 for the output layer, K = 16 per instruction, A from TMEM, B = weights
+// resident in shared memory) and commits them to the group's mbarrier.
+// Groups run independently, so while one group waits on its MMA the others
+// run their epilogues.
 //
-// Numerics:
-//   fp16 (FMT 0): weights and activations fp16 RNE, fp32 accumulation; layers
-//     are rescaled by exact powers of two so activations stay in fp16 range
-//     (ReLU is positively homogeneous, so the output is unchanged).
-//   bf16 (FMT 1): activations bf16 RNE; weights split W = W_hi + W_lo (both
-//     bf16) and both halves multiplied (two MMAs per K chunk), fp32 accumulation.
-//   Biases enter as a (hi, lo) pair against a constant-1 K column (both fmts).
-//   Integer digits / features enter split as 256*hi + lo (exact in both fmts).
+// Numerics (reading r2, §4):
+//   fp16 (FMT 0): weights and activations fp16 RNE; layers are rescaled by
+//     exact powers of two so activations stay in fp16 range (ReLU is
+//     positively homogeneous, so the output is unchanged).  Layer 1 and the
+//     output accumulate in fp32, hidden layers 2-3 in f16 with their biases
+//     added in the f16 epilogue; b4 is added in fp32.
+//   bf16 (FMT 1): layer 1 as in fp16 (fp16 digit / feature operand, fp16
+//     table, fp32 accumulation), then bf16 activations; W2 and w4 bf16 (hi),
+//     W3 = W3_hi + W3_lo (both multiplied); hidden biases as a (hi, lo) pair
+//     against a constant-1 K column; fp32 accumulation; b4 in fp32.
+//   Digits / features enter as the exact fp16 values 1024 + v (v < 1024), or
+//   split as 256 hi + lo above (SPLIT).
 #include <cuda_runtime.h>
 #include <math.h>
 
