@@ -50,6 +50,7 @@ extern "C" {
 #define ABACUS_HIDDEN 32
 #define ABACUS_ABI_VERSION 3
 #define ABACUS_BATCH_MAX (1 << 20) /* decisions per abacus_search_batch call */
+#define ABACUS_WHATIF_MAX (1 << 16) /* variants per abacus_search_whatif call */
 #define ABACUS_TRAIN_MAX_BATCH 65536 /* samples per training step */
 
 /* status codes */
@@ -332,7 +333,7 @@ int abacus_search_grid(abacus_ctx* ctx, const abacus_grid_t* grid, float headroo
  * key ((sum_n + 1) << 40) | (v T + t), index v T + t, end_op / pred_ms /
  * total_ops of that candidate, evaluated n_var T, pred_critical_only_ms =
  * y(index 0) of variant 0; status OK or NONE.  *best_variant (may be NULL)
- * = its v, -1 if nothing fits.  1 <= n_var <= ABACUS_BATCH_MAX and
+ * = its v, -1 if nothing fits.  1 <= n_var <= ABACUS_WHATIF_MAX and
  * n_var T < 2^40.  Tensor precisions with T < 2^24: one batched launch for
  * all variants (each variant a plan of the NEXT-4 batch kernel); fp32, or
  * T >= 2^24: one fused search launch per variant.  Blocking.  Errors: as abacus_search_grid, plus E_INVALID for

@@ -1506,8 +1506,8 @@ int abacus_search_whatif(abacus_ctx* c, const abacus_grid_t* grid, const abacus_
     c->err.clear();
     if (!c->loaded) return fail(c, ABACUS_E_NOT_LOADED, "no predictor loaded");
     if (!variants || (!per_variant && !best)) return fail(c, ABACUS_E_INVALID, "NULL argument");
-    if (n_var < 1 || n_var > ABACUS_BATCH_MAX)
-        return fail(c, ABACUS_E_INVALID, "n_var=%d outside [1,%d]", n_var, ABACUS_BATCH_MAX);
+    if (n_var < 1 || n_var > ABACUS_WHATIF_MAX)
+        return fail(c, ABACUS_E_INVALID, "n_var=%d outside [1,%d]", n_var, ABACUS_WHATIF_MAX);
     if (std::isnan(headroom_ms)) return fail(c, ABACUS_E_INVALID, "headroom is NaN");
     uint64_t T = 0;
     int rc = validate_grid(c, grid, &T);
