@@ -1479,7 +1479,8 @@ int grow_whatif(abacus_ctx* c, int32_t n) {
     c->h_wsegs = nullptr;
     c->d_wsegs = nullptr;
     c->whatif_cap = 0;
-    const int32_t cap = c->batch_cap;  // grow_batch rounded n up
+    int32_t cap = 256;  // own capacity: a large earlier decision batch must not size the plan staging
+    while (cap < n) cap *= 2;
     CUDA_TRY(c, cudaHostAlloc(&c->h_wdecs, (size_t)cap * sizeof(BatchDec), cudaHostAllocDefault));
     CUDA_TRY(c, cudaHostAlloc(&c->h_wsegs, (size_t)cap * kMaxSeg * sizeof(SegP), cudaHostAllocDefault));
     CUDA_TRY(c, cudaMalloc(&c->d_wsegs, (size_t)cap * kMaxSeg * sizeof(SegP)));
