@@ -319,8 +319,15 @@ def main():
 
     # ---- per-decision sharded search (config 3 pure GRID, all ranks) --------
     sharded = None
+    sharded_peer = None
     if not args.no_decisions:
         sharded = sharded_decision_latency(ab, ctx, comm, world, rank)
+        # the same decisions with the combine inside the search kernel (peer mailboxes,
+        # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator)
+        pcomm = ab.peer_comm_from_process_group(ctx) if world > 1 else \
+            ab.abacus_peer_comm_init(ctx, 1, 0, [ab.abacus_peer_export(ctx)])
+        sharded_peer = sharded_decision_latency(ab, ctx, pcomm, world, rank, label="peer")
+        ab.abacus_peer_comm_destroy(pcomm)
 
     # ---- per-decision latency (config 2, 3-way; 1 GPU each) -----------------
     dec = None
@@ -380,6 +387,7 @@ def main():
             "clocks": clk.summary(),
             "decision_latency": dec,
             "decision_latency_sharded": sharded,
+            "decision_latency_sharded_peer": sharded_peer,
             "secondary_paths": secondary,
             "whatif": whatif,
         }
@@ -466,7 +474,7 @@ def whatif_sweep(ab, ctx, slots, H, T, reps=3):
                     "launch each)"}
 
 
-def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50):
+def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50, label="nccl"):
     """Per-decision latency of abacus_search_sharded on config-3 4-way pure
     GRID decisions (up to 4.1e7 candidates each): every rank searches its
     contiguous shard of each decision's grid and one all-gather combines them
@@ -495,7 +503,9 @@ def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50):
             "max_us": float(a.max()), "grid_p50": float(np.percentile(ev, 50)), "grid_p99": float(np.percentile(ev, 99)),
             "grid_max": float(ev.max()),
             "path": "Python binding -> abacus_search_sharded (%s)" % (
-                "NCCL all-gather over %d ranks" % world if world > 1 else "1 GPU, no collective")}
+                ("NCCL all-gather over %d ranks" % world if world > 1 else "1 GPU, no collective")
+                if label == "nccl" else
+                "combine inside the search kernel over %d ranks' peer mailboxes" % world)}
 
 
 def decision_latency(ab, ctx, n=10_000, warm=100, precision="fp16"):

@@ -306,8 +306,9 @@ int abacus_search_mway(abacus_ctx* ctx, const abacus_query_t* q, int32_t k, doub
 
 /* a2..a6 over a sweep grid: candidates t in [first, first+count) of `grid`
  * (host) under `headroom_ms`; this rank's shard.  With nccl_comm != NULL
- * (an ncclComm_t on this device, e.g. from abacus_nccl_comm_init) the
- * per-rank results are combined with one collective so every rank returns
+ * (an ncclComm_t on this device, e.g. from abacus_nccl_comm_init, or a peer
+ * communicator from abacus_peer_comm_init: the combine then runs inside the
+ * search kernel) the per-rank results are combined so every rank returns
  * the same global decision (status OK or NONE, end_op per slot, pred_ms of
  * t*, evaluated summed over ranks, pred_critical_only_ms = y(index 0) from
  * the rank whose shard holds index 0; see abacus_combine_decisions).
@@ -389,6 +390,41 @@ int abacus_nccl_unique_id(uint8_t* id128);
 int abacus_nccl_comm_init(abacus_ctx* ctx, int32_t nranks, int32_t rank, const uint8_t* id128,
                           void** comm_out);
 void abacus_nccl_comm_destroy(void* comm);
+
+/* ------------------------------------------------------------------------ */
+/* a6 over peer memory: the combine inside the search kernel                 */
+/* ------------------------------------------------------------------------ */
+/* Instead of an ncclComm_t, abacus_search_grid and abacus_search_sharded
+ * accept a peer communicator from abacus_peer_comm_init.  Each rank owns a
+ * device mailbox of ABACUS_PEER_MAX tagged 64-byte records.  The last CTA of
+ * a rank's fused search writes its 56-byte result into slot `rank` of every
+ * rank's mailbox (peer stores: NVLink between GPUs, plain stores between
+ * ctxs of one device), then waits in its own mailbox for every rank's record
+ * of the same launch and combines them exactly as the NCCL path does (max
+ * key, evaluated summed, y(0) from the lowest rank that holds index 0) -- no
+ * collective launch, no finalize kernel.  Every rank must make the same
+ * sequence of peer-combined calls (the launches are matched by a counter).
+ * A rank whose record does not arrive within ABACUS_PEER_TIMEOUT_MS
+ * milliseconds (environment, default 10000) fails the call with E_NCCL.
+ * Ranks in one process may share a device (tests); ranks in different
+ * processes exchange CUDA IPC handles. */
+#define ABACUS_PEER_MAX 32   /* ranks per peer communicator */
+#define ABACUS_PEER_BLOB 128 /* bytes of an exported mailbox description */
+
+/* Allocate this ctx's mailbox (first call) and describe it in `blob`
+ * (host, ABACUS_PEER_BLOB bytes: CUDA IPC handle, process id, device
+ * address, device ordinal).  Errors: E_INVALID, E_CUDA. */
+int abacus_peer_export(abacus_ctx* ctx, uint8_t* blob);
+/* Build a peer communicator for (nranks, rank) from every rank's blob
+ * (host, nranks x ABACUS_PEER_BLOB, rank order, e.g. all-gathered with
+ * torch.distributed); opens the other processes' mailboxes with CUDA IPC.
+ * *comm_out is owned by the caller (abacus_peer_comm_destroy).
+ * Errors: E_INVALID (1 <= nranks <= ABACUS_PEER_MAX, blob of this rank not
+ * from this ctx, no abacus_peer_export), E_CUDA. */
+int abacus_peer_comm_init(abacus_ctx* ctx, int32_t nranks, int32_t rank, const uint8_t* blobs, void** comm_out);
+/* Close the IPC mappings and free the communicator (NULL or an unknown
+ * pointer is a no-op). */
+void abacus_peer_comm_destroy(void* comm);
 
 /* ------------------------------------------------------------------------ */
 /* Introspection                                                             */

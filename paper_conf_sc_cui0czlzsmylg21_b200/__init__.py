@@ -31,7 +31,8 @@ EXPORTED = ["abacus_create", "abacus_destroy", "abacus_last_error", "abacus_load
             "abacus_encode_candidates", "abacus_encode_groups", "abacus_predict_batch",
             "abacus_select_group", "abacus_search", "abacus_search_batch", "abacus_search_mway", "abacus_search_grid", "abacus_search_sharded", "abacus_search_whatif",
             "abacus_combine_decisions", "abacus_nccl_unique_id",
-            "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_kernel_launches",
+            "abacus_nccl_comm_init", "abacus_nccl_comm_destroy", "abacus_peer_export", "abacus_peer_comm_init",
+            "abacus_peer_comm_destroy", "abacus_kernel_launches",
             "abacus_last_kernel_ms", "abacus_set_timing", "abacus_set_stream", "abacus_abi_version",
             "abacus_train_begin", "abacus_train_step", "abacus_train_epoch", "abacus_train_params"]
 
@@ -119,6 +120,10 @@ def lib():
         L.abacus_combine_decisions.argtypes = [P(abacus_decision_t), C.c_int32, C.c_int32, P(abacus_decision_t)]
         L.abacus_nccl_unique_id.argtypes = [P(C.c_uint8)]
         L.abacus_nccl_comm_init.argtypes = [vp, C.c_int32, C.c_int32, P(C.c_uint8), P(vp)]
+        L.abacus_peer_export.argtypes = [vp, P(C.c_uint8)]
+        L.abacus_peer_comm_init.argtypes = [vp, C.c_int32, C.c_int32, P(C.c_uint8), P(vp)]
+        L.abacus_peer_comm_destroy.argtypes = [vp]
+        L.abacus_peer_comm_destroy.restype = None
         L.abacus_nccl_comm_destroy.argtypes = [vp]
         L.abacus_nccl_comm_destroy.restype = None
         L.abacus_kernel_launches.argtypes = [vp]
@@ -320,6 +325,37 @@ def abacus_nccl_comm_init(ctx, nranks: int, rank: int, uid: bytes) -> int:
 
 def abacus_nccl_comm_destroy(comm: int) -> None:
     lib().abacus_nccl_comm_destroy(comm)
+
+
+PEER_BLOB = 128
+
+
+def abacus_peer_export(ctx) -> bytes:
+    buf = (C.c_uint8 * PEER_BLOB)()
+    _check(ctx, lib().abacus_peer_export(ctx, buf))
+    return bytes(buf)
+
+
+def abacus_peer_comm_init(ctx, nranks: int, rank: int, blobs: Sequence[bytes]) -> int:
+    raw = b"".join(blobs)
+    buf = (C.c_uint8 * len(raw))(*raw)
+    out = C.c_void_p()
+    _check(ctx, lib().abacus_peer_comm_init(ctx, nranks, rank, buf, C.byref(out)))
+    return out.value
+
+
+def abacus_peer_comm_destroy(comm: int) -> None:
+    lib().abacus_peer_comm_destroy(comm)
+
+
+def peer_comm_from_process_group(ctx, group=None) -> int:
+    """Every rank exports its mailbox, torch.distributed all-gathers the blobs,
+    every rank opens the others' mailboxes (CUDA IPC)."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, abacus_peer_export(ctx), group=group)
+    return abacus_peer_comm_init(ctx, world, rank, blobs)
 
 
 def abacus_kernel_launches(ctx) -> int:

@@ -16,6 +16,9 @@
 #include <atomic>
 #include <chrono>
 #include <cstdlib>
+#include <mutex>
+#include <set>
+#include <unistd.h>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -83,6 +86,8 @@ struct abacus_ctx {
     BatchA1* d_a1 = nullptr;
     int32_t* d_L = nullptr;        // device copy of the registry's op counts
     uint64_t* d_pairs = nullptr;   // [n] tile pairs per decision, then [n] = total
+    // a6 over peer memory: this rank's mailbox of kPeerMax tagged records (abacus_peer_export)
+    MappedRec* d_mailbox = nullptr;
     // what-if sweeps (NEXT-4): host-planned grid plans of up to kMaxSeg segments
     int32_t whatif_cap = 0;
     BatchDec* h_wdecs = nullptr;   // pinned
@@ -877,8 +882,30 @@ void host_decode(const Plan& P, Result& R) {
         R.end_op[j] = (R.key && j < P.k) ? decode_slot_ope(P, R.key & ((1ull << 40) - 1), j) : 0;
 }
 
+// ---- a6 over peer memory (abacus_peer_comm_init) ------------------------------
+struct PeerComm {
+    abacus_ctx* ctx = nullptr;
+    int32_t nranks = 0, rank = 0;
+    uint32_t seq = 0;                 // per-communicator launch counter (same on every rank)
+    PeerComb* d_comb = nullptr;       // device copy of the peer table
+    std::vector<void*> opened;        // IPC-opened peer mailboxes
+};
+std::mutex g_peer_mu;
+std::set<const void*> g_peer_comms;  // communicators this library created (type check of a void* comm)
+
+PeerComm* as_peer(void* comm) {
+    std::lock_guard<std::mutex> lk(g_peer_mu);
+    return g_peer_comms.count(comm) ? static_cast<PeerComm*>(comm) : nullptr;
+}
+
 // (nranks, rank) of an NCCL communicator (the NCCL copy the process already loaded)
 int comm_shape(abacus_ctx* c, void* comm, int* nranks, int* rank) {
+    if (PeerComm* pc = as_peer(comm)) {
+        if (pc->ctx != c) return fail(c, ABACUS_E_INVALID, "peer communicator of another ctx");
+        *nranks = pc->nranks;
+        *rank = pc->rank;
+        return ABACUS_OK;
+    }
     if (!nccl().ok) return fail(c, ABACUS_E_NCCL, "libnccl.so.2 not available");
     if (nccl().CommCount((ncclComm_t)comm, nranks) != ncclSuccess || *nranks < 1 || *nranks > 64 ||
         nccl().CommUserRank((ncclComm_t)comm, rank) != ncclSuccess || *rank < 0 || *rank >= *nranks)
@@ -1012,6 +1039,7 @@ void abacus_destroy(abacus_ctx* c) {
     if (c->h_wdecs) cudaFreeHost(c->h_wdecs);
     if (c->h_wsegs) cudaFreeHost(c->h_wsegs);
     cudaFree(c->d_wsegs);
+    cudaFree(c->d_mailbox);
     cudaFree(c->t_p);
     cudaFree(c->t_m);
     cudaFree(c->t_v);
@@ -1362,22 +1390,31 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
     CUDA_TRY(c, cudaSetDevice(c->device));
     Plan P = plan_grid_segments(c->n_models, c->D, grid, T, first, first + count, headroom_ms);
     const uint32_t seq = next_seq(c);
-    P.mapped = nccl_comm ? nullptr : c->dev_result;  // with a combine, the finalize kernel publishes
+    PeerComm* pc = nccl_comm ? as_peer(nccl_comm) : nullptr;
+    // with an NCCL combine the finalize kernel publishes; with a peer combine the
+    // fused kernel's last CTA combines and publishes itself
+    const bool nccl_combine = nccl_comm && !pc;
+    P.mapped = nccl_combine ? nullptr : c->dev_result;
     P.seq = seq;
     if (nccl_comm) {
         int nranks = 0, rank = 0;
         rc = comm_shape(c, nccl_comm, &nranks, &rank);
         if (rc) return rc;
     }
+    if (pc) {
+        P.peer = pc->d_comb;
+        P.peer_seq = ++pc->seq;
+    }
     rc = launch_fused(c, P);
     if (rc) return rc;
-    if (nccl_comm) {
+    if (nccl_combine) {
         rc = combine_over_comm(c, nccl_comm, seq);
         if (rc) return rc;
     }
     Result R;
     rc = wait_result(c, seq, &R);
     if (rc) return rc;
+    if (R.status == 3) return fail(c, ABACUS_E_NCCL, "peer combine: a rank's record did not arrive in time");
     if (!nccl_comm) host_decode(P, R);
     *out = sweep_decision(R, grid->k, headroom_ms);
     return ABACUS_OK;
@@ -1412,16 +1449,24 @@ int abacus_search_sharded(abacus_ctx* c, const abacus_query_t* q, int32_t k, dou
     const uint64_t last = (uint64_t)(rank + 1) * T / (uint64_t)nranks;
     Plan P;
     plan_grid_segments_into(static_cast<PlanHdr&>(P), PlanSink{&P}, c->n_models, c->D, &g, T, first, last, H);
-    P.mapped = nullptr;  // the finalize kernel publishes the combined record
+    PeerComm* pc = as_peer(nccl_comm);
+    P.mapped = pc ? c->dev_result : nullptr;  // the finalize kernel (NCCL) or the last CTA (peer) publishes
     P.seq = next_seq(c);
+    if (pc) {
+        P.peer = pc->d_comb;
+        P.peer_seq = ++pc->seq;
+    }
     CUDA_TRY(c, cudaSetDevice(c->device));
     rc = launch_fused(c, P);
     if (rc) return rc;
-    rc = combine_over_comm(c, nccl_comm, P.seq);
-    if (rc) return rc;
+    if (!pc) {
+        rc = combine_over_comm(c, nccl_comm, P.seq);
+        if (rc) return rc;
+    }
     Result R;
     rc = wait_result(c, P.seq, &R);
     if (rc) return rc;
+    if (R.status == 3) return fail(c, ABACUS_E_NCCL, "peer combine: a rank's record did not arrive in time");
     *out = assemble_decision(R, order, k, H, R.evaluated);
     return ABACUS_OK;
 }
@@ -1491,7 +1536,7 @@ int grow_whatif(abacus_ctx* c, int32_t n) {
 // segment sink into a what-if variant's fixed slots (host staging)
 struct ArraySink {
     SegP* segs;
-    void operator()(int i, const SegP& sg) const { segs[i] = sg; }
+    __host__ __device__ void operator()(int i, const SegP& sg) const { segs[i] = sg; }
 };
 }  // namespace
 
@@ -1754,6 +1799,129 @@ int abacus_nccl_comm_init(abacus_ctx* c, int32_t nranks, int32_t rank, const uin
 
 void abacus_nccl_comm_destroy(void* comm) {
     if (comm && nccl().ok) nccl().CommDestroy((ncclComm_t)comm);
+}
+
+// ---- a6 over peer memory ----------------------------------------------------
+// blob: [0, 64) cudaIpcMemHandle_t of the mailbox, [64, 72) pid, [72, 80) the
+// mailbox's device address in the exporting process, [80, 84) device ordinal,
+// [84, 88) magic
+static constexpr uint32_t kPeerMagic = 0x41425043u;  // "ABPC"
+
+int abacus_peer_export(abacus_ctx* c, uint8_t* blob) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!blob) return fail(c, ABACUS_E_INVALID, "NULL argument");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    if (!c->d_mailbox) {
+        CUDA_TRY(c, cudaMalloc(&c->d_mailbox, kPeerMax * sizeof(MappedRec)));
+        CUDA_TRY(c, cudaMemset(c->d_mailbox, 0, kPeerMax * sizeof(MappedRec)));
+    }
+    memset(blob, 0, ABACUS_PEER_BLOB);
+    cudaIpcMemHandle_t h;
+    CUDA_TRY(c, cudaIpcGetMemHandle(&h, c->d_mailbox));
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+    memcpy(blob, &h, 64);
+    const uint64_t pid = (uint64_t)getpid(), addr = (uint64_t)(uintptr_t)c->d_mailbox;
+    const int32_t dev = c->device;
+    memcpy(blob + 64, &pid, 8);
+    memcpy(blob + 72, &addr, 8);
+    memcpy(blob + 80, &dev, 4);
+    memcpy(blob + 84, &kPeerMagic, 4);
+    return ABACUS_OK;
+}
+
+int abacus_peer_comm_init(abacus_ctx* c, int32_t nranks, int32_t rank, const uint8_t* blobs, void** comm_out) {
+    if (!c) return ABACUS_E_INVALID;
+    c->err.clear();
+    if (!blobs || !comm_out || nranks < 1 || nranks > kPeerMax || rank < 0 || rank >= nranks)
+        return fail(c, ABACUS_E_INVALID, "bad peer communicator arguments (1 <= nranks <= %d)", kPeerMax);
+    if (!c->d_mailbox) return fail(c, ABACUS_E_INVALID, "abacus_peer_export was not called on this ctx");
+    CUDA_TRY(c, cudaSetDevice(c->device));
+    PeerComm* pc = new PeerComm();
+    pc->ctx = c;
+    pc->nranks = nranks;
+    pc->rank = rank;
+    PeerComb hc{};
+    hc.nranks = nranks;
+    hc.rank = rank;
+    const char* e = getenv("ABACUS_PEER_TIMEOUT_MS");
+    hc.timeout_ms = e && atoi(e) > 0 ? (uint32_t)atoi(e) : 10000u;
+    hc.local = c->d_mailbox;
+    auto cleanup = [&]() {
+        for (void* p : pc->opened) cudaIpcCloseMemHandle(p);
+        delete pc;
+    };
+    for (int32_t r = 0; r < nranks; r++) {
+        const uint8_t* b = blobs + (size_t)r * ABACUS_PEER_BLOB;
+        uint64_t pid, addr;
+        int32_t dev;
+        uint32_t magic;
+        memcpy(&pid, b + 64, 8);
+        memcpy(&addr, b + 72, 8);
+        memcpy(&dev, b + 80, 4);
+        memcpy(&magic, b + 84, 4);
+        if (magic != kPeerMagic) {
+            cleanup();
+            return fail(c, ABACUS_E_INVALID, "rank %d: not a peer blob", r);
+        }
+        if (r == rank) {
+            if (pid != (uint64_t)getpid() || addr != (uint64_t)(uintptr_t)c->d_mailbox) {
+                cleanup();
+                return fail(c, ABACUS_E_INVALID, "rank %d's blob is not this ctx's", r);
+            }
+            hc.dst[r] = c->d_mailbox;
+        } else if (pid == (uint64_t)getpid()) {
+            // same process (tests: two ctxs on one device): the address is valid
+            // here; another device needs peer access
+            if (dev != c->device) {
+                const cudaError_t pe = cudaDeviceEnablePeerAccess(dev, 0);
+                if (pe != cudaSuccess && pe != cudaErrorPeerAccessAlreadyEnabled) {
+                    cleanup();
+                    return fail(c, ABACUS_E_CUDA, "peer access to device %d: %s", dev, cudaGetErrorString(pe));
+                }
+                cudaGetLastError();
+            }
+            hc.dst[r] = reinterpret_cast<MappedRec*>((uintptr_t)addr);
+        } else {
+            cudaIpcMemHandle_t h;
+            memcpy(&h, b, 64);
+            void* ptr = nullptr;
+            const cudaError_t oe = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+            if (oe != cudaSuccess) {
+                cleanup();
+                return fail(c, ABACUS_E_CUDA, "rank %d: cudaIpcOpenMemHandle: %s", r, cudaGetErrorString(oe));
+            }
+            pc->opened.push_back(ptr);
+            hc.dst[r] = static_cast<MappedRec*>(ptr);
+        }
+    }
+    if (cudaMalloc(&pc->d_comb, sizeof(PeerComb)) != cudaSuccess ||
+        cudaMemcpy(pc->d_comb, &hc, sizeof(PeerComb), cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaFree(pc->d_comb);
+        cleanup();
+        return fail(c, ABACUS_E_CUDA, "peer table allocation failed");
+    }
+    {
+        std::lock_guard<std::mutex> lk(g_peer_mu);
+        g_peer_comms.insert(pc);
+    }
+    *comm_out = pc;
+    return ABACUS_OK;
+}
+
+void abacus_peer_comm_destroy(void* comm) {
+    PeerComm* pc = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(g_peer_mu);
+        if (!comm || !g_peer_comms.count(comm)) return;
+        g_peer_comms.erase(comm);
+        pc = static_cast<PeerComm*>(comm);
+    }
+    cudaSetDevice(pc->ctx->device);
+    cudaStreamSynchronize(pc->ctx->stream);
+    for (void* p : pc->opened) cudaIpcCloseMemHandle(p);
+    cudaFree(pc->d_comb);
+    delete pc;
 }
 
 // not in the ABI header (tools/kernel_trace.py): device array of 8 globaltimer

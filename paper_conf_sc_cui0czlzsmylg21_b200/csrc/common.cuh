@@ -161,6 +161,21 @@ __host__ __device__ inline Result combine_results(const Result* r, int n) {
 
 enum PlanMode : int32_t { kModeGrid = 0, kModeChain = 1 };
 
+// a6 over peer memory (abacus_peer_comm_init): every rank owns a mailbox of
+// kPeerMax tagged records in its device memory; the last CTA of a rank's fused
+// search writes its record into slot `rank` of every rank's mailbox (P2P stores
+// through NVLink, or plain stores when the ranks share a device), then waits in
+// its own mailbox for every rank's record of the same sequence number and
+// combines them (combine_results) -- compute and collective in one kernel.
+constexpr int kPeerMax = 32;  // ABACUS_PEER_MAX
+struct PeerComb {
+    int32_t nranks, rank;
+    uint32_t timeout_ms;         // give up waiting for a peer after this long (status 3)
+    uint32_t pad;
+    MappedRec* local;            // this rank's mailbox (kPeerMax slots)
+    MappedRec* dst[kPeerMax];    // every rank's mailbox as mapped into this process
+};
+
 // header of a plan: everything but the segment table (decode of t*, a7)
 struct PlanHdr {
     int32_t k, n_seg, n_models, D;
@@ -175,7 +190,8 @@ struct PlanHdr {
     MappedRec* mapped;      // host-mapped pinned result record (device pointer) or null
     unsigned long long* trace;  // optional %globaltimer stamps (tools only), null in production
     uint32_t seq;           // sequence number the mapped copy is tagged with
-    uint32_t pad2;
+    uint32_t peer_seq;      // tag of this launch's records in the peer mailboxes (with `peer`)
+    const struct PeerComb* peer;  // in-kernel cross-GPU combine (a6 over peer memory) or null
     SlotP slot[kKMax];
 };
 

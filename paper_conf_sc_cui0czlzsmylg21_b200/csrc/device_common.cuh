@@ -349,6 +349,86 @@ __device__ __forceinline__ void publish_mapped(const Result& R, MappedRec* M, ui
                      : "memory");
 }
 
+// device-side reader of a tagged record (the host's rec_read): volatile 16-byte
+// loads, true once all four chunks carry the tag of `seq`
+__device__ __forceinline__ bool rec_read_dev(const MappedRec* M, uint32_t seq, uint32_t (&p)[12]) {
+    bool ok = true;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        uint32_t a, b, c, t;
+        asm volatile("ld.volatile.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(a), "=r"(b), "=r"(c), "=r"(t)
+                     : "l"(&M->w[4 * i])
+                     : "memory");
+        ok = ok && t == rec_tag(seq, a, b, c, (uint32_t)i);
+        p[3 * i] = a;
+        p[3 * i + 1] = b;
+        p[3 * i + 2] = c;
+    }
+    return ok;
+}
+
+// a6 over peer memory, run by warp 0 of the last CTA with this rank's record R
+// (every lane holds it): lane l sends R to rank l's mailbox, then waits for
+// rank l's record in the local mailbox; the warp combines the nranks records
+// exactly as combine_results does (max key with its y / end ops, evaluated
+// summed, y(0) from the lowest rank that holds index 0).  A rank missing after
+// the timeout makes the result status 3.
+static __device__ __noinline__ Result peer_combine(const PeerComb& C, const Result& R, uint32_t seq) {
+    const uint32_t lane = threadIdx.x & 31;
+    const bool act = lane < (uint32_t)C.nranks;
+    if (act) {
+        publish_mapped(R, C.dst[lane] + C.rank, seq);
+        asm volatile("fence.acq_rel.sys;" ::: "memory");
+    }
+    Result mine{};
+    mine.y0 = __int_as_float(0x7fc00000);
+    bool timed_out = false;
+    if (act) {
+        unsigned long long t0, t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        const unsigned long long limit = (unsigned long long)C.timeout_ms * 1000000ull;
+        uint32_t p[12];
+        for (;;) {
+            if (rec_read_dev(C.local + lane, seq, p)) break;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            if (t - t0 > limit) {
+                timed_out = true;
+                break;
+            }
+            __nanosleep(64);
+        }
+        if (!timed_out) rec_unpayload(p, mine);
+    }
+    // combine across the lanes (rank order = lane order)
+    unsigned long long bk = mine.key;
+    uint32_t win = lane;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long k2 = __shfl_xor_sync(0xffffffffu, bk, o);
+        const uint32_t w2 = __shfl_xor_sync(0xffffffffu, win, o);
+        if (k2 > bk || (k2 == bk && w2 < win)) { bk = k2; win = w2; }
+    }
+    unsigned long long ev = mine.evaluated;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) ev += __shfl_xor_sync(0xffffffffu, ev, o);
+    const uint32_t has_y0 = __ballot_sync(0xffffffffu, act && mine.y0 == mine.y0);
+    const float y0 = __shfl_sync(0xffffffffu, mine.y0, has_y0 ? __ffs(has_y0) - 1 : 0);
+    const uint32_t bad = __ballot_sync(0xffffffffu, timed_out);
+    Result out;
+    out.key = bk;
+    out.y_best = __shfl_sync(0xffffffffu, mine.y_best, win);
+    out.y0 = has_y0 ? y0 : __int_as_float(0x7fc00000);
+    out.evaluated = ev;
+#pragma unroll
+    for (int j = 0; j < kKMax; j++) out.end_op[j] = __shfl_sync(0xffffffffu, mine.end_op[j], win);
+    out.total_ops = __shfl_sync(0xffffffffu, mine.total_ops, win);
+    out.status = bad ? 3 : (bk ? 0 : 2);
+    out.seq = 0;
+    out.pad = 0;
+    return out;
+}
+
 static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratch* S, unsigned long long key, float y) {
     __shared__ unsigned long long s_key[32];
     __shared__ float s_y[32];
@@ -411,12 +491,30 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
         trace_stamp(P, 9);
         // a7: lane j decodes slot j's end op of t*; a record that goes to host-mapped
         // memory is decoded by the host instead (off the kernel's critical path)
-        const int32_t my_ope = (!P.mapped && threadIdx.x < (unsigned)P.k && bk)
+        const int32_t my_ope = ((!P.mapped || P.peer) && threadIdx.x < (unsigned)P.k && bk)
                                    ? decode_slot_ope(P, bk & ((1ull << 40) - 1), (int)threadIdx.x)
                                    : 0;
         int32_t ope[kKMax];
 #pragma unroll
         for (int j = 0; j < kKMax; j++) ope[j] = __shfl_sync(0xffffffffu, my_ope, j);
+        if (P.peer) {
+            // this rank's record, then the in-kernel combine over the peers' mailboxes
+            Result R{};
+            R.key = bk;
+            R.y_best = by;
+            R.y0 = y0;
+            R.evaluated = P.n_eval;
+            for (int j = 0; j < kKMax; j++) R.end_op[j] = ope[j];
+            R.total_ops = bk ? (int32_t)(bk >> 40) - 1 : 0;
+            R.status = bk ? 0 : 2;
+            const Result G = peer_combine(*P.peer, R, P.peer_seq);
+            if (threadIdx.x != 0) return;
+            S->result = G;
+            S->y0 = __int_as_float(0x7fc00000);
+            S->counter = 0;
+            if (P.mapped) publish_mapped(G, P.mapped, P.seq);
+            return;
+        }
         if (threadIdx.x != 0) return;
         trace_stamp(P, 10);
         Result& R = S->result;
