@@ -321,7 +321,11 @@ def main():
     sharded = None
     sharded_peer = None
     if not args.no_decisions:
-        sharded = sharded_decision_latency(ab, ctx, comm, world, rank)
+        # at N = 1 through a one-rank NCCL communicator: the sharded path as it runs at N > 1
+        ncomm = comm if world > 1 else ab.abacus_nccl_comm_init(ctx, 1, 0, ab.abacus_nccl_unique_id())
+        sharded = sharded_decision_latency(ab, ctx, ncomm, world, rank)
+        if world == 1:
+            ab.abacus_nccl_comm_destroy(ncomm)
         # the same decisions with the combine inside the search kernel (peer mailboxes,
         # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator)
         pcomm = ab.peer_comm_from_process_group(ctx) if world > 1 else \
@@ -478,7 +482,7 @@ def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50, label=
     """Per-decision latency of abacus_search_sharded on config-3 4-way pure
     GRID decisions (up to 4.1e7 candidates each): every rank searches its
     contiguous shard of each decision's grid and one all-gather combines them
-    (SURVEY §8(d)/(e)).  At N = 1 there is no communicator (the local search).
+    (SURVEY §8(d)/(e)).  At N = 1 the communicator has one rank.
     Host clock around each blocking call on every rank; the per-decision time
     is the max over ranks."""
     import torch
@@ -503,7 +507,7 @@ def sharded_decision_latency(ab, ctx, comm, world, rank, n=3000, warm=50, label=
             "max_us": float(a.max()), "grid_p50": float(np.percentile(ev, 50)), "grid_p99": float(np.percentile(ev, 99)),
             "grid_max": float(ev.max()),
             "path": "Python binding -> abacus_search_sharded (%s)" % (
-                ("NCCL all-gather over %d ranks" % world if world > 1 else "1 GPU, no collective")
+                "NCCL all-gather + finalize kernel over %d rank%s" % (world, "s" if world > 1 else "")
                 if label == "nccl" else
                 "combine inside the search kernel over %d ranks' peer mailboxes" % world)}
 

@@ -60,6 +60,15 @@ def main():
             ab.abacus_select_group(ctx, grid, 5, n, y, 30.0, key, st)
             torch.cuda.synchronize()
             print("encode/predict/select", prec, float(y[:4].sum()), int(key.item()), flush=True)
+    if "peer" not in skip:
+        # the in-kernel cross-GPU combine with a one-rank peer communicator
+        ab.abacus_load_predictor(ctx, params, ab.ABACUS_FP16)
+        pc = ab.abacus_peer_comm_init(ctx, 1, 0, [ab.abacus_peer_export(ctx)])
+        d = ab.abacus_search_grid(ctx, grid, 30.0, 100, T - 200, pc)
+        qs, now, infl = decs[2]
+        d2 = ab.abacus_search_sharded(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID, 2**40, pc)
+        ab.abacus_peer_comm_destroy(pc)
+        print("peer", d.key, d2.key, flush=True)
     if "groups" not in skip:
         G = synth.instance_samples(300, seed=3)
         raw = ab.make_groups([g.slots for g in G])
