@@ -243,6 +243,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-decisions", action="store_true")
     ap.add_argument("--no-secondary", action="store_true", help="skip the bf16 / fp32 sweep keys")
+    ap.add_argument("--combine", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1 sweep combine: NCCL all-gather + finalize kernel, or inside the search kernel")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -276,7 +278,9 @@ def main():
     torch.cuda.set_stream(stream)
     ab.abacus_set_stream(ctx, stream)
     ab.abacus_set_timing(ctx, True)
-    comm = ab.nccl_comm_from_process_group(ctx) if world > 1 else None
+    comm = None
+    if world > 1:
+        comm = ab.nccl_comm_from_process_group(ctx) if args.combine == "nccl" else ab.peer_comm_from_process_group(ctx)
 
     for _ in range(args.warmup):
         d = ab.abacus_search_grid(ctx, grid, H, first, count, comm)
@@ -322,9 +326,12 @@ def main():
     sharded_peer = None
     if not args.no_decisions:
         # at N = 1 through a one-rank NCCL communicator: the sharded path as it runs at N > 1
-        ncomm = comm if world > 1 else ab.abacus_nccl_comm_init(ctx, 1, 0, ab.abacus_nccl_unique_id())
+        if world > 1:
+            ncomm = comm if args.combine == "nccl" else ab.nccl_comm_from_process_group(ctx)
+        else:
+            ncomm = ab.abacus_nccl_comm_init(ctx, 1, 0, ab.abacus_nccl_unique_id())
         sharded = sharded_decision_latency(ab, ctx, ncomm, world, rank)
-        if world == 1:
+        if ncomm is not comm:
             ab.abacus_nccl_comm_destroy(ncomm)
         # the same decisions with the combine inside the search kernel (peer mailboxes,
         # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator)
@@ -374,7 +381,7 @@ def main():
             "metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed / args.steps * 1e3, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[args.precision], "data": "synthetic",
-            "config": arm_config(T, H, args.precision, world),
+            "config": dict(arm_config(T, H, args.precision, world), combine=args.combine if world > 1 else None),
             "per_gpu": value / world,
             "selected": {"key": d.key, "index": d.index, "total_ops": d.total_ops, "pred_ms": d.pred_ms,
                          "end_op": list(d.end_op)},
@@ -401,7 +408,7 @@ def main():
         # down the library's communicator together (ncclCommDestroy finalizes)
         dist.barrier()
     if comm:
-        ab.abacus_nccl_comm_destroy(comm)
+        (ab.abacus_nccl_comm_destroy if args.combine == "nccl" else ab.abacus_peer_comm_destroy)(comm)
     ab.abacus_destroy(ctx)
     if world > 1:
         dist.destroy_process_group()
