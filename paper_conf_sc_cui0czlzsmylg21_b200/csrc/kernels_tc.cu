@@ -233,6 +233,10 @@ struct TcPipe {
     uint32_t tCx, tCy, lane_off, bar_id, ph;  // bias constant chunk of X / Y (may be shared)
     uint64_t* bar;
     uint64_t db2, db3, db4;
+#ifndef EXP_NO_PRE
+    uint64_t db2u, db3u, db4u;  // the layers' second K chunk
+    uint32_t xa8, ya8;          // the second half of A
+#endif
 
     uint32_t hb_smem;  // fp16: shared address of layer 2's bias words (layer 3's follow one blob later)
     bool me[4];
@@ -287,6 +291,18 @@ struct TcPipe {
         asm volatile("mov.b64 %0, %0;" : "+l"(db2));
         asm volatile("mov.b64 %0, %0;" : "+l"(db3));
         asm volatile("mov.b64 %0, %0;" : "+l"(db4));
+#ifndef EXP_NO_PRE
+        db2u = db2 + (kChunkBytesN32 >> 4);
+        db3u = db3 + (kChunkBytesN32 >> 4);
+        db4u = db4 + (kChunkBytesN16 >> 4);
+        xa8 = X.a + 8;
+        ya8 = Y.a + 8;
+        asm volatile("mov.b64 %0, %0;" : "+l"(db2u));
+        asm volatile("mov.b64 %0, %0;" : "+l"(db3u));
+        asm volatile("mov.b64 %0, %0;" : "+l"(db4u));
+        asm volatile("mov.b32 %0, %0;" : "+r"(xa8));
+        asm volatile("mov.b32 %0, %0;" : "+r"(ya8));
+#endif
 
         // fp16: the bias chunk of each hidden layer holds its 16 f16 bias pairs instead
         hb_smem = ((uint32_t)(d2 & 0x3FFFu) << 4) + 2u * kChunkBytesN32;
@@ -352,6 +368,14 @@ struct TcPipe {
             return;
         }
         // fp16: no bias MMA in any layer (hidden biases in the f16 epilogue, b4 in fp32)
+#ifndef EXP_NO_PRE
+        // every issue operand precomputed (+0.9 % on config 4)
+        if (TWO) {
+            const uint64_t dbu = LAYER == 0 ? db2u : (LAYER == 1 ? db3u : db4u);
+            issue_pair2_pre<ID>(X.d, X.a, xa8, Y.d, Y.a, ya8, db, dbu, bar);
+            return;
+        }
+#endif
         if (TWO) issue_layer2_asm<0, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
         else issue_layer_asm<0, ID, CH, false>(X.d, X.a, tCx, db, bar);
     }

@@ -318,6 +318,28 @@ __device__ __forceinline__ void issue_layer2_asm(uint32_t tDx, uint32_t tAx, uin
         : "memory");
 }
 
+// issue_layer2_asm<.., false> with every operand precomputed by the caller
+// (the second A half, the second chunk's descriptor): no address arithmetic
+// between the barrier and the MMAs
+template <uint32_t IDESC>
+__device__ __forceinline__ void issue_pair2_pre(uint32_t tDx, uint32_t tAx, uint32_t tAx8, uint32_t tDy, uint32_t tAy,
+                                                uint32_t tAy8, uint64_t d0, uint64_t d1, uint64_t* bar) {
+    asm volatile(
+        "{\n\t"
+        ".reg .pred e, pf, pt;\n\t"
+        "setp.ne.b32 pf, 0, 0;\n\t"
+        "setp.eq.b32 pt, 0, 0;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %6, %9, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], %7, %9, pt;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%4], %6, %9, pf;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%5], %7, %9, pt;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%8];\n\t"
+        "}" ::"r"(tDx),
+        "r"(tAx), "r"(tAx8), "r"(tDy), "r"(tAy), "r"(tAy8), "l"(d0), "l"(d1), "r"(smem_u32(bar)), "n"(IDESC)
+        : "memory");
+}
+
 // bf16 layer for TWO tiles: hi chunks 0, 1, lo chunks 2, 3 (W = W_hi + W_lo)
 // and (BIAS) the bias chunk 4, one commit
 template <uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
