@@ -566,10 +566,20 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     pp.zero_a();
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
+#ifndef EXP_NO_SEGLO
+    // the segment's table descriptor differs from d1base only in its low word (the
+    // start address field, < 2^14): one shuffle of that word, no 64-bit arithmetic
+    const uint32_t d1lo = (uint32_t)d1base, d1hi = (uint32_t)(d1base >> 32);
+    auto issue_l1 = [&](const TileIO& T, int s) {
+        const uint32_t lo = __shfl_sync(0xffffffffu, d1lo + (uint32_t)s * kSegStep, 0);
+        pp.issue_l1(T, ((uint64_t)d1hi << 32) | lo);
+    };
+#else
     auto issue_l1 = [&](const TileIO& T, int s) {
         const int su = __shfl_sync(0xffffffffu, s, 0);
         pp.issue_l1(T, d1base + (uint64_t)((uint32_t)su * kSegStep));
     };
+#endif
     using T1 = std::integral_constant<bool, false>;
     using T2 = std::integral_constant<bool, true>;
 
