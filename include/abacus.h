@@ -396,7 +396,8 @@ void abacus_nccl_comm_destroy(void* comm);
 /* ------------------------------------------------------------------------ */
 /* Instead of an ncclComm_t, abacus_search_grid and abacus_search_sharded
  * accept a peer communicator from abacus_peer_comm_init.  Each rank owns a
- * device mailbox of ABACUS_PEER_MAX tagged 64-byte records.  The last CTA of
+ * device mailbox of 2 x ABACUS_PEER_MAX tagged 64-byte records (two banks by
+ * launch parity).  The last CTA of
  * a rank's fused search writes its 56-byte result into slot `rank` of every
  * rank's mailbox (peer stores: NVLink between GPUs, plain stores between
  * ctxs of one device), then waits in its own mailbox for every rank's record

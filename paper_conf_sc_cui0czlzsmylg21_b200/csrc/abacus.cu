@@ -1813,8 +1813,8 @@ int abacus_peer_export(abacus_ctx* c, uint8_t* blob) {
     if (!blob) return fail(c, ABACUS_E_INVALID, "NULL argument");
     CUDA_TRY(c, cudaSetDevice(c->device));
     if (!c->d_mailbox) {
-        CUDA_TRY(c, cudaMalloc(&c->d_mailbox, kPeerMax * sizeof(MappedRec)));
-        CUDA_TRY(c, cudaMemset(c->d_mailbox, 0, kPeerMax * sizeof(MappedRec)));
+        CUDA_TRY(c, cudaMalloc(&c->d_mailbox, 2 * kPeerMax * sizeof(MappedRec)));
+        CUDA_TRY(c, cudaMemset(c->d_mailbox, 0, 2 * kPeerMax * sizeof(MappedRec)));
     }
     memset(blob, 0, ABACUS_PEER_BLOB);
     cudaIpcMemHandle_t h;

@@ -172,7 +172,7 @@ struct PeerComb {
     int32_t nranks, rank;
     uint32_t timeout_ms;         // give up waiting for a peer after this long (status 3)
     uint32_t pad;
-    MappedRec* local;            // this rank's mailbox (kPeerMax slots)
+    MappedRec* local;            // this rank's mailbox (2 banks of kPeerMax slots)
     MappedRec* dst[kPeerMax];    // every rank's mailbox as mapped into this process
 };
 

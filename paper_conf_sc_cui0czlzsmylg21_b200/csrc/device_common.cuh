@@ -377,8 +377,13 @@ __device__ __forceinline__ bool rec_read_dev(const MappedRec* M, uint32_t seq, u
 static __device__ __noinline__ Result peer_combine(const PeerComb& C, const Result& R, uint32_t seq) {
     const uint32_t lane = threadIdx.x & 31;
     const bool act = lane < (uint32_t)C.nranks;
+    // two banks by launch parity: a rank that finished launch k and started k + 1
+    // writes the other bank, so it never overwrites a launch-k record a slower
+    // rank has not read yet (it cannot get two launches ahead: launch k + 1
+    // needs every rank's k + 1 record)
+    const uint32_t bank = (seq & 1u) * (uint32_t)kPeerMax;
     if (act) {
-        publish_mapped(R, C.dst[lane] + C.rank, seq);
+        publish_mapped(R, C.dst[lane] + bank + C.rank, seq);
         asm volatile("fence.acq_rel.sys;" ::: "memory");
     }
     Result mine{};
@@ -390,7 +395,7 @@ static __device__ __noinline__ Result peer_combine(const PeerComb& C, const Resu
         const unsigned long long limit = (unsigned long long)C.timeout_ms * 1000000ull;
         uint32_t p[12];
         for (;;) {
-            if (rec_read_dev(C.local + lane, seq, p)) break;
+            if (rec_read_dev(C.local + bank + lane, seq, p)) break;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
             if (t - t0 > limit) {
                 timed_out = true;
