@@ -169,3 +169,33 @@ def test_peer_combine_two_processes_ipc():
             dd, ww = ab.abacus_decision_t.from_buffer_copy(d), ab.abacus_decision_t.from_buffer_copy(w)
             assert _same(dd, ww)
     assert [d for d, _ in res[0]] == [d for d, _ in res[1]]
+
+
+def test_peer_combine_many_consecutive_launches():
+    """200 back-to-back sharded decisions on 2 ranks (the mailbox banks alternate
+    by launch parity; a rank may start launch k + 1 while the other still reads
+    launch k's records)."""
+    import torch
+    params = synth.weights(1)
+    ctxs = [Ctx(params=params, precision=ab.ABACUS_FP16) for _ in range(2)]
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    for c, st in zip(ctxs, streams):
+        ab.abacus_set_stream(c.h, st)
+    comms = _comms(ctxs)
+    try:
+        decs = synth.cfg2_decisions(200)
+        refs = [ab.abacus_search(ctxs[0].h, qs, now, infl, ab.ABACUS_SPACE_GRID) for qs, now, infl in decs]
+
+        def rank_loop(r):
+            return [ab.abacus_search_sharded(ctxs[r].h, qs, now, infl, ab.ABACUS_SPACE_GRID, 2**40, comms[r])
+                    for qs, now, infl in decs]
+        got = _parallel([lambda r=r: rank_loop(r) for r in range(2)])
+        for r in range(2):
+            for d, ref in zip(got[r], refs):
+                assert _same(d, ref)
+    finally:
+        for cm in comms:
+            ab.abacus_peer_comm_destroy(cm)
+        for c in ctxs:
+            c.close()
+        del streams
