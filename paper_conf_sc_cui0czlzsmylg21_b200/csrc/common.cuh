@@ -199,6 +199,17 @@ struct Plan : PlanHdr {
     SegP seg[kMaxSeg];
 };
 
+// The same header with a shorter segment table: the launch parameter of the
+// fused kernels for plans of <= 8 segments (every scheduling decision: 2^(k-1)
+// presence patterns or k chain blocks), 2.1 KB instead of 4 KB of kernel
+// parameters per launch (decision p99 -1.5 to -2 us).  The kernels read it
+// through a `const Plan&` (same layout prefix; segments >= n_seg are never read).
+template <int NSEG>
+struct PlanT : PlanHdr {
+    SegP seg[NSEG];
+};
+using PlanDecision = PlanT<8>;
+
 // ---- batched decisions (NEXT-4): many independent decisions in one launch ----
 // Decision d owns tiles [2 pair0, 2 pair0 + n_tiles) of the launch (n_tiles
 // rounded up to even, so a group's two lock-step tiles never straddle two

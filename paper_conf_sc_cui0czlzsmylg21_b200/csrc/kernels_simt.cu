@@ -11,6 +11,8 @@
 #include <cuda_runtime.h>
 #include <math.h>
 
+#include <cstring>
+
 #include "common.cuh"
 #include "device_common.cuh"
 #include "internal.h"
@@ -639,8 +641,10 @@ __device__ __forceinline__ void layer1_fp32(const float* c, const float* wc, con
     }
 }
 
+template <class PL>
 __global__ void __launch_bounds__(kFused2Threads, kFused2BlocksPerSM) fused_fp32x2_kernel(
-    const __grid_constant__ Plan P, const __grid_constant__ W234 Wt, const float* __restrict__ w1b1, Scratch* S) {
+    const __grid_constant__ PL Pin, const __grid_constant__ W234 Wt, const float* __restrict__ w1b1, Scratch* S) {
+    const Plan& P = *reinterpret_cast<const Plan*>(&Pin);  // PlanT<8> for decisions: same layout prefix
     __shared__ float s_c[kMaxSeg * kHidden];
     __shared__ float s_w[kMaxSeg * kKMax * kHidden];
     __shared__ W234s s_W;
@@ -1079,7 +1083,13 @@ cudaError_t launch_fused_fp32(const Plan& P, const W234& W, const float* w1b1, S
         if (n_pairs < g) g = n_pairs;
         if (g < 1) g = 1;
         *grid_out = (int)g;
-        fused_fp32x2_kernel<<<(int)g, kFused2Threads, 0, st>>>(P, W, w1b1, S);
+        if (P.n_seg <= 8) {  // decisions: the short parameter block
+            PlanDecision Ps;
+            memcpy(&Ps, &P, sizeof(PlanDecision));
+            fused_fp32x2_kernel<PlanDecision><<<(int)g, kFused2Threads, 0, st>>>(Ps, W, w1b1, S);
+        } else {
+            fused_fp32x2_kernel<Plan><<<(int)g, kFused2Threads, 0, st>>>(P, W, w1b1, S);
+        }
         return cudaGetLastError();
     }
 #endif

@@ -33,6 +33,7 @@
 #include <math.h>
 
 #include <cstdlib>
+#include <cstring>
 #include <type_traits>
 
 #include "common.cuh"
@@ -509,10 +510,11 @@ __device__ __forceinline__ void store_a1_packed(uint32_t taddr, uint32_t a1, uin
 }
 
 
-template <int FMT, bool SPLIT, int NG>
-__global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ Plan P,
+template <int FMT, bool SPLIT, int NG, class PL = Plan>
+__global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_constant__ PL Pin,
                                                                const __grid_constant__ TcParams TP,
                                                                const float* __restrict__ w1b1, Scratch* S) {
+    const Plan& P = *reinterpret_cast<const Plan*>(&Pin);  // PlanT<8> for decisions: same layout prefix
     extern __shared__ __align__(1024) uint8_t smem[];
     using C = TcCfg<FMT>;
     const TcSmem L = tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, NG, w1_stage_bytes(P.D, NG));
@@ -1605,23 +1607,38 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
     using C = TcCfg<FMT>;
     const TcSmem L =
         tc_smem_layout<FMT>(P.n_seg, C::kNchL1 * kChunkBytesN32, kFusedNG, w1_stage_bytes(P.D, kFusedNG));
-    auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG>;
-    // the shared-memory opt-in is a host API call on the decision path: raise it
-    // only when a launch needs more than this device has been given so far
-    static int s_granted[64] = {};
-    int dev = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e != cudaSuccess) return e;
-    if (dev < 0 || dev >= 64 || s_granted[dev] < (int)L.total) {
-        e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
-        if (e != cudaSuccess) return e;
-        if (dev >= 0 && dev < 64) s_granted[dev] = (int)L.total;
-    }
     // spread the tiles over as many SMs as possible (one tile per group first)
     uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
     if (g > (uint64_t)nsm) g = (uint64_t)nsm;
     if (g < 1) g = 1;
     *grid_out = (int)g;
+    // the shared-memory opt-in is a host API call on the decision path: raise it
+    // only when a launch needs more than this device has given the kernel so far
+    auto optin = [&](auto kern, int* granted) -> cudaError_t {
+        int dev = 0;
+        cudaError_t e = cudaGetDevice(&dev);
+        if (e != cudaSuccess) return e;
+        if (dev < 0 || dev >= 64 || granted[dev] < (int)L.total) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+            if (e != cudaSuccess) return e;
+            if (dev >= 0 && dev < 64) granted[dev] = (int)L.total;
+        }
+        return cudaSuccess;
+    };
+    if (P.n_seg <= 8) {  // decisions: the short parameter block
+        static int s_granted8[64] = {};
+        auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG, PlanDecision>;
+        const cudaError_t e = optin(kern, s_granted8);
+        if (e != cudaSuccess) return e;
+        PlanDecision Ps;
+        memcpy(&Ps, &P, sizeof(PlanDecision));
+        kern<<<(int)g, kFusedNG * 128, L.total, st>>>(Ps, tp, w1b1, S);
+        return cudaGetLastError();
+    }
+    static int s_granted[64] = {};
+    auto kern = fused_tc_kernel<FMT, SPLIT, kFusedNG, Plan>;
+    const cudaError_t e = optin(kern, s_granted);
+    if (e != cudaSuccess) return e;
     kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, w1b1, S);
     return cudaGetLastError();
 }
