@@ -26,10 +26,26 @@ def build(force: bool = False, verbose: bool = False) -> str:
     deps = [os.path.join(CSRC, f) for f in SOURCES + HEADERS]
     deps.append(os.path.join(os.path.dirname(HERE), "include", "abacus.h"))
     if force or _stale(LIB, deps):
-        cmd = [NVCC] + ARCH + FLAGS + ["-o", LIB] + [os.path.join(CSRC, f) for f in SOURCES] + ["-ldl"]
-        if verbose:
-            print(" ".join(cmd))
-        subprocess.check_call(cmd)
+        # one nvcc per translation unit, in parallel (no device code crosses files:
+        # the kernels' helpers are header-inline), then one link
+        import tempfile
+        with tempfile.TemporaryDirectory() as tmp:
+            objs, procs = [], []
+            cflags = [f for f in FLAGS if f != "-shared"]
+            for f in SOURCES:
+                o = os.path.join(tmp, f + ".o")
+                cmd = [NVCC] + ARCH + cflags + ["-c", "-o", o, os.path.join(CSRC, f)]
+                if verbose:
+                    print(" ".join(cmd))
+                procs.append((subprocess.Popen(cmd), cmd))
+                objs.append(o)
+            for p, cmd in procs:
+                if p.wait() != 0:
+                    raise subprocess.CalledProcessError(p.returncode, cmd)
+            cmd = [NVCC] + ARCH + ["-shared", "-Xcompiler", "-fPIC", "-o", LIB] + objs + ["-ldl"]
+            if verbose:
+                print(" ".join(cmd))
+            subprocess.check_call(cmd)
     pdeps = [os.path.join(CSRC, "probe_umma.cu"), os.path.join(CSRC, "tc_ptx.cuh")]
     if force or _stale(PROBE_LIB, pdeps):
         cmd = [NVCC] + ARCH + FLAGS + ["-o", PROBE_LIB, os.path.join(CSRC, "probe_umma.cu")]
