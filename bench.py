@@ -334,11 +334,28 @@ def main():
         if ncomm is not comm:
             ab.abacus_nccl_comm_destroy(ncomm)
         # the same decisions with the combine inside the search kernel (peer mailboxes,
-        # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator)
-        pcomm = ab.peer_comm_from_process_group(ctx) if world > 1 else \
-            ab.abacus_peer_comm_init(ctx, 1, 0, [ab.abacus_peer_export(ctx)])
-        sharded_peer = sharded_decision_latency(ab, ctx, pcomm, world, rank, label="peer")
-        ab.abacus_peer_comm_destroy(pcomm)
+        # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator).
+        # Optional leg: every rank must agree that the communicator works (one probe
+        # decision) before the loop, or all of them skip it.
+        pcomm, err = None, None
+        try:
+            pcomm = ab.peer_comm_from_process_group(ctx) if world > 1 else \
+                ab.abacus_peer_comm_init(ctx, 1, 0, [ab.abacus_peer_export(ctx)])
+            qs, now, infl = synth.cfg3_decisions(1)[0]
+            ab.abacus_search_sharded(ctx, qs, now, infl, ab.ABACUS_SPACE_GRID, 2**40, pcomm)
+        except Exception as e:  # noqa: BLE001 -- report, do not fail the bench line
+            err = repr(e)
+        ok = err is None
+        if world > 1:
+            flag = torch.tensor([1 if ok else 0], dtype=torch.int32, device="cuda")
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+            ok = bool(flag.item())
+        if ok:
+            sharded_peer = sharded_decision_latency(ab, ctx, pcomm, world, rank, label="peer")
+        else:
+            sharded_peer = {"error": err or "the peer communicator failed on another rank"}
+        if pcomm:
+            ab.abacus_peer_comm_destroy(pcomm)
 
     # ---- per-decision latency (config 2, 3-way; 1 GPU each) -----------------
     dec = None
