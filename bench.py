@@ -366,8 +366,15 @@ def main():
     secondary = None
     whatif = None
     if world == 1 and not args.no_secondary:
-        whatif = whatif_sweep(ab, ctx, slots, H, T)
-        secondary = secondary_paths(ab, ctx, params, grid, H, T, args.precision, stream)
+        try:
+            whatif = whatif_sweep(ab, ctx, slots, H, T)
+        except Exception as e:  # noqa: BLE001 -- report, do not fail the bench line
+            whatif = {"error": repr(e)}
+        try:
+            secondary = secondary_paths(ab, ctx, params, grid, H, T, args.precision, stream)
+        except Exception as e:  # noqa: BLE001
+            secondary = {"error": repr(e)}
+            ab.abacus_load_predictor(ctx, params, PREC[args.precision])
 
     if rank == 0:
         pk, src = peaks()
