@@ -358,9 +358,19 @@ struct TcPipe {
             // layer 3 = hi + lo weights + bias chunk (0..4), output = hi weights (0, 1),
             // b4 added in fp32 when y is read
             if (TWO) {
+#ifndef EXP_NO_PRE
+                const uint64_t dbu = LAYER == 0 ? db2u : (LAYER == 1 ? db3u : db4u);
+                if (LAYER == 0)
+                    issue_pair_bf16_pre<ID, (CH >> 4), 3>(X.d, X.a, xa8, Y.d, Y.a, ya8, tCx, tCy, db, dbu, bar);
+                else if (LAYER == 1)
+                    issue_pair_bf16_pre<ID, (CH >> 4), 5>(X.d, X.a, xa8, Y.d, Y.a, ya8, tCx, tCy, db, dbu, bar);
+                else
+                    issue_pair2_pre<ID>(X.d, X.a, xa8, Y.d, Y.a, ya8, db, dbu, bar);
+#else
                 if (LAYER == 0) issue_layer2_asm<1, ID, CH, true, 4>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
                 else if (LAYER == 1) issue_layer2x5_asm<ID, CH>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
                 else issue_layer2_asm<1, ID, CH, false>(X.d, X.a, Y.d, Y.a, tCx, tCy, db, bar);
+#endif
             } else {
                 if (LAYER == 0) issue_layer_asm<1, ID, CH, true, 4, false>(X.d, X.a, tCx, db, bar);
                 else if (LAYER == 1) issue_layer_asm<1, ID, CH, true, 4, true>(X.d, X.a, tCx, db, bar);

@@ -340,6 +340,62 @@ __device__ __forceinline__ void issue_pair2_pre(uint32_t tDx, uint32_t tAx, uint
         : "memory");
 }
 
+// bf16 layer 2 / layer 3 for TWO tiles with the first two chunk descriptors and
+// the second A halves precomputed (issue_pair2_pre's bf16 counterparts):
+//   NCH 3: chunks 0, 1 and the bias chunk 4;  NCH 5: chunks 0..3 and the bias chunk 4
+template <uint32_t IDESC, uint32_t U, int NCH>
+__device__ __forceinline__ void issue_pair_bf16_pre(uint32_t tDx, uint32_t tAx, uint32_t tAx8, uint32_t tDy,
+                                                    uint32_t tAy, uint32_t tAy8, uint32_t tCx, uint32_t tCy,
+                                                    uint64_t d0, uint64_t d1, uint64_t* bar) {
+    if (NCH == 3) {
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d4;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d4, %8, %12;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %8, %11, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], %9, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%6], d4, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%4], %8, %11, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%5], %9, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%7], d4, %11, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%10];\n\t"
+            "}" ::"r"(tDx),
+            "r"(tAx), "r"(tAx8), "r"(tDy), "r"(tAy), "r"(tAy8), "r"(tCx), "r"(tCy), "l"(d0), "l"(d1),
+            "r"(smem_u32(bar)), "n"(IDESC), "n"((uint64_t)(4 * U))
+            : "memory");
+    } else {
+        asm volatile(
+            "{\n\t"
+            ".reg .pred e, pf, pt;\n\t"
+            ".reg .b64 d2, d3, d4;\n\t"
+            "setp.ne.b32 pf, 0, 0;\n\t"
+            "setp.eq.b32 pt, 0, 0;\n\t"
+            "add.s64 d2, %8, %12;\n\t"
+            "add.s64 d3, %9, %12;\n\t"
+            "add.s64 d4, %8, %13;\n\t"
+            "elect.sync _|e, 0xffffffff;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %8, %11, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], %9, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%2], d3, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%6], d4, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%4], %8, %11, pf;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%5], %9, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%4], d2, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%5], d3, %11, pt;\n\t"
+            "@e tcgen05.mma.cta_group::1.kind::f16 [%3], [%7], d4, %11, pt;\n\t"
+            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%10];\n\t"
+            "}" ::"r"(tDx),
+            "r"(tAx), "r"(tAx8), "r"(tDy), "r"(tAy), "r"(tAy8), "r"(tCx), "r"(tCy), "l"(d0), "l"(d1),
+            "r"(smem_u32(bar)), "n"(IDESC), "n"((uint64_t)(2 * U)), "n"((uint64_t)(4 * U))
+            : "memory");
+    }
+}
+
 // bf16 layer for TWO tiles: hi chunks 0, 1, lo chunks 2, 3 (W = W_hi + W_lo)
 // and (BIAS) the bias chunk 4, one commit
 template <uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
