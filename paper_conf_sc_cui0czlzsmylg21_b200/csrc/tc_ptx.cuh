@@ -191,30 +191,6 @@ __device__ __forceinline__ void issue_layer_asm(uint32_t tD, uint32_t tA, uint32
             : "memory");
         return;
     }
-    if (LO && !BIAS) {  // hi + lo weight chunks, no bias
-        asm volatile(
-            "{\n\t"
-            ".reg .pred e, pf, pt;\n\t"
-            ".reg .b64 d1, d2, d3;\n\t"
-            ".reg .b32 a8;\n\t"
-            "setp.ne.b32 pf, 0, 0;\n\t"
-            "setp.eq.b32 pt, 0, 0;\n\t"
-            "add.s64 d1, %2, %4;\n\t"
-            "add.s64 d2, %2, %5;\n\t"
-            "add.s64 d3, %2, %6;\n\t"
-            "add.u32 a8, %1, 8;\n\t"
-            "elect.sync _|e, 0xffffffff;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %7, pf;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d1, %7, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %7, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [a8], d3, %7, pt;\n\t"
-            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%3];\n\t"
-            "}" ::"r"(tD),
-            "r"(tA), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U), "n"((uint64_t)(2 * U)),
-            "n"((uint64_t)(3 * U)), "n"(IDESC)
-            : "memory");
-        return;
-    }
     if (!LO) {
         asm volatile(
             "{\n\t"
@@ -396,41 +372,12 @@ __device__ __forceinline__ void issue_pair_bf16_pre(uint32_t tDx, uint32_t tAx, 
     }
 }
 
-// bf16 layer for TWO tiles: hi chunks 0, 1, lo chunks 2, 3 (W = W_hi + W_lo)
-// and (BIAS) the bias chunk 4, one commit
-template <uint32_t IDESC, uint32_t CHUNK, bool BIAS = true>
+// bf16 layer 3 for TWO tiles: hi chunks 0, 1, lo chunks 2, 3 (W = W_hi + W_lo)
+// and the bias chunk 4, one commit
+template <uint32_t IDESC, uint32_t CHUNK>
 __device__ __forceinline__ void issue_layer2x5_asm(uint32_t tDx, uint32_t tAx, uint32_t tDy, uint32_t tAy,
                                                    uint32_t tCx, uint32_t tCy, uint64_t dbase, uint64_t* bar) {
     constexpr uint32_t U = CHUNK >> 4;
-    if (!BIAS) {
-        asm volatile(
-            "{\n\t"
-            ".reg .pred e, pf, pt;\n\t"
-            ".reg .b64 d1, d2, d3;\n\t"
-            ".reg .b32 ax8, ay8;\n\t"
-            "setp.ne.b32 pf, 0, 0;\n\t"
-            "setp.eq.b32 pt, 0, 0;\n\t"
-            "add.s64 d1, %4, %6;\n\t"
-            "add.s64 d2, %4, %7;\n\t"
-            "add.s64 d3, %4, %8;\n\t"
-            "add.u32 ax8, %1, 8;\n\t"
-            "add.u32 ay8, %3, 8;\n\t"
-            "elect.sync _|e, 0xffffffff;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %4, %9, pf;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d1, %9, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], d2, %9, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [ax8], d3, %9, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], %4, %9, pf;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d1, %9, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [%3], d2, %9, pt;\n\t"
-            "@e tcgen05.mma.cta_group::1.kind::f16 [%2], [ay8], d3, %9, pt;\n\t"
-            "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%5];\n\t"
-            "}" ::"r"(tDx),
-            "r"(tAx), "r"(tDy), "r"(tAy), "l"(dbase), "r"(smem_u32(bar)), "n"((uint64_t)U),
-            "n"((uint64_t)(2 * U)), "n"((uint64_t)(3 * U)), "n"(IDESC)
-            : "memory");
-        return;
-    }
     asm volatile(
         "{\n\t"
         ".reg .pred e, pf, pt;\n\t"
