@@ -230,10 +230,22 @@ def run_reference(args, rank, world):
             "cpu_baseline": {"value": rate, "unit": "candidates/s", "cores": ncores, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": rate, "unit": "candidates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line))
+    emit(line)
+
+
+_JSON_OUT = None
+
+
+def emit(line):
+    """The one contract line goes to the process's original stdout; everything
+    else printed at C level (NCCL's version banner, driver messages) was moved
+    to stderr by main()."""
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    print(json.dumps(line), file=out, flush=True)
 
 
 def main():
+    global _JSON_OUT
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -246,6 +258,9 @@ def main():
     ap.add_argument("--combine", default="nccl", choices=["nccl", "peer"],
                     help="N > 1 sweep combine: NCCL all-gather + finalize kernel, or inside the search kernel")
     args = ap.parse_args()
+    sys.stdout.flush()
+    _JSON_OUT = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -426,7 +441,7 @@ def main():
             "secondary_paths": secondary,
             "whatif": whatif,
         }
-        print(json.dumps(line), flush=True)
+        emit(line)
     if world > 1:
         # rank 0 ran the single-GPU latency and CPU legs alone: every rank tears
         # down the library's communicator together (ncclCommDestroy finalizes)
