@@ -170,12 +170,15 @@ def cpu_oracle_rate_all_cores(params, slots, H, budget_s=8.0, chunk=50_000):
     return n / dt, n, dt, ncores
 
 
-def arm_config(T, H, precision, world):
+def arm_config(T, H, precision, world, combine="nccl"):
     """The workload both arms report (the reference arm times a bounded sample of it)."""
+    how = ("NCCL all-gather of the per-rank results + finalize kernel" if combine == "nccl" else
+           "combine inside the search kernel over peer mailboxes")
     return {"workload": "cfg4: 4-way exhaustive overlap sweep (ResNet-152, Inception-v3, BERT-base "
                         "seq128, BERT-large seq512), %d candidates" % T,
             "candidates_per_step": T, "headroom_ms": H, "precision": precision,
-            "parallelism": "candidate shards x%d, NCCL all-gather of the best key" % world,
+            "parallelism": "candidate shards x%d" % world + (", " + how if world > 1 else ""),
+            "combine": combine if world > 1 else None,
             "l2": "no per-candidate memory traffic (candidates generated on chip)"}
 
 
@@ -273,10 +276,22 @@ def main():
     import torch.distributed as dist
     import paper_conf_sc_cui0czlzsmylg21_b200 as ab
 
+    # test mode (tests/test_gpu_bench_multirank.py): every rank on cuda:0, gloo for the
+    # torch.distributed plumbing, so the N > 1 path (shards, in-kernel peer combine,
+    # max-over-ranks timing, one line from rank 0) runs on a one-GPU box.  NCCL refuses
+    # two ranks on one GPU, so the NCCL legs are skipped there.  Never a bench number.
+    share = os.environ.get("ABACUS_BENCH_SHARE_GPU") == "1" and world > 1
+    if share:
+        if args.combine != "peer":
+            raise SystemExit("ABACUS_BENCH_SHARE_GPU=1 needs --combine peer (NCCL refuses two ranks on one GPU)")
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     params = synth.weights(1)
     slots = synth.cfg4_grid()
     H = synth.cfg4_headroom()
@@ -341,13 +356,16 @@ def main():
     sharded_peer = None
     if not args.no_decisions:
         # at N = 1 through a one-rank NCCL communicator: the sharded path as it runs at N > 1
-        if world > 1:
-            ncomm = comm if args.combine == "nccl" else ab.nccl_comm_from_process_group(ctx)
+        if share:
+            sharded = {"skipped": "ranks share one GPU (test mode): NCCL refuses that"}
         else:
-            ncomm = ab.abacus_nccl_comm_init(ctx, 1, 0, ab.abacus_nccl_unique_id())
-        sharded = sharded_decision_latency(ab, ctx, ncomm, world, rank)
-        if ncomm is not comm:
-            ab.abacus_nccl_comm_destroy(ncomm)
+            if world > 1:
+                ncomm = comm if args.combine == "nccl" else ab.nccl_comm_from_process_group(ctx)
+            else:
+                ncomm = ab.abacus_nccl_comm_init(ctx, 1, 0, ab.abacus_nccl_unique_id())
+            sharded = sharded_decision_latency(ab, ctx, ncomm, world, rank)
+            if ncomm is not comm:
+                ab.abacus_nccl_comm_destroy(ncomm)
         # the same decisions with the combine inside the search kernel (peer mailboxes,
         # CUDA IPC between the ranks' processes; at N = 1 a one-rank communicator).
         # Optional leg: every rank must agree that the communicator works (one probe
@@ -420,7 +438,7 @@ def main():
             "metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": elapsed / args.steps * 1e3, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[args.precision], "data": "synthetic",
-            "config": dict(arm_config(T, H, args.precision, world), combine=args.combine if world > 1 else None),
+            "config": dict(arm_config(T, H, args.precision, world, args.combine), shared_gpu_test_mode=share),
             "per_gpu": value / world,
             "selected": {"key": d.key, "index": d.index, "total_ops": d.total_ops, "pred_ms": d.pred_ms,
                          "end_op": list(d.end_op)},
