@@ -460,15 +460,18 @@ static __device__ __noinline__ void cta_publish_and_finish(const Plan& P, Scratc
     if (threadIdx.x == 0) {
         S->cta_key[blockIdx.x] = bk;
         S->cta_y[blockIdx.x] = by;
-        __threadfence();
-        const unsigned int ticket = atomicAdd(&S->counter, 1u);
+        // one acquire-release ticket instead of fence + atomic (+ a fence in the
+        // last CTA): the release publishes this CTA's record (and, through the
+        // CTA barrier above, y(0) stored by another thread); the last CTA's
+        // acquire, followed by the barrier below, orders its loads of every record
+        unsigned int ticket;
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(ticket) : "l"(&S->counter) : "memory");
         s_last = ticket == gridDim.x - 1;
     }
     }
     __syncthreads();
     trace_stamp(P, 5);
     if (!s_last) return;
-    __threadfence();
     trace_stamp(P, 8);
     if (threadIdx.x < 32) {
         // warp 0 reduces the per-CTA records (independent loads, then shuffles)
