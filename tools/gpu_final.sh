@@ -19,6 +19,12 @@ timeout 600 python tools/bench_kernels.py --out gpurun_out/${TAG}_kernels.json >
 for k in encode_grid24 select_kernel encode_groups24; do
   timeout 600 ncu --set full --clock-control none -k regex:$k -c 1 -o gpurun_out/${TAG}_$k python tools/bench_kernels.py --rows 16777216 --reps 1 > gpurun_out/${TAG}_ncu_$k.log 2>&1
 done
+# text summaries on the box; only the top kernel's report comes back whole (gpurun_out <= 64 MiB)
+for r in gpurun_out/${TAG}_*.ncu-rep; do
+  n=$(basename $r .ncu-rep)
+  python tools/ncu_summary.py $r > gpurun_out/${n}_ncu_summary.txt 2>&1
+  [ "$n" = "${TAG}_fused_fp16" ] || rm -f $r
+done
 timeout 900 python tests/accuracy_replay.py --out gpurun_out/${TAG}_cfg5_accuracy.json > gpurun_out/${TAG}_acc.log 2>&1
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err
 bash tools/gpu_sanitize.sh ${TAG}
