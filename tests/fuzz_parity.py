@@ -55,23 +55,23 @@ def rand_round(rng):
     return qs, now, float(rng.uniform(0, 5))
 
 
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--minutes", type=float, default=5.0)
-    ap.add_argument("--seed", type=int, default=1234)
-    a = ap.parse_args()
-    rng = np.random.default_rng(a.seed)
+def run(seed, minutes=None, iterations=None):
+    """Fuzz until the time or the iteration budget is spent (one iteration =
+    one precision: 4 grids, 8 rounds single + batched, one what-if set).
+    Returns (counts, failures)."""
+    rng = np.random.default_rng(seed)
     params = synth.weights(1)
     ctx = ab.abacus_create(0, list(synth.OPS_PER_MODEL))
     st = torch.cuda.Stream()
+    prev = torch.cuda.current_stream()
     torch.cuda.set_stream(st)
     ab.abacus_set_stream(ctx, st)
-    t_end = time.time() + a.minutes * 60
+    t_end = time.time() + (minutes if minutes is not None else 1e9) * 60
     n = {"grid": 0, "round": 0, "batch": 0, "whatif": 0}
     fails = 0
     precs = [ab.ABACUS_FP32, ab.ABACUS_FP16, ab.ABACUS_BF16]
     it = 0
-    while time.time() < t_end:
+    while time.time() < t_end and (iterations is None or it < iterations):
         prec = precs[it % 3]
         it += 1
         eps = EPS[prec]
@@ -141,6 +141,16 @@ def main():
                 fails += 1
                 print("FAIL whatif", prec, g, variants, H, flush=True)
     ab.abacus_destroy(ctx)
+    torch.cuda.set_stream(prev)
+    return n, fails
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--minutes", type=float, default=5.0)
+    ap.add_argument("--seed", type=int, default=1234)
+    a = ap.parse_args()
+    n, fails = run(a.seed, minutes=a.minutes)
     print("fuzz done:", n, "failures:", fails, flush=True)
 
 
