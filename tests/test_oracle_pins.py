@@ -323,6 +323,41 @@ def test_search_invariants():
         assert a1.space_used == 0 and a2.space_used == 1
 
 
+def test_fit_is_against_the_fp32_headroom():
+    """Reading c11: the fit test compares y with the fp32 headroom both sides
+    use, H = (float)h_c.  Constant predictor y = 1 exactly (unit 0 = bias 1,
+    passed through): h_c = 1 - 2^-30 rounds to H = 1.0 in fp32, so the
+    critical query fits (y <= H, inclusive); h_c = 1 - 2^-23 is an fp32 value
+    below 1, so it is dropped."""
+    d = 8 + 4 * 4
+    p = unit0_params(d, 1.0, {})
+    q = synth.Query(5, 1, 1, 0, 1.0 - 2.0 ** -30, 0.0)
+    r = oracle.search(p, [q], 0.0, 0.0, space=0)
+    assert r.h[0] == 1.0 - 2.0 ** -30 and r.headroom_ms == 1.0
+    assert r.pred_critical_only_ms == 1.0 and r.status == 0 and r.pred_ms == 1.0
+    q = synth.Query(5, 1, 1, 0, 1.0 - 2.0 ** -23, 0.0)
+    r = oracle.search(p, [q], 0.0, 0.0, space=0)
+    assert r.headroom_ms == 1.0 - 2.0 ** -23 and r.status == 1
+
+
+def test_acceptance_window_is_relative():
+    """Reading c18: the acceptance window is y <= H -/+ eps |H| (relative).
+    Constant predictor y = 16 exactly: with H = 16 (1 + eps/2) every candidate
+    fits but none fits the strict window, so maxkey_strict = 0 and
+    maxkey_loose = best_key = the brute-force maximum key; with
+    H = 16 (1 - eps/2) nothing fits, only the loose window holds every
+    candidate."""
+    d = 8 + 4 * 4
+    p = unit0_params(d, 16.0, {})
+    eps = 1e-2
+    for grid in synth.tiny_grids(6, seed=91, max_len=5):
+        top = max(((brute.sum_n(grid, o) + 1) << 40) | t for t, o in enumerate(brute.enumerate_grid(grid)))
+        r, _, _, _ = oracle.sweep(p, grid, 16.0 * (1 + eps / 2), eps=eps)
+        assert r.best_key == top and r.maxkey_loose == top and r.maxkey_strict == 0
+        r, _, _, _ = oracle.sweep(p, grid, 16.0 * (1 - eps / 2), eps=eps)
+        assert r.best_key == 0 and r.maxkey_strict == 0 and r.maxkey_loose == top
+
+
 # ------------------------------------------------------- multi-way search ---
 def test_fig12_multiway_two_predictions():
     """P:1349-1355: 3-way search -- first between queries, then among q1's ops;

@@ -75,3 +75,11 @@ def test_training_reduces_the_loss_and_beats_linear_regression():
     lr_mape = T.mape(np.hstack([Xte, np.ones((len(Xte), 1))]) @ coef, tte)
     mlp_mape = T.mape(T.forward(p, Xte, D)[0], tte)
     assert mlp_mape < 0.6 * lr_mape
+
+
+def test_mape_eq1_hand_values():
+    """Eq. 1 (P:1099-1104): error = |predicted - real| / real, averaged.
+    Hand values: (2 vs 1) -> 1, (3 vs 4) -> 1/4, (5 vs 5) -> 0; mean 5/12."""
+    assert T.mape([2.0], [1.0]) == 1.0
+    assert T.mape([3.0], [4.0]) == 0.25
+    assert abs(T.mape([2.0, 3.0, 5.0], [1.0, 4.0, 5.0]) - 5.0 / 12.0) < 1e-15
