@@ -111,6 +111,20 @@ MUTANTS = [
     ("what-if: first variant wins ties", PY, "if r.best_key and lift(r.best_key) > best[0]:",
      "if r.best_key and (lift(r.best_key) >> 40) > (best[0] >> 40):", None),
     ("brute: absent digit last instead of first", BR, None, None, None),
+    ("Eq.3: in-flight prediction subtracted from the first query only (c15)", C,
+     "h[i] = orc_headroom(q[i].qos_ms, q[i].t_start_ms, now_ms, inflight_ms);",
+     "h[i] = orc_headroom(q[i].qos_ms, q[i].t_start_ms, now_ms, i == 0 ? inflight_ms : 0.0);", 0),
+    ("bf16 emulation: layer-1 activations not rounded", C, "h1[i] = RA(s > 0.0 ? s : 0.0);",
+     "h1[i] = (s > 0.0 ? s : 0.0);", None),
+    ("bf16 emulation: biases rounded under the weight flag", C,
+     "#define RB(v) ((flags & 2) ?", "#define RB(v) ((flags & 1) ?", None),
+    ("encode_groups: unused slots kept", C, "if (groups[g * kmax + j].model_id != 0) s[n++]",
+     "if (groups[g * kmax + j].model_id >= 0) s[n++]", None),
+    ("sweep range: shard starts one index late", C, "if (st->counter >= st->first && st->counter < st->last) orc_visit(st);",
+     "if (st->counter > st->first && st->counter < st->last) orc_visit(st);", None),
+    ("CHAIN: block length without the +1", C, "int32_t R = j == 0 ? 1 : g[j].end_hi - g[j].start_op + 1;",
+     "int32_t R = j == 0 ? 1 : g[j].end_hi - g[j].start_op;", None),
+    ("m-way: never drops", C, "if (!fit[0]) {", "if (0 && !fit[0]) {", None),
 ]
 
 

@@ -455,8 +455,8 @@ def test_reading_r2_plain_bf16_misses_the_bar_on_config5():
 
 
 def test_bf16_emulation_against_torch_rounding():
-    """orc_mlp64_emu pinned beyond single rounding points: flags 1|2 (weights,
-    biases) and 4 (features) equal the plain fp64 MLP evaluated on operands
+    """orc_mlp64_emu pinned beyond single rounding points: flags 1 (weights),
+    2 (biases), 1|2 and 4 (features) equal the plain fp64 MLP evaluated on operands
     pre-rounded by torch's own fp32 -> bf16 conversion (RNE), bit for bit; with
     flag 8 (activations) a float64 numpy forward that rounds each post-ReLU
     activation through torch bf16 agrees to fp64 rounding noise."""
@@ -466,6 +466,16 @@ def test_bf16_emulation_against_torch_rounding():
     X = oracle.encode_groups(8, 4, [g.slots for g in G])
     pr = torch.from_numpy(params.astype(np.float32)).to(torch.bfloat16).float().numpy()
     assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=3), oracle.mlp64_batch(pr, X))
+    # flag 1 rounds the weights only, flag 2 the biases only
+    o = offsets(24)
+    bias = np.zeros(params.size, dtype=bool)
+    for name, n in (("b1", 32), ("b2", 32), ("b3", 32), ("b4", 1)):
+        bias[o[name]:o[name] + n] = True
+    pw = np.where(bias, params, pr).astype(np.float32)
+    pb = np.where(bias, pr, params).astype(np.float32)
+    assert not np.array_equal(pw, params) and not np.array_equal(pb, params)
+    assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=1), oracle.mlp64_batch(pw, X))
+    assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=2), oracle.mlp64_batch(pb, X))
     Xr = torch.from_numpy(X.astype(np.float32)).to(torch.bfloat16).float().numpy().astype(np.int16)
     assert not np.array_equal(Xr, X)  # some features (>= 256) do round
     assert np.array_equal(oracle.mlp64_emu_batch(params, X, flags=4), oracle.mlp64_batch(params, Xr))
