@@ -725,12 +725,7 @@ int decision_slots(abacus_ctx* c, const abacus_query_t* q, int32_t k, double now
 
 unsigned long long* trace_ptr();
 
-// sweep: a grid sweep call (abacus_search_grid, what-if variants launched one
-// by one); decisions pass false.  Sweeps over grids of >= 2^24 candidates take
-// the line path of the fp16 kernel (kernels_tc.cu); decisions, batches and
-// smaller grids keep the layer-1 MMA path, so every bit-identity between the
-// single, batched and what-if searches of the same grid holds as before.
-int launch_fused(abacus_ctx* c, Plan& P, bool sweep = false) {
+int launch_fused(abacus_ctx* c, Plan& P) {
     P.trace = trace_ptr();
     int grid = 0;
     cudaError_t e;
@@ -739,8 +734,7 @@ int launch_fused(abacus_ctx* c, Plan& P, bool sweep = false) {
         e = launch_fused_fp32(P, c->w234, c->d_w1b1, c->S, c->nsm, c->stream, &grid);
     } else {
         const int fmt = c->precision == ABACUS_FP16 ? 0 : 1;
-        const bool line = sweep && P.mode == kModeGrid && P.T >= (1ull << 24);
-        e = launch_fused_tc(P, c->tw[fmt], c->d_w1b1, c->S, c->nsm, c->stream, &grid, line);
+        e = launch_fused_tc(P, c->tw[fmt], c->d_w1b1, c->S, c->nsm, c->stream, &grid);
     }
     if (c->timed) cudaEventRecord(c->ev1, c->stream);
     if (e != cudaSuccess) return fail(c, ABACUS_E_CUDA, "fused search launch: %s", cudaGetErrorString(e));
@@ -1411,7 +1405,7 @@ int abacus_search_grid(abacus_ctx* c, const abacus_grid_t* grid, float headroom_
         P.peer = pc->d_comb;
         P.peer_seq = ++pc->seq;
     }
-    rc = launch_fused(c, P, true);
+    rc = launch_fused(c, P);
     if (rc) return rc;
     if (nccl_combine) {
         rc = combine_over_comm(c, nccl_comm, seq);
@@ -1594,7 +1588,7 @@ int abacus_search_whatif(abacus_ctx* c, const abacus_grid_t* grid, const abacus_
             Plan P = plan_grid_segments(c->n_models, c->D, &g, T, 0, T, headroom_ms);
             P.mapped = c->dev_result;
             P.seq = next_seq(c);
-            rc = launch_fused(c, P, true);
+            rc = launch_fused(c, P);
             if (rc) return rc;
             rc = wait_result(c, P.seq, &res[(size_t)v]);
             if (rc) return rc;

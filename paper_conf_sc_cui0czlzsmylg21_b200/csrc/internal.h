@@ -49,7 +49,7 @@ cudaError_t launch_mway(const Plan& P, const W234& W, const float* w1b1, int way
 cudaError_t launch_finalize_gather(Scratch* S, int nranks, MappedRec* mapped, uint32_t seq, cudaStream_t st);
 
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
-                            cudaStream_t st, int* grid_out, bool line = false);
+                            cudaStream_t st, int* grid_out);
 // batched decisions: d_decs[n_dec] and d_segs planned on the device, *d_n_pairs their tile-pair total
 // (pairs_ub >= it sizes the grid); acc/y0s zeroed / NaN-filled by the caller
 // NEXT-3: one Adam step on a minibatch (kernels_train.cu)

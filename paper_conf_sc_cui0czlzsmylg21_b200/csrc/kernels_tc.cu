@@ -790,584 +790,6 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
 }
 
 // ---------------------------------------------------------------------------
-// Line path of the fused fp16 search (the headline kernel since round 3).
-//
-// Layer 1 is affine in the box digits (the end ops enter the Fig.-8
-// vector linearly), so with the fastest digit v3 split off,
-//     W1 x(v) + b1 = base(line) + v3 w3,    line = (v0, v1, v2),
-//     base(line)   = c_s + v0 w0 + v1 w1 + v2 w2,
-// and a row's layer-1 activation is one packed f16 FMA per pair of hidden
-// units: h1 = relu(fma(v3, w3, base)) -- 16 HFMA2.RELU per row, no layer-1 MMA
-// round trip and no 16 KB TMEM read of an fp32 layer-1 accumulator per tile.
-// base is computed in fp32 from the fp32 W1 (then rounded to f16) for a window
-// of 128 consecutive lines at a time by the group's 128 threads (one line each)
-// into a shared-memory ring; a tile's rows touch <= 2 lines when cnt3 >= 128,
-// so the per-row loads are broadcasts.  The next tiles' layer-1 operand is
-// written while the current tiles' output MMA runs, into TMEM columns that MMA
-// does not touch (per-tile layout below), so after the output MMA completes
-// only the y read and the hand-off stand before the next tiles' layer-2 MMAs:
-// three MMA round trips per tile instead of four.
-//
-// Per tile 48 TMEM columns [T, T+48):
-//   layer 2:  A = h1   [T, T+16),    D [T+16, T+48)
-//   layer 3:  A        [T+32, T+48), D [T, T+32)
-//   output:   A        [T+32, T+48), D [T+16, T+24)   (N = 8)
-//   next h1 written to [T, T+16) while the output MMA runs (disjoint from both).
-// Lines: a segment's box ordinal u = line * cnt3 + v3; global line numbers run
-// over the plan's segments (LineSegInfo.lstart).  Rows past a segment's end get
-// sn = 0 (never folded); their line may be anything (the ring is indexed by
-// line & 127, every entry finite).
-// ---------------------------------------------------------------------------
-struct LineSegInfo {
-    uint32_t lstart;  // global line of the segment's first (shard) line
-    uint32_t lbeg;    // box line of the segment's first candidate (u_begin / cnt3)
-    uint32_t lmax;    // global line of the segment's last candidate
-    uint32_t cnt3, rem3, q3;  // 128 = q3 cnt3 + rem3 (one tile advance of the fastest digit)
-    uint32_t span;    // a tile's valid rows reach at most line(row 0) + span
-    uint32_t pad;
-};
-struct __align__(16) LineMeta {
-    unsigned long long idx;  // t_base + sum_{d<3} v_d istride_d (the key's index at v3 = 0)
-    uint32_t sn;             // n_base + 1 + v0 + v1 + v2 (the key's high part at v3 = 0)
-    uint32_t pad;
-};
-constexpr int kLineRing = 128;   // base entries (indexed line & 127)
-constexpr int kMetaRing = 512;   // meta entries (indexed line & 511; outlive one refill)
-constexpr int kLineSpanMax = 40; // host condition (line_plan_ok): a tile pair touches < 128 lines
-
-struct LineSmem {
-    uint32_t w2, w3, w4;  // weight chunks (blob layout, as tc_smem_layout<0>)
-    uint32_t stage;       // W1 | b1 fp32 staging
-    uint32_t vec;         // per segment: c, w0, w1, w2 (fp32, scaled), 4 x 32 floats
-    uint32_t w3h;         // per segment: w3 as 16 f16 pairs
-    uint32_t info;        // per segment LineSegInfo
-    uint32_t ring;        // per group: base ring (128 x 64 B) then meta ring (512 x 16 B)
-    uint32_t bars, tmem_slot, total;
-};
-constexpr uint32_t kLineGroupBytes = kLineRing * 64u + kMetaRing * 16u;
-
-__host__ __device__ inline LineSmem line_smem_layout(int D, int ng) {
-    LineSmem L{};
-    uint32_t o = 0;
-    L.w2 = o;
-    o += TcCfg<0>::kNchHid * kChunkBytesN32;
-    L.w3 = o;
-    o += TcCfg<0>::kNchHid * kChunkBytesN32;
-    L.w4 = o;
-    o += TcCfg<0>::kNchOut * kChunkBytesN16;
-    o = (o + 15u) & ~15u;
-    L.stage = o;
-    o += (uint32_t)(kHidden * D + kHidden) * 4u;
-    o = (o + 15u) & ~15u;
-    L.vec = o;
-    o += (uint32_t)kMaxSeg * 4u * kHidden * 4u;
-    L.w3h = o;
-    o += (uint32_t)kMaxSeg * 64u;
-    L.info = o;
-    o += (uint32_t)kMaxSeg * sizeof(LineSegInfo);
-    o = (o + 127u) & ~127u;
-    L.ring = o;
-    o += (uint32_t)ng * kLineGroupBytes;
-    L.bars = o;
-    o += 8u * (uint32_t)ng;
-    L.tmem_slot = o;
-    o += 16;
-    L.total = o;
-    return L;
-}
-
-// Per segment (prologue): the fp32 layer-1 vectors c_s, w0, w1, w2 and the f16
-// pairs of w3 (all times the layer-1 scale), from the staged W1 | b1 -- the
-// same terms build_b1_fused puts into its MMA tables (Fig.-8 positions,
-// P:859-866), here split into the line part and the fastest digit
-__device__ void build_line_vectors(const Plan& P, const float* __restrict__ w1b1, float scale, float* vec,
-                                   uint16_t* w3h, int t0, int nt) {
-    const int D = P.D;
-    const float* b1 = w1b1 + kHidden * D;
-    for (int e = t0; e < P.n_seg * kHidden; e += nt) {
-        const int s = e / kHidden, n = e % kHidden;
-        const SegP& g = P.seg[s];
-        const float* w = w1b1 + n * D;
-        float c = b1[n];
-        float wd[kKMax] = {0.0f, 0.0f, 0.0f, 0.0f};  // per box digit
-        for (int j = 0; j < kKMax; j++) {
-            if (j >= P.k || !((g.mask >> j) & 1u)) continue;
-            const SlotP& sl = P.slot[j];
-            const int f = P.n_models + 4 * g.pos[j];
-            c = fmaf(w[sl.model_id - 1], 1.0f, c);
-            c = fmaf(w[f + 0], (float)sl.ops, c);
-            c = fmaf(w[f + 1], (float)g.ope0[j], c);
-            c = fmaf(w[f + 2], (float)sl.bs, c);
-            c = fmaf(w[f + 3], (float)sl.seqlen, c);
-            wd[g.dpos[j]] = w[f + 1];
-        }
-        float* v = vec + s * 4 * kHidden;
-        v[n] = c * scale;
-        v[kHidden + n] = wd[0] * scale;
-        v[2 * kHidden + n] = wd[1] * scale;
-        v[3 * kHidden + n] = wd[2] * scale;
-        w3h[s * kHidden + n] = to16<0>(wd[3] * scale);
-    }
-}
-
-// one thread per segment: global line numbering of the plan (thread 0)
-__device__ void build_line_info(const Plan& P, LineSegInfo* info) {
-    uint32_t next = 0;
-    for (int s = 0; s < P.n_seg; s++) {
-        const SegP& g = P.seg[s];
-        LineSegInfo I{};
-        I.cnt3 = g.cnt[kKMax - 1];
-        I.q3 = (uint32_t)kTileM / I.cnt3;
-        I.rem3 = (uint32_t)kTileM - I.q3 * I.cnt3;
-        const uint64_t lb = div_rcp(g.u_begin, I.cnt3, g.rbstride[kKMax - 2]);
-        const uint64_t le = div_rcp(g.u_end - 1, I.cnt3, g.rbstride[kKMax - 2]);
-        I.lbeg = (uint32_t)lb;
-        I.lstart = next;
-        I.lmax = next + (uint32_t)(le - lb);
-        I.span = (I.cnt3 + (uint32_t)kTileM - 2u) / I.cnt3;
-        next = I.lmax + 1;
-        info[s] = I;
-    }
-}
-
-// Refill the group's window with lines [G0, G0 + 128): thread r computes line
-// G0 + r in fp32 and rounds its 32 base values to f16 pairs; then the group
-// synchronises (every thread of the group calls this with the same G0).
-__device__ __forceinline__ void line_refill(const Plan& P, const LineSegInfo* info, const float* vec,
-                                            uint8_t* ring, uint32_t G0, uint32_t r, uint32_t bar_id) {
-    const uint32_t G = G0 + r;
-    int s = 0;
-    for (int i = 1; i < P.n_seg; i++)
-        if (G >= info[i].lstart) s = i;
-    const LineSegInfo& I = info[s];
-    const SegP& sp = P.seg[s];
-    const uint32_t l = G - I.lstart + I.lbeg;  // box line (past the end for invalid rows: still finite)
-    const uint32_t c2 = sp.cnt[2], c1 = sp.cnt[1];
-    const uint32_t t = l / c2, v2 = l - t * c2;
-    const uint32_t v0 = t / c1, v1 = t - v0 * c1;
-    const float* c = vec + s * 4 * kHidden;
-    const float f0 = (float)v0, f1 = (float)v1, f2 = (float)v2;
-    uint32_t words[16];
-#pragma unroll
-    for (int i = 0; i < 16; i++) {
-        const int n = 2 * i;
-        float a = fmaf(f2, c[3 * kHidden + n], fmaf(f1, c[2 * kHidden + n], fmaf(f0, c[kHidden + n], c[n])));
-        float b = fmaf(f2, c[3 * kHidden + n + 1],
-                       fmaf(f1, c[2 * kHidden + n + 1], fmaf(f0, c[kHidden + n + 1], c[n + 1])));
-        words[i] = pack2<0>(a, b);
-    }
-    uint4* dst = reinterpret_cast<uint4*>(ring + (G & (kLineRing - 1)) * 64u);
-#pragma unroll
-    for (int i = 0; i < 4; i++) dst[i] = make_uint4(words[4 * i], words[4 * i + 1], words[4 * i + 2], words[4 * i + 3]);
-    LineMeta* meta = reinterpret_cast<LineMeta*>(ring + kLineRing * 64u);
-    LineMeta m;
-    m.idx = sp.t_base + (uint64_t)v0 * sp.istride[0] + (uint64_t)v1 * sp.istride[1] + (uint64_t)v2 * sp.istride[2];
-    m.sn = (uint32_t)(sp.n_base + 1) + v0 + v1 + v2;
-    m.pad = 0;
-    meta[G & (kMetaRing - 1)] = m;
-    named_bar_sync(bar_id, 128);
-}
-
-// per-row line walker: (G, v3) of this row, (g0, w0) of row 0 (uniform)
-struct LineWalker {
-    uint32_t G, v3;        // this row
-    uint32_t g0, w0;       // row 0 of the tile (uniform)
-    int32_t s;             // segment (uniform)
-    uint32_t tl;           // tiles of the segment left, the current one included (uniform)
-    uint32_t last_rows;    // valid rows of the segment's last tile (uniform)
-    uint32_t cnt3, rem3, q3, span, lmax;  // segment constants (uniform)
-
-    __device__ __forceinline__ void enter(const Plan& P, const LineSegInfo* info, int seg, uint64_t w, uint32_t r) {
-        const SegP& gs = P.seg[seg];
-        const LineSegInfo I = info[seg];
-        s = seg;
-        const uint64_t o = w - gs.tile0;
-        const uint64_t n = gs.u_end - gs.u_begin;
-        const uint64_t nt = (n + kTileM - 1) / kTileM;
-        tl = (uint32_t)(nt - o);
-        last_rows = (uint32_t)(n - (nt - 1) * kTileM);
-        cnt3 = I.cnt3;
-        rem3 = I.rem3;
-        q3 = I.q3;
-        span = I.span;
-        lmax = I.lmax;
-        const uint64_t ub = gs.u_begin + o * kTileM;
-        const uint64_t l0 = div_rcp(ub, cnt3, gs.rbstride[kKMax - 2]);
-        w0 = (uint32_t)(ub - l0 * cnt3);
-        g0 = I.lstart + (uint32_t)(l0 - I.lbeg);
-        const uint32_t x = w0 + r, q = x / cnt3;
-        v3 = x - q * cnt3;
-        G = g0 + q;
-    }
-    __device__ __forceinline__ void begin(const Plan& P, const LineSegInfo* info, uint64_t w, uint32_t r) {
-        enter(P, info, find_segment(P, w), w, r);
-    }
-    __device__ __forceinline__ void next(const Plan& P, const LineSegInfo* info, uint32_t r) {
-        if (tl == 1) {
-            enter(P, info, s + 1, P.seg[s + 1].tile0, r);
-            return;
-        }
-        tl--;
-        v3 += rem3;
-        G += q3;
-        if (v3 >= cnt3) { v3 -= cnt3; G++; }
-        w0 += rem3;
-        g0 += q3;
-        if (w0 >= cnt3) { w0 -= cnt3; g0++; }
-    }
-    __device__ __forceinline__ bool valid(uint32_t r) const { return !(tl == 1 && r >= last_rows); }
-    // the last line this tile's valid rows reach (uniform)
-    __device__ __forceinline__ uint32_t max_line() const { return min(g0 + span, lmax); }
-};
-
-// one row of a tile in flight: what the fold needs after the output MMA
-struct LineRow {
-    uint32_t G, v3, sn;
-    int32_t s;
-};
-
-template <int NG, class PL>
-__global__ void __launch_bounds__(NG * 128, 1) fused_line_kernel(const __grid_constant__ PL Pin,
-                                                                 const __grid_constant__ TcParams TP,
-                                                                 const float* __restrict__ w1b1, Scratch* S) {
-    const Plan& P = *reinterpret_cast<const Plan*>(&Pin);
-    extern __shared__ __align__(1024) uint8_t smem[];
-    const LineSmem L = line_smem_layout(P.D, NG);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + L.tmem_slot);
-    float* vec = reinterpret_cast<float*>(smem + L.vec);
-    const LineSegInfo* info = reinterpret_cast<const LineSegInfo*>(smem + L.info);
-
-    const int tid = threadIdx.x;
-    const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
-    const int g = warp >> 2, wq = warp & 3;
-    trace_stamp(P, 0);
-    if (tid == 0) {
-        for (int i = 0; i < NG; i++) mbar_init(&bars[i], 1);
-        mbar_fence_init();
-    }
-    if (warp == 0) {
-        tmem_alloc(tmem_slot, 512);
-        tmem_relinquish();
-    }
-    {
-        const int4* src = reinterpret_cast<const int4*>(TP.blob);
-        int4* dst = reinterpret_cast<int4*>(smem);
-        for (uint32_t i = tid; i < TP.bytes / 16; i += blockDim.x) dst[i] = src[i];
-        float* s_w1 = reinterpret_cast<float*>(smem + L.stage);
-        for (int i = tid; i < kHidden * P.D + kHidden; i += blockDim.x) s_w1[i] = __ldg(w1b1 + i);
-    }
-    __syncthreads();
-#ifdef LINE_BMMA
-    // hidden biases as a B chunk (row n: k0 = b_n) against the constant TMEM chunk
-    // (1, 1, 0, ...): the bias add runs on the tensor core, the epilogue ReLU is a
-    // max.f16x2 (ALU pipe) instead of an HFMA2 (FMA pipe)
-    {
-        uint16_t bh = 0;
-        const int lr = tid >> 5, n = tid & 31;
-        uint8_t* cb = smem + (lr ? L.w3 : L.w2) + 2u * kChunkBytesN32;
-        const int nl = LINE_BMMA == 1 ? 64 : 32;
-        if (tid < nl) bh = reinterpret_cast<const uint16_t*>(cb)[n];
-        __syncthreads();
-        if (tid < nl)
-            for (int k = 0; k < 16; k++) *reinterpret_cast<uint16_t*>(cb + b_offset(n, k)) = k == 0 ? bh : (uint16_t)0;
-    }
-#endif
-    build_line_vectors(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, vec,
-                       reinterpret_cast<uint16_t*>(smem + L.w3h), tid, blockDim.x);
-    if (tid == blockDim.x - 1) build_line_info(P, reinterpret_cast<LineSegInfo*>(smem + L.info));
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // weights -> tensor core
-    fence_before();
-    __syncthreads();
-    fence_after();
-    trace_stamp(P, 2);
-    const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
-
-    const uint32_t r = (uint32_t)(tid & 127);
-    const uint32_t lane_off = (uint32_t)(wq * 32) << 16;
-    const uint32_t X = tbase + (uint32_t)g * 96u, Y = X + 48u;
-#ifdef LINE_BMMA
-    const uint32_t tC = tbase + 480u;
-    if (g == 0) {
-        uint32_t c8[8] = {0x3C003C00u, 0, 0, 0, 0, 0, 0, 0};
-        tmem_st8(tC + lane_off, c8);
-        tmem_wait_st();
-    }
-    fence_before();
-    __syncthreads();
-    fence_after();
-#endif
-    const uint32_t sbase = smem_u32(smem);
-    uint64_t* bar = &bars[g];
-    const uint32_t bar_id = 1 + (uint32_t)g, ref_id = 8 + (uint32_t)g;
-    uint8_t* ring = smem + L.ring + (uint32_t)g * kLineGroupBytes;
-    const uint32_t ring_s = smem_u32(ring);
-    const LineMeta* meta = reinterpret_cast<const LineMeta*>(ring + kLineRing * 64u);
-    const uint32_t w3h_s = sbase + L.w3h;
-    uint64_t db2 = smem_desc(sbase + L.w2), db3 = smem_desc(sbase + L.w3), db4 = smem_desc(sbase + L.w4);
-    asm volatile("mov.b64 %0, %0;" : "+l"(db2));
-    asm volatile("mov.b64 %0, %0;" : "+l"(db3));
-    asm volatile("mov.b64 %0, %0;" : "+l"(db4));
-    const uint32_t hb2 = sbase + L.w2 + 2u * kChunkBytesN32;  // f16 bias pairs of layer 2 (layer 3's one blob later)
-    const uint32_t hb3 = hb2 + (uint32_t)TcCfg<0>::kNchHid * kChunkBytesN32;
-    const float b4 = TP.b4;
-    uint32_t ph = 0;
-    auto wait = [&]() {
-        mbar_wait(bar, ph);
-        ph ^= 1u;
-        fence_after();
-    };
-    auto handoff = [&](bool mine) {
-        fence_before();
-        if (mine) {
-            named_bar_sync(bar_id, 128);
-            fence_after();
-        } else {
-            named_bar_arrive(bar_id, 128);
-        }
-        return mine;
-    };
-    // hidden-layer epilogue: bias + ReLU on the f16 accumulators at D, A written at A
-    auto hidden = [&](auto two_c, uint32_t dofs, uint32_t hb) {
-        constexpr bool TWO = decltype(two_c)::value;
-#ifdef LINE_BMMA
-        if (LINE_BMMA == 1 || dofs == 16u) {
-        (void)hb;
-        wait();
-        uint32_t a[16], b[16];
-        if (TWO) tmem_ld16p_x2(X + dofs + lane_off, Y + dofs + lane_off, a, b);
-        else tmem_ld16p_x2(X + dofs + lane_off, X + dofs + lane_off, a, b);
-#pragma unroll
-        for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(a[c]) : "r"(0u));
-        tmem_st16(X + 32u + lane_off, a);
-        if (TWO) {
-#pragma unroll
-            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(b[c]) : "r"(0u));
-            tmem_st16(Y + 32u + lane_off, b);
-        }
-        } else {
-        uint32_t hbw[16];
-        lds_words16(hb, hbw);
-        wait();
-        uint32_t a[16], b[16];
-        if (TWO) tmem_ld16p_x2(X + dofs + lane_off, Y + dofs + lane_off, a, b);
-        else tmem_ld16p_x2(X + dofs + lane_off, X + dofs + lane_off, a, b);
-        const uint32_t one = 0x3C003C00u;
-#pragma unroll
-        for (int c = 0; c < 16; c++) asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(a[c]) : "r"(one), "r"(hbw[c]));
-        tmem_st16(X + 32u + lane_off, a);
-        if (TWO) {
-#pragma unroll
-            for (int c = 0; c < 16; c++)
-                asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(b[c]) : "r"(one), "r"(hbw[c]));
-            tmem_st16(Y + 32u + lane_off, b);
-        }
-        }
-#else
-        uint32_t hbw[16];
-        lds_words16(hb, hbw);
-        wait();
-        uint32_t a[16], b[16];
-        if (TWO) tmem_ld16p_x2(X + dofs + lane_off, Y + dofs + lane_off, a, b);
-        else tmem_ld16p_x2(X + dofs + lane_off, X + dofs + lane_off, a, b);
-        const uint32_t one = 0x3C003C00u;
-#pragma unroll
-        for (int c = 0; c < 16; c++) asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(a[c]) : "r"(one), "r"(hbw[c]));
-        tmem_st16(X + 32u + lane_off, a);
-        if (TWO) {
-#pragma unroll
-            for (int c = 0; c < 16; c++)
-                asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(b[c]) : "r"(one), "r"(hbw[c]));
-            tmem_st16(Y + 32u + lane_off, b);
-        }
-#endif
-        tmem_wait_st();
-    };
-    constexpr uint32_t ID32h = idesc_f16(0, 32, false);  // hidden layers: f16 accumulation
-    constexpr uint32_t ID8 = idesc_f16(0, 8, true);      // output: fp32
-    auto issue = [&](auto two_c, uint32_t dofs, uint32_t aofs, uint64_t db, auto id_c, auto ch_c) {
-        constexpr bool TWO = decltype(two_c)::value;
-        constexpr uint32_t ID = decltype(id_c)::value;
-        constexpr uint32_t CH = decltype(ch_c)::value;
-#ifdef LINE_BMMA
-        constexpr bool BIAS = CH == kChunkBytesN32;  // hidden layers: + the bias chunk
-        if (BIAS && (LINE_BMMA == 1 || aofs == 0u)) {
-            if (TWO) issue_layer2_asm<0, ID, CH, true, 2>(X + dofs, X + aofs, Y + dofs, Y + aofs, tC, tC, db, bar);
-            else issue_layer_asm<0, ID, CH, true, 2, false>(X + dofs, X + aofs, tC, db, bar);
-        } else {
-            if (TWO) issue_layer2_asm<0, ID, CH, false>(X + dofs, X + aofs, Y + dofs, Y + aofs, 0u, 0u, db, bar);
-            else issue_layer_asm<0, ID, CH, false>(X + dofs, X + aofs, 0u, db, bar);
-        }
-#else
-        if (TWO) issue_layer2_asm<0, ID, CH, false>(X + dofs, X + aofs, Y + dofs, Y + aofs, 0u, 0u, db, bar);
-        else issue_layer_asm<0, ID, CH, false>(X + dofs, X + aofs, 0u, db, bar);
-#endif
-    };
-    using IDh = std::integral_constant<uint32_t, ID32h>;
-    using ID8c = std::integral_constant<uint32_t, ID8>;
-    using CH32 = std::integral_constant<uint32_t, kChunkBytesN32>;
-    using CH16 = std::integral_constant<uint32_t, kChunkBytesN16>;
-    using T1 = std::integral_constant<bool, false>;
-    using T2 = std::integral_constant<bool, true>;
-
-    // issuer roles rotate with the group, so every SMSP issues stages of some groups
-    const bool me0 = ((g + 0) & 3) == wq, me1 = ((g + 1) & 3) == wq, me2 = ((g + 2) & 3) == wq;
-
-    unsigned long long best = 0;
-    float best_y = __int_as_float(0x7fc00000);
-    uint32_t bsn = 1u;
-    uint64_t wb, we;
-    work_range(P.n_tiles, (uint64_t)blockIdx.x * NG + g, (uint64_t)gridDim.x * NG, wb, we);
-    if (wb < we) {
-        LineWalker W;
-        W.begin(P, info, wb, r);
-        // the rows of a tile pair in flight (what the fold needs); two sets alternate
-        struct Rows {
-            uint32_t Gx, vx, snx, Gy, vy, sny;
-            int32_t sx, sy;
-        };
-        // layer-1 operand of one row: relu(fma(v3, w3, base(line))) -> TMEM [T, T+16)
-        auto h1 = [&](const uint32_t (&ww)[16], uint32_t T) {
-            uint32_t bw[16];
-            lds_words16(ring_s + (W.G & (kLineRing - 1)) * 64u, bw);
-            uint32_t v3h = 0x64006400u + W.v3 * 0x10001u;                 // (1024 + v3) twice, exact
-            asm("sub.rn.f16x2 %0, %0, %1;" : "+r"(v3h) : "r"(0x64006400u));  // (v3, v3)
-#pragma unroll
-            for (int c = 0; c < 16; c++)
-                asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(bw[c]) : "r"(v3h), "r"(ww[c]));
-            tmem_st16(T + lane_off, bw);
-            return W.valid(r) ? meta[W.G & (kMetaRing - 1)].sn + W.v3 : 0u;
-        };
-        // W is at tile X' of the pair; takes X' (and Y', advancing W)
-        auto take_pair = [&](auto ntwo_c, Rows& R) {
-            constexpr bool NTWO = decltype(ntwo_c)::value;
-            uint32_t ww[16];
-            lds_words16(w3h_s + (uint32_t)W.s * 64u, ww);
-            R.sx = W.s;
-            R.Gx = W.G;
-            R.vx = W.v3;
-            R.snx = h1(ww, X);
-            if (NTWO) {
-                const int32_t sx = W.s;
-                W.next(P, info, r);
-                if (W.s != sx) lds_words16(w3h_s + (uint32_t)W.s * 64u, ww);  // uniform, rare
-                R.sy = W.s;
-                R.Gy = W.G;
-                R.vy = W.v3;
-                R.sny = h1(ww, Y);
-            }
-        };
-        // the window must hold every valid line of the pair W (X') starts
-        uint32_t G0 = W.g0;
-        auto window = [&](bool two) {
-            uint32_t hi;
-            if (!two) hi = W.max_line();
-            else if (W.tl > 1) hi = min(W.g0 + W.q3 + 1u + W.span, W.lmax);
-            else hi = W.lmax + 1u + (uint32_t)kLineSpanMax;
-            if (hi >= G0 + (uint32_t)kLineRing) {  // uniform over the group
-                G0 = W.g0;
-                line_refill(P, info, vec, ring, G0, r, ref_id);
-            }
-        };
-        const bool yLive = wb + 1 < we;  // warp-uniform
-        Rows RA, RB;
-        RB.sx = RB.sy = 0;
-        RB.Gx = RB.vx = RB.snx = RB.Gy = RB.vy = RB.sny = 0u;
-        line_refill(P, info, vec, ring, G0, r, ref_id);
-        if (yLive) take_pair(T2{}, RA);
-        else take_pair(T1{}, RA);
-        tmem_wait_st();
-        if (handoff(me2)) {
-            if (yLive) issue(T2{}, 16u, 0u, db2, IDh{}, CH32{});
-            else issue(T1{}, 16u, 0u, db2, IDh{}, CH32{});
-        }
-        const uint32_t nw = (uint32_t)(we - wb);
-        uint32_t w = 0;
-        bool owe_y0 = wb == 0 && P.want_y0 && r == 0;
-        auto fold = [&](uint32_t G, uint32_t v3, uint32_t sn, int32_t s, float y) {
-            if (y <= P.H && sn >= bsn) {
-                const unsigned long long idx =
-                    meta[G & (kMetaRing - 1)].idx + (unsigned long long)v3 * P.seg[s].istride[kKMax - 1];
-                const unsigned long long key = ((unsigned long long)sn << 40) | idx;
-                if (key > best) {
-                    best = key;
-                    best_y = y;
-                    bsn = sn;
-                }
-            }
-        };
-        auto iteration = [&](auto two_c, auto next_two_c, Rows& cur, Rows& nxt) {
-            constexpr bool TWO = decltype(two_c)::value;
-            constexpr bool NTWO = decltype(next_two_c)::value;
-            // layer 2 -> layer 3
-            hidden(two_c, 16u, hb2);
-            if (handoff(me0)) issue(two_c, 0u, 32u, db3, IDh{}, CH32{});
-            // layer 3 -> output
-            hidden(two_c, 0u, hb3);
-            if (handoff(me1)) issue(two_c, 16u, 32u, db4, ID8c{}, CH16{});
-            // while the output MMA runs: the next pair's rows, window and layer-1 operand
-            const bool more = w + 2 < nw;  // warp-uniform
-            if (more) {
-                W.next(P, info, r);
-                window(NTWO);
-                take_pair(next_two_c, nxt);
-            }
-            wait();
-            uint32_t ybx, yby = 0;
-            if (TWO) tmem_ld1x2(X + 16u + lane_off, Y + 16u + lane_off, ybx, yby);
-            else tmem_ld1(X + 16u + lane_off, ybx);
-            if (more) {
-                tmem_wait_st();
-                if (handoff(me2)) {
-                    if (NTWO) issue(T2{}, 16u, 0u, db2, IDh{}, CH32{});
-                    else issue(T1{}, 16u, 0u, db2, IDh{}, CH32{});
-                }
-            }
-            const float yx = __uint_as_float(ybx) + b4;
-            if (owe_y0) {
-                S->y0 = yx;
-                owe_y0 = false;
-            }
-            const float yy = __uint_as_float(yby) + b4;
-            const bool cx = yx <= P.H && cur.snx >= bsn;
-            const bool cy = TWO && yy <= P.H && cur.sny >= bsn;
-            if (cx || cy) {
-                if (cx) fold(cur.Gx, cur.vx, cur.snx, cur.sx, yx);
-                if (cy) fold(cur.Gy, cur.vy, cur.sny, cur.sy, yy);
-            }
-            w += 2;
-        };
-        auto tail = [&](Rows& cur, Rows& nxt) {
-            if (w + 1 < nw) {
-                iteration(T2{}, T1{}, cur, nxt);
-                if (w < nw) iteration(T1{}, T1{}, nxt, cur);
-            } else if (w < nw) {
-                iteration(T1{}, T1{}, cur, nxt);
-            }
-        };
-        for (;;) {
-            if (!(w + 3 < nw)) {
-                tail(RA, RB);
-                break;
-            }
-            iteration(T2{}, T2{}, RA, RB);
-            if (!(w + 3 < nw)) {
-                tail(RB, RA);
-                break;
-            }
-            iteration(T2{}, T2{}, RB, RA);
-        }
-    }
-    trace_stamp(P, 3);
-    fence_before();
-    __syncthreads();
-    fence_after();
-    if (warp == 0) tmem_dealloc(tbase, 512);
-    trace_stamp(P, 4);
-    cta_publish_and_finish(P, S, best, best_y);
-}
-
-// ---------------------------------------------------------------------------
 // batched decisions (NEXT-4): one launch searches many independent decisions.
 // The launch's tile PAIRS are split contiguously over all groups; a group
 // walks its pairs decision by decision.  On entering a decision it copies the
@@ -2235,76 +1657,14 @@ static cudaError_t launch_fused_fmt(const Plan& P, const TcParams& tp, const flo
 // formats enter layer 1 through the same fp16 digit operand
 static bool need_split(int, uint32_t maxcnt) { return maxcnt > 1025; }
 
-// The line path needs every segment's tiles to touch few lines (a tile pair
-// fits the 128-line window), global line numbers below 2^31 and the fastest
-// digit exact in f16 (the !split condition).  ABACUS_LINE=0 disables it.
-bool line_plan_ok(const Plan& P) {
-    static const int s_env = [] {
-        const char* e = getenv("ABACUS_LINE");
-        return e ? atoi(e) : 1;
-    }();
-    if (!s_env) return false;
-    uint64_t lines = 0;
-    for (int s = 0; s < P.n_seg; s++) {
-        const SegP& g = P.seg[s];
-        const uint64_t c3 = g.cnt[kKMax - 1];
-        if (c3 == 0 || c3 > 1025) return false;
-        const uint64_t box_lines = g.bstride[0] * g.cnt[0] / c3;
-        if (box_lines >= (1ull << 31)) return false;
-        const uint64_t nl = (g.u_end - 1) / c3 - g.u_begin / c3 + 1;
-        uint64_t span = (c3 + kTileM - 2) / c3;
-        if (span > nl - 1) span = nl - 1;
-        if (span > (uint64_t)kLineSpanMax) return false;
-        lines += nl;
-    }
-    return lines < (1ull << 31);
-}
-
-static cudaError_t launch_line(const Plan& P, const TcParams& tp, const float* w1b1, Scratch* S, int nsm,
-                               cudaStream_t st, int* grid_out) {
-    const LineSmem L = line_smem_layout(P.D, kFusedNG);
-    uint64_t g = (P.n_tiles + kFusedNG - 1) / kFusedNG;
-    if (g > (uint64_t)nsm) g = (uint64_t)nsm;
-    if (g < 1) g = 1;
-    *grid_out = (int)g;
-    auto optin = [&](auto kern, int* granted) -> cudaError_t {
-        int dev = 0;
-        cudaError_t e = cudaGetDevice(&dev);
-        if (e != cudaSuccess) return e;
-        if (dev < 0 || dev >= 64 || granted[dev] < (int)L.total) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
-            if (e != cudaSuccess) return e;
-            if (dev >= 0 && dev < 64) granted[dev] = (int)L.total;
-        }
-        return cudaSuccess;
-    };
-    if (P.n_seg <= 8) {
-        static int s_granted8[64] = {};
-        auto kern = fused_line_kernel<kFusedNG, PlanDecision>;
-        const cudaError_t e = optin(kern, s_granted8);
-        if (e != cudaSuccess) return e;
-        PlanDecision Ps;
-        memcpy(&Ps, &P, sizeof(PlanDecision));
-        kern<<<(int)g, kFusedNG * 128, L.total, st>>>(Ps, tp, w1b1, S);
-        return cudaGetLastError();
-    }
-    static int s_granted[64] = {};
-    auto kern = fused_line_kernel<kFusedNG, Plan>;
-    const cudaError_t e = optin(kern, s_granted);
-    if (e != cudaSuccess) return e;
-    kern<<<(int)g, kFusedNG * 128, L.total, st>>>(P, tp, w1b1, S);
-    return cudaGetLastError();
-}
-
 cudaError_t launch_fused_tc(const Plan& P, const TcWeights& TW, const float* w1b1, Scratch* S, int nsm,
-                            cudaStream_t st, int* grid_out, bool line) {
+                            cudaStream_t st, int* grid_out) {
     TcParams tp{TW.blob, TW.bytes, TW.l1_scale, TW.b4};
     uint32_t maxcnt = 0;
     for (int s = 0; s < P.n_seg; s++)
         for (int j = 0; j < kKMax; j++) maxcnt = P.seg[s].cnt[j] > maxcnt ? P.seg[s].cnt[j] : maxcnt;
     const bool split = need_split(TW.fmt, maxcnt);
     if (TW.fmt == 0) {
-        if (!split && line && line_plan_ok(P)) return launch_line(P, tp, w1b1, S, nsm, st, grid_out);
         if (!split) return launch_fused_fmt<0, false>(P, tp, w1b1, S, nsm, st, grid_out);
         return launch_fused_fmt<0, true>(P, tp, w1b1, S, nsm, st, grid_out);
     }
