@@ -233,6 +233,24 @@ struct PackedWalkerT {
                 a2 += (uint32_t)kTileM << 16;
                 sn += kTileM;
             }
+            if (!GEN) {
+                // a carry out of v3 touches only some tiles of a warp's 32 consecutive
+                // rows (cnt3 >= 128: a fraction (159 / cnt3) of them, 34 % on config 4);
+                // the rest skip the carry chain with one vote (+1.6 % on config 4)
+                const bool c3 = a2 >= lim3;
+                if (__any_sync(0xffffffffu, c3)) {
+                    if (c3) { a2 -= dec3; sn -= dsn3; }
+                    const bool c2 = (a2 & 0xFFFFu) >= lim2;
+                    if (c2) { a2 -= cnt2; a1 += 0x10000u; sn -= dsn2; }
+                    const bool c1 = a1 >= lim1;
+                    if (c1) { a1 -= dec1; sn -= dsn1; }
+                }
+                // the segment's last tile (uniform, rare): rows past its end never fold
+                if (tl == 1 && last_rows < (uint32_t)kTileM) {
+                    if (r >= last_rows) sn = 0u;
+                }
+                return;
+            }
             const bool c3 = a2 >= lim3;  // v3 >= cnt3 (the low half never reaches bit 16)
             if (c3) { a2 -= dec3; sn -= dsn3; }  // v3 -= cnt3, v2 += 1
             const bool c2 = (a2 & 0xFFFFu) >= lim2;
