@@ -298,6 +298,49 @@ __device__ __forceinline__ void fold_packed(const Plan& P, int s, uint32_t a1, u
     }
 }
 
+// The headroom test on the output accumulator before its fp32 bias: with
+// y = fl(y_raw + b4) monotone in y_raw, {y_raw : fl(y_raw + b4) <= H} is
+// {y_raw <= T} for T = the largest float with fl(T + b4) <= H, so testing
+// y_raw <= T decides exactly what y <= H decides (and b4 is added only when a
+// row folds).  H = NaN keeps NaN (no row fits), H = +inf gives +inf.
+__host__ __device__ __forceinline__ float add_rn(float a, float b) {
+#ifdef __CUDA_ARCH__
+    return __fadd_rn(a, b);
+#else
+    volatile float r = a + b;  // one IEEE single rounding (no contraction)
+    return r;
+#endif
+}
+__host__ __device__ inline float raw_threshold(float H, float b4) {
+    if (!(H == H) || isinf(H)) return H;
+    float t = add_rn(H, -b4);
+    while (add_rn(t, b4) > H) t = nextafterf(t, -INFINITY);
+    for (;;) {
+        const float u = nextafterf(t, INFINITY);
+        if (isinf(u) || add_rn(u, b4) > H) break;
+        t = u;
+    }
+    return t;
+}
+
+// fold_packed2 on raw outputs (yr = y - b4 before rounding; Tr = raw_threshold)
+__device__ __forceinline__ void fold_packed2_raw(const Plan& P, float Tr, float b4, int sx, uint32_t x1, uint32_t x2,
+                                                 uint32_t xs, float yrx, int sy, uint32_t y1, uint32_t y2,
+                                                 uint32_t ys, float yry, unsigned long long& best, float& best_y,
+                                                 uint32_t& bsn) {
+    const bool cx = yrx <= Tr && xs >= bsn;
+    const bool cy = yry <= Tr && ys >= bsn;
+    if (cx || cy) {
+        if (cx) fold_packed(P, sx, x1, x2, xs, __fadd_rn(yrx, b4), best, best_y, bsn);
+        if (cy) fold_packed(P, sy, y1, y2, ys, __fadd_rn(yry, b4), best, best_y, bsn);
+    }
+}
+__device__ __forceinline__ void fold_packed_raw(const Plan& P, float Tr, float b4, int s, uint32_t a1, uint32_t a2,
+                                                uint32_t sn, float yr, unsigned long long& best, float& best_y,
+                                                uint32_t& bsn) {
+    if (yr <= Tr && sn >= bsn) fold_packed(P, s, a1, a2, sn, __fadd_rn(yr, b4), best, best_y, bsn);
+}
+
 // fold the two lock-step rows of a thread with one divergent branch: the cheap
 // tests of both rows first, the key construction only for a row that passes
 // (the key comparison inside is authoritative, so testing Y against the bsn

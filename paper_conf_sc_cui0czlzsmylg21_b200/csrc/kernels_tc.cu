@@ -639,7 +639,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             // only by the row that holds index 0 (the plan's first tile)
             const uint32_t nw = (uint32_t)(we - wb);
             uint32_t w = 0;
-            bool owe_y0 = wb == 0 && P.want_y0 && r == 0;
+            bool owe_y0 = wb == 0 && P.want_y0 && wq == 0;
+            const float Tr = raw_threshold(P.H, pp.b4);  // pp.outbias: b4 is added to y in fp32
             auto iteration = [&](auto two_c, auto next_two_c, Row& cx, Row& nx) {
                 constexpr bool TWO = decltype(two_c)::value;
                 constexpr bool NTWO = decltype(next_two_c)::value;
@@ -658,17 +659,17 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                 uint32_t ybx, yby = 0;
                 if (TWO) tmem_ld1x2(pp.X.d + pp.lane_off, pp.Y.d + pp.lane_off, ybx, yby);
                 else tmem_ld1(pp.X.d + pp.lane_off, ybx);
-                ybx = pp.add_b4(ybx);
-                if (TWO) yby = pp.add_b4(yby);
-                if (owe_y0) {
-                    S->y0 = __uint_as_float(ybx);
+                // raw outputs (before b4): the headroom test against Tr, b4 added on a fold
+                if (owe_y0) {  // warp-uniform (warp 0 of the group holding index 0)
+                    if (r == 0) S->y0 = __fadd_rn(__uint_as_float(ybx), pp.b4);
                     owe_y0 = false;
                 }
                 if (TWO)
-                    fold_packed2(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), sY, y1, y2, ys,
-                                 __uint_as_float(yby), best, best_y, bsn);
+                    fold_packed2_raw(P, Tr, pp.b4, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), sY, y1, y2, ys,
+                                     __uint_as_float(yby), best, best_y, bsn);
                 else
-                    fold_packed(P, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y, bsn);
+                    fold_packed_raw(P, Tr, pp.b4, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y,
+                                    bsn);
                 if (more) {
                     store_a1_packed(pp.X.a1 + pp.lane_off, nx.a1, nx.a2);
                     if (NTWO) takeY();
