@@ -27,7 +27,6 @@ for r in gpurun_out/${TAG}_*.ncu-rep; do
 done
 timeout 900 python tests/accuracy_replay.py --out gpurun_out/${TAG}_cfg5_accuracy.json > gpurun_out/${TAG}_acc.log 2>&1
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/${TAG}_ref.json 2> gpurun_out/${TAG}_ref.err
-bash tools/gpu_sanitize.sh ${TAG}
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/${TAG}_gputests.log 2>&1
 echo "pytest exit $?" >> gpurun_out/${TAG}_gputests.log
 cat gpurun_out/${TAG}_bench.json | cut -c1-400; tail -3 gpurun_out/${TAG}_bench.err; tail -2 gpurun_out/${TAG}_gputests.log
