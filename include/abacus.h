@@ -75,11 +75,13 @@ enum {
                      /* of exact features / digits (1024 + v).  Error vs the fp64  */
                      /* oracle on config 5: max 8.1e-3 relative (DESIGN.md r2)      */
     ABACUS_FP16 = 2  /* tcgen05 kind::f16, fp16 operands with exact power-of-two    */
-                     /* layer scaling; accumulation in TMEM is fp32 for layer 1 and */
-                     /* the output layer but F16 for hidden layers 2 and 3 (their   */
-                     /* biases are added in f16 in the epilogue); the output bias   */
-                     /* is added in fp32.  Error vs the fp64 oracle on config 5:    */
-                     /* max 1.5e-3 relative (reading r2)                  */
+                     /* layer scaling; accumulation in TMEM is fp32 for the output  */
+                     /* layer but F16 for hidden layers 2 and 3 (their biases are   */
+                     /* added in f16 in the epilogue) and, in the search calls, for */
+                     /* layer 1 (fp32 in abacus_predict_batch); the output bias is  */
+                     /* added in fp32.  Error vs the fp64 oracle: predict_batch on  */
+                     /* config 5 max 1.5e-3 relative, y(t*) of config-1 searches    */
+                     /* max 6.5e-4 (reading r2)                           */
 };
 
 /* candidate space of abacus_search (reading c13) */

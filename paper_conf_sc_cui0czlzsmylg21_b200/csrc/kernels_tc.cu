@@ -20,9 +20,11 @@
 // Numerics (reading r2, §4):
 //   fp16 (FMT 0): weights and activations fp16 RNE; layers are rescaled by
 //     exact powers of two so activations stay in fp16 range (ReLU is
-//     positively homogeneous, so the output is unchanged).  Layer 1 and the
-//     output accumulate in fp32, hidden layers 2-3 in f16 with their biases
-//     added in the f16 epilogue; b4 is added in fp32.
+//     positively homogeneous, so the output is unchanged).  The output
+//     accumulates in fp32, hidden layers 2-3 in f16 with their biases added in
+//     the f16 epilogue; b4 is added in fp32.  Layer 1 accumulates in f16 in the
+//     search kernels (true digits v against an uncompensated table) and in fp32
+//     in the standalone predict kernels (features as 1024 + v).
 //   bf16 (FMT 1): layer 1 as in fp16 (fp16 digit / feature operand, fp16
 //     table, fp32 accumulation), then bf16 activations; W2 and w4 bf16 (hi),
 //     W3 = W3_hi + W3_lo (both multiplied); hidden biases as a (hi, lo) pair
@@ -77,7 +79,7 @@ __device__ __forceinline__ void split16(float v, uint16_t& hi, uint16_t& lo) {
 // bf16 operands from layer 2 on).
 // c = b1 + W1 x0 (Fig.-8 vector of the segment's v = 0 group), w_j = the
 // W1 column of slot j's ope at its Fig.-8 position.
-template <int FMT, bool SPLIT>
+template <int FMT, bool SPLIT, bool TRUEV = false>
 __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, float scale, uint8_t* s_b1, int t0,
                                int nt) {
     constexpr int NCH = TcCfg<FMT>::kNchL1;
@@ -101,7 +103,7 @@ __device__ void build_b1_fused(const Plan& P, const float* __restrict__ w1b1, fl
             wj[g.dpos[j]] = w[f + 1] * scale;  // column of slot j's box digit
         }
         c *= scale;
-        if (FMT == 0 && !SPLIT) {  // digits enter as 1024 + v (store_a1): remove 1024 w_j as the MMA sees it
+        if (FMT == 0 && !SPLIT && !TRUEV) {  // digits enter as 1024 + v (store_a1): remove 1024 w_j as the MMA sees it
             for (int j = 0; j < kKMax; j++) c -= 1024.0f * from16<FMT>(to16<FMT>(wj[j]));
         }
         uint16_t ch, cl;
@@ -241,6 +243,10 @@ struct TcPipe {
 
     uint32_t hb_smem;  // fp16: shared address of layer 2's bias words (layer 3's follow one blob later)
     bool me[4];
+    // fp16 unsplit kernels: layer 1 accumulates in f16 from the true digits v
+    // (store_a1_true) against a table without the 1024 offset, so its epilogue is
+    // a packed 16-bit TMEM load and a max.f16x2 ReLU (the bias is in the MMA)
+    bool l1f16 = false;
     // fp16: the output layer runs without its bias K chunk and b4 is added to y
     // in fp32 when y is read (one MMA fewer per tile)
     bool outbias = false;
@@ -341,6 +347,11 @@ struct TcPipe {
     // operands from layer 2 on (its layer-1 epilogue packs bf16)
     __device__ __forceinline__ void issue_l1(const TileIO& T, uint64_t db) const {
         constexpr uint32_t id32 = idesc_f16(0, 32);
+        if (l1f16) {
+            constexpr uint32_t id16 = idesc_f16(0, 32, false);
+            mma_ts_elect(T.d, T.a1, db, id16, 0u);
+            return;
+        }
         mma_ts_elect(T.d, T.a1, db, id32, 0u);
     }
     __device__ __forceinline__ void commit() const { mma_commit_elect(bar); }
@@ -435,6 +446,22 @@ struct TcPipe {
                     asm("fma.rn.relu.f16x2 %0, %1, %2, %0;" : "+r"(b[c]) : "r"(one), "r"(hbw[c]));
                 tmem_st16(Y.a + lane_off, b);
             }
+        } else if (FMT == 0 && LAYER == 0 && TWO && l1f16) {
+            // f16 layer-1 accumulator (c and the digits' terms in one MMA): ReLU only
+            uint32_t a[16], b[16];
+            tmem_ld16p_x2(X.d + lane_off, Y.d + lane_off, a, b);
+#pragma unroll
+            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(a[c]) : "r"(0u));
+            tmem_st16(X.a + lane_off, a);
+#pragma unroll
+            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(b[c]) : "r"(0u));
+            tmem_st16(Y.a + lane_off, b);
+        } else if (FMT == 0 && LAYER == 0 && !TWO && l1f16) {
+            uint32_t a[16], b[16];
+            tmem_ld16p_x2(X.d + lane_off, X.d + lane_off, a, b);
+#pragma unroll
+            for (int c = 0; c < 16; c++) asm("max.f16x2 %0, %0, %1;" : "+r"(a[c]) : "r"(0u));
+            tmem_st16(X.a + lane_off, a);
         } else if (TWO) {
             uint32_t a[32], b[32], h[16];
             tmem_ld32x2(X.d + lane_off, Y.d + lane_off, a, b);
@@ -513,6 +540,16 @@ __device__ __forceinline__ uint32_t fused_prologue_tmem(uint64_t* bars, uint32_t
 }
 
 // layer-1 operand row (1, 1, 1024 + v0 .. 1024 + v3, 0, 0) of a packed tile row
+__device__ __forceinline__ void store_a1_packed_true(uint32_t taddr, uint32_t a1, uint32_t a2) {
+    // (1024 + v) - 1024 = v exactly in f16 (v < 1024)
+    asm volatile(
+        "{\n\t.reg .b32 t1, t2;\n\t"
+        "sub.rn.f16x2 t1, %1, %3;\n\t"
+        "sub.rn.f16x2 t2, %2, %3;\n\t"
+        "tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%4, t1, t2, %5};\n\t}" ::"r"(taddr),
+        "r"(a1), "r"(a2), "r"(0x64006400u), "r"(0x3C003C00u), "r"(0u)
+        : "memory");
+}
 __device__ __forceinline__ void store_a1_packed(uint32_t taddr, uint32_t a1, uint32_t a2) {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(0x3C003C00u),
                  "r"(a1), "r"(a2), "r"(0u)
@@ -557,7 +594,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     fence_after();
     trace_stamp(P, 1);
     const uint32_t tbase = __shfl_sync(0xffffffffu, *tmem_slot, 0);
-    build_b1_fused<0, SPLIT>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
+    constexpr bool kL1 = FMT == 0 && !SPLIT;  // layer 1 in f16 from the true digits (TcPipe::l1f16)
+    build_b1_fused<0, SPLIT, kL1>(P, reinterpret_cast<const float*>(smem + L.stage), TP.l1_scale, smem + L.b1, tid,
                                blockDim.x);
     if (g == 0) {  // the constant chunk (1, 1, 0, ...) of the bias rows
         uint32_t c8[8] = {TcCfg<FMT>::kOne2, 0, 0, 0, 0, 0, 0, 0};
@@ -576,6 +614,11 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
     pp.set_outbias(TP.b4);
     pp.zero_a();
+    pp.l1f16 = kL1;
+    auto st1 = [&](uint32_t taddr, uint32_t a1, uint32_t a2) {
+        if constexpr (kL1) store_a1_packed_true(taddr, a1, a2);
+        else store_a1_packed(taddr, a1, a2);
+    };
     const uint64_t d1base = smem_desc(sbase + L.b1);
     constexpr uint32_t kSegStep = C::kNchL1 * (kChunkBytesN32 >> 4);
 #ifndef EXP_NO_SEGLO
@@ -621,10 +664,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
             uint32_t y1 = 0, y2 = 0, ys = 0;  // Y row: a1, a2, sn
             int sY = 0;
             uint32_t bsn = 1u;
-            auto takeY = [&]() { y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s; store_a1_packed(pp.Y.a1 + pp.lane_off, W.a1, W.a2); };
+            auto takeY = [&]() { y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s; st1(pp.Y.a1 + pp.lane_off, W.a1, W.a2); };
             const bool yLive = wb + 1 < we;  // warp-uniform
             RA = Row{W.a1, W.a2, W.sn, W.s};
-            store_a1_packed(pp.X.a1 + pp.lane_off, RA.a1, RA.a2);
+            st1(pp.X.a1 + pp.lane_off, RA.a1, RA.a2);
             if (yLive) {
                 W.next(P, r);
                 takeY();
@@ -671,7 +714,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_tc_kernel(const __grid_cons
                     fold_packed_raw(P, Tr, pp.b4, cx.s, cx.a1, cx.a2, cx.sn, __uint_as_float(ybx), best, best_y,
                                     bsn);
                 if (more) {
-                    store_a1_packed(pp.X.a1 + pp.lane_off, nx.a1, nx.a2);
+                    st1(pp.X.a1 + pp.lane_off, nx.a1, nx.a2);
                     if (NTWO) takeY();
                     tmem_wait_st();
                     pp.stamp(3, 1);
@@ -869,6 +912,12 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
     pp.init(tbase, g, wq, &bars[g], smem_desc(sbase + L.w2), smem_desc(sbase + L.w3), smem_desc(sbase + L.w4));
     pp.set_outbias(TP.b4);
     pp.zero_a();
+    constexpr bool kL1 = FMT == 0 && !SPLIT;  // as fused_tc_kernel: layer 1 in f16 from the true digits
+    pp.l1f16 = kL1;
+    auto st1 = [&](uint32_t taddr, uint32_t a1, uint32_t a2) {
+        if constexpr (kL1) store_a1_packed_true(taddr, a1, a2);
+        else store_a1_packed(taddr, a1, a2);
+    };
     constexpr uint32_t kTable = C::kNchL1 * kChunkBytesN32;
     uint8_t* my_b1 = smem + L.b1 + (size_t)g * kMaxSegSlot * kTable;
     const uint64_t d1base = smem_desc(sbase + L.b1 + (uint32_t)g * kMaxSegSlot * kTable);
@@ -909,7 +958,7 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
             dec_pair0 = bd.pair0;
             dec_pair_end = d + 1 < n_dec ? decs[d + 1].pair0 : n_pairs;
             named_bar_sync(pp.bar_id, 128);
-            build_b1_fused<0, SPLIT>(P, s_w1, TP.l1_scale, my_b1, (int)r, 128);
+            build_b1_fused<0, SPLIT, kL1>(P, s_w1, TP.l1_scale, my_b1, (int)r, 128);
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             named_bar_sync(pp.bar_id, 128);
         };
@@ -941,10 +990,10 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
                 if (fresh) W.begin(P, lt, r);
                 else adv(lt);
                 x1 = W.a1; x2 = W.a2; xs = W.sn; sX = W.s; ltX = lt;
-                store_a1_packed(pp.X.a1 + pp.lane_off, W.a1, W.a2);
+                st1(pp.X.a1 + pp.lane_off, W.a1, W.a2);
                 adv(lt + 1);
                 y1 = W.a1; y2 = W.a2; ys = W.sn; sY = W.s;
-                store_a1_packed(pp.Y.a1 + pp.lane_off, W.a1, W.a2);
+                st1(pp.Y.a1 + pp.lane_off, W.a1, W.a2);
                 tmem_wait_st();
                 if (pp.handoff(wq == 3)) {
                     issue_l1(pp.X, sX);
@@ -987,8 +1036,8 @@ __global__ void __launch_bounds__(NG * 128, 1) fused_batch_tc_kernel(const Batch
                 if (same) {
                     x1 = n1; x2 = n2; xs = ns; sX = nsX;
                     y1 = m1; y2 = m2; ys = ms; sY = nsY;
-                    store_a1_packed(pp.X.a1 + pp.lane_off, x1, x2);
-                    store_a1_packed(pp.Y.a1 + pp.lane_off, y1, y2);
+                    st1(pp.X.a1 + pp.lane_off, x1, x2);
+                    st1(pp.Y.a1 + pp.lane_off, y1, y2);
                     tmem_wait_st();
                     if (pp.handoff(wq == 3)) {
                         issue_l1(pp.X, sX);
