@@ -36,7 +36,7 @@ import synth  # noqa: E402
 FLOP_PER_CAND = 2 * (synth.D * 32 + 32 * 32 + 32 * 32 + 32)  # 5,696 algorithmic FLOP (D = 24)
 METRIC = "predictor candidates/sec (config 4 exhaustive overlap sweep, abacus_search_grid)"
 PREC = {"fp32": 0, "bf16": 1, "fp16": 2}
-DTYPE = {"fp32": "f32", "bf16": "bf16 (layers 2, 3, output bf16 operands, W3 hi+lo; layer-1 digit operand f16), f32 accum", "fp16": "f16 (layers 1 + output: f32 accum; layers 2-3: f16 accum)"}
+DTYPE = {"fp32": "f32", "bf16": "bf16 (layers 2, 3, output bf16 operands, W3 hi+lo; layer-1 digit operand f16), f32 accum", "fp16": "f16 (layers 1-3: f16 accum; output: f32 accum)"}
 
 
 def peaks():
