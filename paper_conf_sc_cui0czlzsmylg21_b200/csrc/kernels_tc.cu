@@ -342,9 +342,11 @@ struct TcPipe {
         fence_after();
     }
     // layer-1 MMA of one tile against its segment's B operand (no commit).  Both
-    // formats: fp16 operands (the digits enter as the exact fp16 1024 + v, the
-    // segment table is fp16, fp32 accumulation); the bf16 path switches to bf16
-    // operands from layer 2 on (its layer-1 epilogue packs bf16)
+    // formats: fp16 operands and an fp16 segment table; the fp16 search kernels
+    // (l1f16) store the true digits v and accumulate in f16, the bf16 path the
+    // digits as the exact fp16 1024 + v against a compensated table with fp32
+    // accumulation, then bf16 operands from layer 2 on (its layer-1 epilogue
+    // packs bf16)
     __device__ __forceinline__ void issue_l1(const TileIO& T, uint64_t db) const {
         constexpr uint32_t id32 = idesc_f16(0, 32);
         if (l1f16) {
@@ -360,8 +362,7 @@ struct TcPipe {
     __device__ __forceinline__ void issue_next() const {
         constexpr uint32_t CH = LAYER == 2 ? kChunkBytesN16 : kChunkBytesN32;
         // fp16: hidden layers 2 and 3 accumulate in f16 (their epilogues then read
-        // half the TMEM bytes); layer 1 (the 1024 + v digits cancel there) and
-        // the output layer accumulate in fp32
+        // half the TMEM bytes), the output layer in fp32 (layer 1: issue_l1)
         constexpr uint32_t ID = idesc_f16(FMT, LAYER == 2 ? 8 : 32, FMT != 0 || LAYER == 2);
         const uint64_t db = LAYER == 0 ? db2 : (LAYER == 1 ? db3 : db4);
         if (FMT == 1) {
@@ -539,7 +540,8 @@ __device__ __forceinline__ uint32_t fused_prologue_tmem(uint64_t* bars, uint32_t
     return tbase;
 }
 
-// layer-1 operand row (1, 1, 1024 + v0 .. 1024 + v3, 0, 0) of a packed tile row
+// layer-1 operand row (1, 1, v0 .. v3, 0, 0) of a packed tile row (the fp16
+// search kernels: f16 layer-1 accumulation, uncompensated table)
 __device__ __forceinline__ void store_a1_packed_true(uint32_t taddr, uint32_t a1, uint32_t a2) {
     // (1024 + v) - 1024 = v exactly in f16 (v < 1024)
     asm volatile(
@@ -550,6 +552,8 @@ __device__ __forceinline__ void store_a1_packed_true(uint32_t taddr, uint32_t a1
         "r"(a1), "r"(a2), "r"(0x64006400u), "r"(0x3C003C00u), "r"(0u)
         : "memory");
 }
+// layer-1 operand row (1, 1, 1024 + v0 .. 1024 + v3, 0, 0) of a packed tile row
+// (the bf16 path: fp32 layer-1 accumulation, compensated table)
 __device__ __forceinline__ void store_a1_packed(uint32_t taddr, uint32_t a1, uint32_t a2) {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "r"(0x3C003C00u),
                  "r"(a1), "r"(a2), "r"(0u)
