@@ -1,4 +1,4 @@
-# A/B of exp/*.so variants (ABACUS_LINE as set per entry "name:LINE"), default bench, N reps
+# A/B of exp/*.so variants, default bench, REPS rounds; entries "name:X" (X ignored: the line-path switch of an earlier experiment)
 cd /root/repo
 python -c "import oracle; oracle.build()" >/dev/null 2>&1
 L=paper_conf_sc_cui0czlzsmylg21_b200/libabacus.so
