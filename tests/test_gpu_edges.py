@@ -154,3 +154,30 @@ def test_long_models_split_digits(prec):
             assert max(keys) == full.key
     finally:
         c.close()
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_digit_range_boundary_1025(prec):
+    """The largest unsplit digit range: a slot with exactly 1,025 end-op options
+    (digits 0..1024, the fp16 operand 1024 + v reaches 2048; the fp16 search
+    kernels convert it to the true digit v = 1024 exactly) and one with 1,024,
+    each beside a short slot, full sweeps and shards against the oracle; the
+    1,026-option range (split operand) beside it."""
+    ops = list(synth.OPS_PER_MODEL)
+    ops[0] = 1500
+    c = Ctx(ops=ops, params=synth.weights(1), precision=prec)
+    rng = np.random.default_rng(44)
+    try:
+        for n_opts in (1024, 1025, 1026):
+            lo = int(rng.integers(2, 400))
+            slots = [synth.GridSlot(1, 1, 8, 0, lo, lo + n_opts - 1, 0),
+                     synth.GridSlot(5, 1, 4, 0, 1, int(rng.integers(20, 40)), 1)]
+            T = oracle.grid_size(slots)
+            _, y64, _, _ = oracle.sweep(c.params, slots, 0.0, want_y=True)
+            for q in (0.2, 0.8):
+                H = float(np.float32(np.quantile(y64, q)))
+                full = _check_sweep(c, slots, H)
+                keys = [_check_sweep(c, slots, H, *ab.shard_range(T, r, 2)).key for r in range(2)]
+                assert max(keys) == full.key
+    finally:
+        c.close()
