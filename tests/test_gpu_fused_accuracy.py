@@ -40,3 +40,33 @@ def test_selected_y_against_oracle(prec):
             assert e.max() <= 0.5 * EPS[prec], (NAMES[prec], e.max())
     finally:
         c.close()
+
+
+@pytest.mark.parametrize("prec", [ab.ABACUS_FP32, ab.ABACUS_FP16, ab.ABACUS_BF16])
+def test_headroom_boundary_is_inclusive(prec):
+    """The fit test is y <= H with H inclusive (reading c11), decided in the tensor
+    kernels on the raw output accumulator (y_raw <= T): a search at H = y*, the
+    prediction of the group a first search selected, selects the same group, and
+    a search at the next float below y* selects a smaller key (that group no
+    longer fits)."""
+    params = synth.weights(1)
+    rng = np.random.default_rng(33)
+    c = Ctx(params=params, precision=prec)
+    try:
+        for b, slots in synth.cfg1_grids():
+            _, y64, _, _ = oracle.sweep(params, slots, 0.0, want_y=True)
+            g = ab.make_grid(slots)
+            T = len(y64)
+            for _ in range(8):
+                H1 = float(np.float32(np.quantile(y64, rng.uniform(0.05, 0.95))))
+                d1 = ab.abacus_search_grid(c.h, g, H1, 0, T)
+                assert d1.key != 0
+                ystar = float(np.float32(d1.pred_ms))
+                d2 = ab.abacus_search_grid(c.h, g, ystar, 0, T)
+                assert d2.key == d1.key and d2.pred_ms == d1.pred_ms, (NAMES[prec], H1, ystar)
+                below = float(np.nextafter(np.float32(ystar), np.float32(-np.inf)))
+                d3 = ab.abacus_search_grid(c.h, g, below, 0, T)
+                assert d3.key < d1.key, (NAMES[prec], ystar, below)
+                assert d3.key == 0 or d3.pred_ms <= below
+    finally:
+        c.close()
